@@ -1,0 +1,360 @@
+#!/usr/bin/env python3
+"""Benchmark of the B200 Tigr hot path (driver contract: one JSON line on rank 0).
+
+Workload (BASELINE.json configs[3]): R-MAT scale 24 (16,777,216 vertices,
+268,435,456 arcs, Graph500 a/b/c), PageRank 20 iterations, degree bound K = 8, strided
+(coalesced) layout.  One step = the whole hot path over the arc list resident in HBM:
+CSR build (a1) -> virtual split + layout (a2-a5) -> init + 20 x (relax -> [all-reduce] ->
+apply) (a6-a10).  value = 20 * m / step time (GTEPS, input-normalised; every arc is
+processed every iteration).  The other configs are parity-test cases (tests/).
+
+  python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--config cfg4]
+Multi-GPU: torchrun --nproc-per-node N bench.py --gpus N ...  (vnode ranges, NCCL all-reduce).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+# Algorithmic bytes of the push relax (fixed before measurement; DESIGN.md
+# "Roofline"): per processed arc s_e + s_v (read the target value) -- PageRank: s_e + 2 s_v
+# (RED = read + write of acc[dst]); per virtual node 4 (vn_phys); per node with d > 0 the
+# source value + its row_ptr pair (s_v + 8).
+S_E = 4
+
+
+def relax_bytes_pr(m, nv, n_out):
+    return m * (S_E + 16) + nv * 4 + n_out * (8 + 8)
+
+
+def pr_apply_bytes(n):
+    return n * 28
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="tigr", choices=["tigr", "reference"])
+    ap.add_argument("--config", default="cfg4")
+    ap.add_argument("--K", type=int, default=8)
+    ap.add_argument("--layout", default="strided", choices=["strided", "consecutive"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-extra", action="store_true", help="skip the per-algorithm extras")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras, no e2e)")
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.rows, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except OSError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+        sms = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------------------------------------ reference arm
+def cpu_pr_sample(rec, iters, threads_note=True):
+    """The oracle as it stands (single-threaded C power iteration) on the same workload:
+    host generator -> oracle CSR (untimed) -> `iters` PageRank iterations (timed)."""
+    import graphgen
+    import oracle
+
+    src, dst, _ = graphgen.generate(rec, weighted=False)
+    g = oracle.csr_build(rec.n, src, dst)
+    del src, dst
+    t0 = time.perf_counter()
+    oracle.pagerank(g, iters)
+    dt = time.perf_counter() - t0
+    return dt, g
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle timed on the box's host cores (rank 0 only)."""
+    import graphgen
+    import oracle
+
+    if rank != 0:
+        return
+    rec = graphgen.recipe(args.config)
+    src, dst, _ = graphgen.generate(rec, weighted=False)
+    g = oracle.csr_build(rec.n, src, dst)
+    del src, dst
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.pagerank(g, 1)  # one power iteration per step: a bounded sample of the 20-iteration run
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+    t = sum(times) / len(times)
+    val = rec.m / t / 1e9
+    print(json.dumps({
+        "impl": "reference", "metric": metric_name(args), "value": val, "unit": "GTEPS", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_obj(args, rec),
+        "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                         "sample": "1 of the 20 PageRank iterations per step on the full cfg4 graph "
+                                   "(oracle/oracle.c or_pagerank, single thread)"},
+        "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def metric_name(args):
+    return "GTEPS per algorithm at 1/2/4/8 B200; % of HBM roofline; vs CPU oracle"
+
+
+def config_obj(args, rec):
+    return {"workload": f"{args.config}: R-MAT n={rec.n:,} m={rec.m:,} (a,b,c)=({rec.a},{rec.b},{rec.c}) "
+                        f"PageRank 20 iterations, K={args.K}, {args.layout} layout",
+            "algorithm": "pagerank", "K": args.K, "layout": args.layout, "n": rec.n, "m": rec.m,
+            "parallelism": "vnode-range data parallel + NCCL all-reduce" if args.gpus > 1 else "single GPU",
+            "l2": "flushed between steps (512 MiB write outside the timed events); arc list 2.1 GB > L2"}
+
+
+# ------------------------------------------------------------------------------------------ main arm
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import graphgen
+    import paper_conf_asplos_sabetq018_b200 as tigr
+
+    torch.cuda.set_device(local)
+    comm = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        uid = [tigr.tigr_comm_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        comm = tigr.tigr_comm_init(world, rank, uid[0])
+
+    rec = graphgen.recipe(args.config)
+    n, m = rec.n, rec.m
+    s = torch.cuda.current_stream()
+    # inputs resident in HBM: the arc list, drawn on the device (counter-based; identical on every rank)
+    src = torch.empty(m, dtype=torch.int32, device="cuda")
+    dst = torch.empty_like(src)
+    tigr.tigr_rmat_coo(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, src, dst, None, stream=s)
+    out = torch.empty(n, dtype=torch.float64, device="cuda")
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
+    opts = tigr.tigr_run_opts_default()
+    opts.stream = s.cuda_stream
+    opts.time_kernels = 1
+    if comm is not None:
+        opts.comm = comm.ptr.value
+
+    def one_step(src_t, dst_t, out_t, host=False):
+        """a1 CSR build -> a2-a5 virtualize -> a6-a10 PageRank; returns per-phase events."""
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
+        ev[0].record(s)
+        g = tigr.tigr_graph_from_coo(n, src_t, dst_t, None, stream=s)
+        ev[1].record(s)
+        vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+        if comm is not None:
+            tigr.tigr_vgraph_partition(vg, world, rank)
+        ev[2].record(s)
+        _, st = tigr.tigr_run(vg, "pr", 0, opts=opts, out=out_t, return_stats=True)
+        ev[3].record(s)
+        nv = vg.info()["nv"]
+        vg.free()
+        g.free()
+        return ev, st, nv
+
+    # warm-up (W >= 3 by contract)
+    for _ in range(max(args.warmup, 0)):
+        one_step(src, dst, out)
+    torch.cuda.synchronize()
+
+    deg_t = torch.bincount(src, minlength=n)
+    n_out = int(torch.count_nonzero(deg_t).item())
+    clocks = ClockSampler(local)
+    clocks.start()
+    l0 = tigr.tigr_launch_count()
+    step_ms, phase, relax_ms, relax_launches, nv = [], [[], [], []], 0.0, 0, 0
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    for _ in range(args.steps):
+        flush.fill_(1)  # L2 flush outside the timed events
+        ev, st, nv = one_step(src, dst, out)
+        torch.cuda.synchronize()
+        step_ms.append(ev[0].elapsed_time(ev[3]))
+        for i in range(3):
+            phase[i].append(ev[i].elapsed_time(ev[i + 1]))
+        relax_ms += st["ms_relax"]
+        relax_launches += st["relax_launches"]
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = tigr.tigr_launch_count() - l0
+    clk = clocks.stop()
+
+    t_step = sum(step_ms) / len(step_ms)
+    if world > 1:
+        tt = torch.tensor([t_step], dtype=torch.float64, device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        t_step = float(tt.item())
+    gteps = 20 * m / (t_step * 1e-3) / 1e9
+
+    # roofline of the dominant kernel (PR relax), live CUDA-event durations from the timed region
+    relax_avg_ms = relax_ms / max(relax_launches, 1)
+    my_nv = nv
+    bytes_launch = relax_bytes_pr(m // world if world > 1 else m, my_nv, n_out // world if world > 1 else n_out)
+    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(peaks_path):
+        peak = json.load(open(peaks_path))["hbm_gbs"]
+        peak_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)"
+    else:
+        peak, peak_src = 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+    achieved = bytes_launch / (relax_avg_ms * 1e-3) / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "relax_pr_traffic.json")
+    if os.path.exists(tpath):
+        traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
+
+    result = {
+        "metric": metric_name(args), "value": gteps, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t_step, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_obj(args, rec),
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": traffic, "kernel": "k_relax_pr (PageRank push relax)",
+                     "algorithmic_bytes_per_launch": bytes_launch, "avg_launch_ms": relax_avg_ms,
+                     "peak_source": peak_src},
+        "breakdown_ms": {"csr_build": statistics.mean(phase[0]), "virtualize": statistics.mean(phase[1]),
+                         "pagerank_20it": statistics.mean(phase[2]), "relax_total": relax_ms / args.steps},
+        "algo_gteps": 20 * m / (statistics.mean(phase[2]) * 1e-3) / 1e9,
+        "nv": my_nv, "gpu_launches": launches, "clocks": clk,
+    }
+
+    # e2e through the public API with HOST buffers (pinned), H2D and D2H inside the timed region
+    if not args.no_e2e and not args.profile:
+        hsrc = src.cpu().pin_memory()
+        hdst = dst.cpu().pin_memory()
+        hout = torch.empty(n, dtype=torch.float64).pin_memory()
+        e2e = []
+        for _ in range(max(1, min(args.steps, 5))):
+            flush.fill_(1)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            one_step(hsrc, hdst, hout)
+            e1.record(s)
+            torch.cuda.synchronize()
+            e2e.append(e0.elapsed_time(e1))
+        te = sum(e2e) / len(e2e)
+        if world > 1:
+            tt = torch.tensor([te], dtype=torch.float64, device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            te = float(tt.item())
+        result["e2e"] = {"value": 20 * m / (te * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": te,
+                         "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8}
+
+    if not args.no_extra and not args.profile and world == 1:
+        result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy())
+
+    if rank == 0 and world == 1 and not args.no_cpu and not args.profile:
+        dt, _ = cpu_pr_sample(rec, 2)
+        v = 2 * m / dt / 1e9
+        result["cpu_baseline"] = {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
+                                  "sample": "2 of the 20 PageRank iterations on the full cfg4 graph "
+                                            f"({dt:.1f} s; oracle/oracle.c or_pagerank, single thread)"}
+    if rank == 0:
+        print(json.dumps(result), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def per_algo(tigr, torch, rec, args, s, deg):
+    """Algorithm-only GTEPS for BFS/SSSP/CC/SSWP on the same scale-24 graph (weights 1-64;
+    CC on the symmetrised graph), device-timed; input-normalised GTEPS = arcs out of reached
+    vertices (CC: all 2m arcs) / time, plus processed-arc GTEPS from collect_stats."""
+    res = {}
+    n, m = rec.n, rec.m
+    g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, weighted=True,
+                             stream=s)
+    vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+    for algo in ("bfs", "sssp", "sswp", "cc"):
+        if algo == "cc":
+            vg.free(); g.free()
+            g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, symmetrize=True,
+                                     stream=s)
+            vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+        out = torch.empty(n, dtype=torch.int32, device="cuda")
+        _, st = tigr.tigr_run(vg, algo, 0, out=out, stream=s, collect_stats=1, return_stats=True)
+        times = []
+        for _ in range(3):
+            _, st2 = tigr.tigr_run(vg, algo, 0, out=out, stream=s, return_stats=True)
+            times.append(st2["ms_total"])
+        t = statistics.median(times)
+        if algo == "cc":
+            m_in = 2 * m
+        else:
+            reached = out.cpu().numpy().view(np.uint32)
+            mask = reached != (0 if algo == "sswp" else 0xFFFFFFFF)
+            m_in = int(deg[mask].sum())
+        res[algo] = {"ms": t, "iterations": st["iterations"], "gteps_input": m_in / (t * 1e-3) / 1e9,
+                     "gteps_processed": st["edges_processed"] / (t * 1e-3) / 1e9,
+                     "edges_processed": st["edges_processed"]}
+    vg.free()
+    g.free()
+    return res
+
+
+if __name__ == "__main__":
+    main()

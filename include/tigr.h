@@ -1,0 +1,211 @@
+/*
+ * tigr.h -- C ABI of the B200-native Tigr hot path (libtigr.so).
+ *
+ * Tigr (Nodehi Sabet, Qiu, Zhao, ASPLOS'18; /root/reference/PAPER.md) runs
+ * push-style vertex-centric graph analytics over a VIRTUALLY split graph: every
+ * node of out-degree d is split into ceil(d/K) virtual nodes (Def. 1-2;
+ * §4.1 "Virtual Node Array", L819-901, Fig. 10), whose edges are assigned in a
+ * coalesced stride order (§4.4 "Edge-array Coalescing", L1104-1180, Fig. 12,
+ * Alg. 3), and all virtual nodes of a family read/write the one value slot of
+ * their physical node ("Implicit Value Synchronization", L978-1001).  A relax
+ * kernel per algorithm (Alg. 2/3, L1080-1090 / L1161-1172) runs to a fixed point
+ * under a worklist (§5).
+ *
+ * Conventions for every call:
+ *  - Returns tigr_status; 0 == TIGR_OK.  Never aborts or exits.  On failure the
+ *    message is available from tigr_last_error() (thread-local, valid until the
+ *    next call on the same thread) and output handles are left NULL.
+ *  - "device" pointers are CUDA device (or managed) pointers on the current
+ *    device; "host" pointers are plain host memory (pinned memory is faster).
+ *    `is_device_ptr` says which one the caller passes.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    All work is ordered on it; calls that return host-visible results
+ *    synchronise it.
+ *  - Handles own their device memory and are freed with the matching *_free.
+ *    A tigr_vgraph references its tigr_graph: free the vgraph first.
+ *  - Vertex ids are uint32 in [0, n); n <= 0xFFFFFFFE (0xFFFFFFFF is "infinity").
+ *  - There is no CPU fallback: without a usable CUDA device every call that
+ *    needs one returns TIGR_ECUDA.
+ */
+#ifndef TIGR_H_
+#define TIGR_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    TIGR_OK = 0,
+    TIGR_EINVAL = -1,      /* bad argument: id >= n, K == 0, source >= n, unweighted SSSP/SSWP, ... */
+    TIGR_ENOMEM = -2,      /* device allocation failed */
+    TIGR_ECUDA = -3,       /* CUDA runtime / driver error (no device, launch failure, ...) */
+    TIGR_ENCCL = -4,       /* NCCL error (multi-GPU) */
+    TIGR_ERANGE = -5,      /* size limit: n > 0xFFFFFFFE, edge/vnode counts beyond 32-bit slots */
+    TIGR_ENOTCONV = -6,    /* max_iters reached before the fixed point */
+    TIGR_EUNSUPPORTED = -7 /* option combination not implemented */
+} tigr_status;
+
+/* Algorithms (Table 4; semantics in DESIGN.md "Readings"). */
+typedef enum {
+    TIGR_BFS = 0,   /* level (hop count) from source; unreached = 0xFFFFFFFF (L718-720) */
+    TIGR_SSSP = 1,  /* min weight sum from source; unreached = 0xFFFFFFFF (Fig. 2, Alg. 2/3) */
+    TIGR_CC = 2,    /* min vertex id of the weakly connected component (Cor. 1, L688-694);
+                       needs a graph built with symmetrize=1 (or symmetric_hint=1) */
+    TIGR_SSWP = 3,  /* max over paths of the min edge weight; source = 0xFFFFFFFF,
+                       unreached = 0 (Cor. 3, L725-734) */
+    TIGR_PR = 4     /* PageRank, float64, fixed iteration count (fn. 7 L1078, Cor. 4 L787-791) */
+} tigr_algo;
+
+/* Edge assignment of the virtual nodes of one family. */
+typedef enum {
+    TIGR_LAYOUT_CONSECUTIVE = 0, /* Fig. 10 / Alg. 2: vnode j owns segment positions [jK, (j+1)K) */
+    TIGR_LAYOUT_STRIDED = 1      /* Fig. 12 / Alg. 3: vnode j owns units j, j+m_v, j+2m_v, ...
+                                    (unit = one 16-byte chunk of 4 edges when 4 | K, else 1 edge) */
+} tigr_layout;
+
+/* Worklist policy (§5; Table 8). */
+typedef enum {
+    TIGR_FRONTIER_AUTO = 0,    /* = DENSE in this version */
+    TIGR_FRONTIER_DENSE = 1,   /* per-node active flags; inactive vnodes exit early */
+    TIGR_FRONTIER_NONE = 2     /* every vnode every iteration (Table 8 "without worklist") */
+} tigr_frontier;
+
+typedef struct tigr_graph tigr_graph;   /* device CSR; owns its buffers */
+typedef struct tigr_vgraph tigr_vgraph; /* virtual node array + per-node info; refs its graph */
+typedef struct tigr_comm tigr_comm;     /* NCCL communicator + rank/size (multi-GPU) */
+
+typedef struct {
+    uint32_t max_iters;   /* frontier algorithms: iteration cap (0 = n + 1); exceeded -> TIGR_ENOTCONV */
+    uint32_t pr_iters;    /* PR iterations (default 20, BASELINE config 4) */
+    double pr_damping;    /* PR damping d (default 0.85) */
+    int pr_dangling;      /* 0 = dangling mass dropped (default), 1 = spread uniformly */
+    int schedule;         /* 0 = asynchronous in place ("synchronization relaxation", §5),
+                             1 = BSP (each vnode reads its node's value from the previous iteration).
+                             PR is always Jacobi. */
+    int frontier;         /* tigr_frontier */
+    int use_graph;        /* 1 (default) = iteration loop as a CUDA graph with a device-side
+                             conditional WHILE node (no host round trip per iteration); 0 = host loop */
+    int collect_stats;    /* 1 = count processed edges / updates on the device (slower) */
+    int time_kernels;     /* 1 = CUDA-event time every relax launch into tigr_stats.ms_relax (host loop) */
+    tigr_comm* comm;      /* NULL = single GPU; else this rank's communicator (see tigr_vgraph_partition) */
+    void* stream;         /* cudaStream_t */
+} tigr_run_opts;
+
+typedef struct {
+    uint32_t iterations;      /* relax iterations executed (frontier algorithms: the last changes nothing) */
+    uint32_t relax_launches;  /* relax kernel launches */
+    uint64_t edges_processed; /* sum over iterations of the edges of active vnodes (collect_stats) */
+    uint64_t updates;         /* successful atomic improvements (collect_stats; not PR) */
+    uint64_t active_vnodes;   /* sum over iterations of active vnodes (collect_stats) */
+    double ms_total;          /* device time of the whole run (init -> values on device) */
+    double ms_relax;          /* device time of the relax launches (time_kernels) */
+    double ms_exchange;       /* device time of the multi-GPU exchanges (time_kernels) */
+} tigr_stats;
+
+/* Fill *opts with the defaults above. */
+void tigr_run_opts_default(tigr_run_opts* opts);
+
+/* ---------------------------------------------------------------- graphs ---- */
+
+/* Build a device CSR from an arc list (src[e] -> dst[e], weight w[e]); w may be NULL
+ * (unweighted graph).  Arcs are grouped by source (Fig. 10a); duplicates
+ * and self-loops are kept; the order of arcs within a source is unspecified.
+ * symmetrize=1 appends (dst[e] -> src[e], w[e]) for every arc (weak connectivity, CC).
+ * Errors: EINVAL (an id >= n, n == 0), ERANGE (n > 0xFFFFFFFE or too many arcs). */
+tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                const uint32_t* w, int is_device_ptr, int symmetrize, void* stream,
+                                tigr_graph** out);
+
+/* Build from a CSR (row_ptr[n+1] int64, col[m], optional w[m]).  symmetric_hint=1 declares
+ * the caller's graph symmetric (required for TIGR_CC).  Errors: EINVAL on a non-monotone
+ * row_ptr, row_ptr[0] != 0, row_ptr[n] != m, or col >= n. */
+tigr_status tigr_graph_from_csr(uint32_t n, uint64_t m, const int64_t* row_ptr, const uint32_t* col,
+                                const uint32_t* w, int is_device_ptr, int symmetric_hint, void* stream,
+                                tigr_graph** out);
+
+/* Draw an R-MAT arc list on the device (Philox4x32-10 counter-based; spec in DESIGN.md
+ * "Generator spec"; bit-identical to graphgen/) into caller-owned DEVICE buffers
+ * src[m], dst[m] and (if non-NULL) w[m] with weights in [wmin, wmax]. */
+tigr_status tigr_rmat_coo(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed,
+                          uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src, uint32_t* dst,
+                          uint32_t* w, void* stream);
+
+/* tigr_rmat_coo into temporary device memory + tigr_graph_from_coo. weighted=0 -> no weights. */
+tigr_status tigr_graph_rmat(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed,
+                            uint64_t wseed, uint32_t wmin, uint32_t wmax, int weighted, int symmetrize,
+                            void* stream, tigr_graph** out);
+
+/* Sizes and flags of a graph (any pointer may be NULL). */
+tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* weighted,
+                            int* symmetric, uint64_t* device_bytes);
+
+/* Copy the CSR out (row_ptr[n+1], col[m], w[m] if weighted and w != NULL), arcs of a
+ * source contiguous in the graph's internal order. */
+tigr_status tigr_graph_export_csr(const tigr_graph* g, int64_t* row_ptr, uint32_t* col, uint32_t* w,
+                                  int is_device_ptr, void* stream);
+
+void tigr_graph_free(tigr_graph* g);
+
+/* --------------------------------------------------------- virtual split ---- */
+
+/* Virtual split transformation with degree bound K >= 1 (Def. 1-2; K = 0xFFFFFFFF means
+ * "no split", the K=inf baseline of Table 2).  Builds on the device: family sizes
+ * m_v = ceil(d_v / K) (0 for d_v = 0), vnode_ptr = exclusive scan of m_v, the virtual node
+ * array vn_phys[NV] (Fig. 10b physicalNodeId row) and a 16-byte per-node record
+ * {edge chunk, degree, first vnode, m_v}.  Errors: EINVAL (K == 0), ERANGE (NV >= 2^32). */
+tigr_status tigr_virtualize(const tigr_graph* g, uint32_t K, tigr_layout layout, void* stream,
+                            tigr_vgraph** out);
+
+/* nv = number of virtual nodes; bytes = device bytes of the virtual structures;
+ * ms_build = device time of the last tigr_virtualize (Table 7 analogue). */
+tigr_status tigr_vgraph_info(const tigr_vgraph* vg, uint64_t* nv, uint64_t* bytes, double* ms_build,
+                             uint32_t* vnode_lo, uint32_t* vnode_hi);
+
+/* Copy vnode_ptr[n+1] and vn_phys[NV] out (either may be NULL). */
+tigr_status tigr_vgraph_export(const tigr_vgraph* vg, uint32_t* vnode_ptr, uint32_t* vn_phys,
+                               int is_device_ptr, void* stream);
+
+/* The edges each virtual node owns, walked with the relax kernels' own index arithmetic:
+ * counts[NV] and, grouped by vnode in vnode order (offsets = exclusive scan of counts),
+ * nbr[m] and (weighted graphs, if non-NULL) w[m].  For layout parity tests. */
+tigr_status tigr_vgraph_assignment(const tigr_vgraph* vg, uint32_t* counts, uint32_t* nbr, uint32_t* w,
+                                   int is_device_ptr, void* stream);
+
+/* Restrict this rank's relax work to a contiguous, family-aligned vnode range balanced by
+ * edge count (rank r of nranks).  nranks = 1 restores the full range. */
+tigr_status tigr_vgraph_partition(tigr_vgraph* vg, int nranks, int rank);
+
+void tigr_vgraph_free(tigr_vgraph* vg);
+
+/* ------------------------------------------------------------------ runs ---- */
+
+/* Run `algo` from `source` (ignored by CC and PR) to the fixed point (PR: pr_iters
+ * iterations) and write n values to out_values: uint32 for BFS/SSSP/CC/SSWP, float64
+ * for PR.  opts may be NULL (defaults).  stats may be NULL.
+ * Errors: EINVAL (source >= n; SSSP/SSWP on an unweighted graph; CC on a graph not built
+ * symmetric), ENOTCONV (max_iters hit; values hold the last iterate), ENCCL. */
+tigr_status tigr_run(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tigr_run_opts* opts,
+                     void* out_values, int out_is_device, tigr_stats* stats);
+
+/* ------------------------------------------------------------- multi-GPU ---- */
+
+/* NCCL bootstrap: rank 0 creates the 128-byte id and broadcasts it (e.g. over
+ * torch.distributed); every rank then calls tigr_comm_init on its own device. */
+tigr_status tigr_comm_unique_id(uint8_t id[128]);
+tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
+void tigr_comm_free(tigr_comm* comm);
+
+/* ----------------------------------------------------------------- misc ---- */
+
+const char* tigr_last_error(void);
+/* Number of CUDA kernels this library launched in this process (graph-launched ones
+ * included, counted per executed node). */
+uint64_t tigr_launch_count(void);
+const char* tigr_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TIGR_H_ */

@@ -1,0 +1,293 @@
+// api.cu -- the extern "C" boundary of libtigr.so (include/tigr.h).  Argument checking,
+// host<->device staging, error state; every compute step runs in the kernels of the other
+// translation units.
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "internal.cuh"
+#include "vgraph.cuh"
+
+namespace tigr {
+
+std::atomic<uint64_t> g_launches{0};
+static thread_local std::string t_err;
+
+void set_error(const std::string& msg) { t_err = msg; }
+
+tigr_status fail(tigr_status st, const std::string& msg) {
+    t_err = msg;
+    return st;
+}
+
+tigr_status cuda_fail(cudaError_t e, const char* what, const char* file, int line) {
+    char buf[512];
+    snprintf(buf, sizeof(buf), "%s: %s (%s) at %s:%d", what, cudaGetErrorName(e), cudaGetErrorString(e), file, line);
+    t_err = buf;
+    return (e == cudaErrorMemoryAllocation) ? TIGR_ENOMEM : TIGR_ECUDA;
+}
+
+tigr_status DevBuf::alloc(size_t nbytes) {
+    release();
+    cudaError_t e = cudaMalloc(&p, nbytes ? nbytes : 16);
+    if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMalloc", __FILE__, __LINE__); }
+    bytes = nbytes;
+    return TIGR_OK;
+}
+
+void DevBuf::release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    bytes = 0;
+}
+
+tigr_status TmpBuf::alloc(size_t nbytes, cudaStream_t stream) {
+    s = stream;
+    cudaError_t e = cudaMallocAsync(&p, nbytes ? nbytes : 16, stream);
+    if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMallocAsync", __FILE__, __LINE__); }
+    return TIGR_OK;
+}
+
+TmpBuf::~TmpBuf() {
+    if (p) cudaFreeAsync(p, s);
+}
+
+// other translation units
+tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double b, double c, uint64_t seed,
+                       uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src, uint32_t* dst, uint32_t* w,
+                       cudaStream_t s);
+tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                  const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out);
+tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col, const uint32_t* w,
+                                  int symmetric_hint, cudaStream_t s, tigr_graph** out);
+tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w, cudaStream_t s);
+tigr_status graph_rmat_device(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed, uint64_t wseed,
+                              uint32_t wmin, uint32_t wmax, int weighted, int symmetrize, cudaStream_t s,
+                              tigr_graph** out);
+tigr_status virtualize_device(const tigr_graph* g, uint32_t K, tigr_layout layout, cudaStream_t s, tigr_vgraph** out);
+tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tigr_run_opts& o, void* out,
+                       int out_is_device, tigr_stats* st);
+tigr_status assignment_device(const tigr_vgraph* vg, uint32_t* counts, uint32_t* nbr, uint32_t* w, cudaStream_t s);
+tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank);
+tigr_status comm_unique_id(uint8_t id[128]);
+tigr_status comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
+void comm_free(tigr_comm* c);
+
+namespace {
+
+tigr_status need_device() {
+    int count = 0;
+    cudaError_t e = cudaGetDeviceCount(&count);
+    if (e != cudaSuccess || count == 0)
+        return fail(TIGR_ECUDA, std::string("no CUDA device available (libtigr has no CPU fallback): ") +
+                                    cudaGetErrorString(e));
+    return TIGR_OK;
+}
+
+// stage a host array into a temporary device buffer (or pass a device pointer through)
+template <class T>
+tigr_status stage(const T* p, uint64_t count, int is_device, cudaStream_t s, TmpBuf& tmp, const T** out) {
+    if (!p || is_device) { *out = p; return TIGR_OK; }
+    TIGR_TRY(tmp.alloc(sizeof(T) * (count ? count : 1), s));
+    if (count) TIGR_CK(cudaMemcpyAsync(tmp.p, p, sizeof(T) * count, cudaMemcpyHostToDevice, s));
+    *out = tmp.as<T>();
+    return TIGR_OK;
+}
+
+}  // namespace
+}  // namespace tigr
+
+using namespace tigr;
+
+extern "C" {
+
+void tigr_run_opts_default(tigr_run_opts* o) {
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->max_iters = 0;
+    o->pr_iters = 20;
+    o->pr_damping = 0.85;
+    o->pr_dangling = 0;
+    o->schedule = 0;
+    o->frontier = TIGR_FRONTIER_AUTO;
+    o->use_graph = 1;
+}
+
+tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
+                                int is_device_ptr, int symmetrize, void* stream, tigr_graph** out) {
+    if (!out) return fail(TIGR_EINVAL, "graph_from_coo: out is NULL");
+    *out = nullptr;
+    if (n == 0) return fail(TIGR_EINVAL, "graph_from_coo: n == 0");
+    if (n > 0xFFFFFFFEu) return fail(TIGR_ERANGE, "graph_from_coo: n > 0xFFFFFFFE");
+    if (m && (!src || !dst)) return fail(TIGR_EINVAL, "graph_from_coo: src/dst NULL");
+    TIGR_TRY(need_device());
+    cudaStream_t s = (cudaStream_t)stream;
+    TmpBuf ts, td, tw;
+    const uint32_t *ds = nullptr, *dd = nullptr, *dw = nullptr;
+    TIGR_TRY(stage(src, m, is_device_ptr, s, ts, &ds));
+    TIGR_TRY(stage(dst, m, is_device_ptr, s, td, &dd));
+    TIGR_TRY(stage(w, m, is_device_ptr, s, tw, &dw));
+    TIGR_TRY(graph_from_coo_device(n, m, ds, dd, dw, symmetrize, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_graph_from_csr(uint32_t n, uint64_t m, const int64_t* row_ptr, const uint32_t* col, const uint32_t* w,
+                                int is_device_ptr, int symmetric_hint, void* stream, tigr_graph** out) {
+    if (!out) return fail(TIGR_EINVAL, "graph_from_csr: out is NULL");
+    *out = nullptr;
+    if (n == 0) return fail(TIGR_EINVAL, "graph_from_csr: n == 0");
+    if (n > 0xFFFFFFFEu) return fail(TIGR_ERANGE, "graph_from_csr: n > 0xFFFFFFFE");
+    if (!row_ptr || (m && !col)) return fail(TIGR_EINVAL, "graph_from_csr: NULL array");
+    TIGR_TRY(need_device());
+    cudaStream_t s = (cudaStream_t)stream;
+    TmpBuf tr, tc, tw;
+    const int64_t* dr = nullptr;
+    const uint32_t *dc = nullptr, *dw = nullptr;
+    TIGR_TRY(stage(row_ptr, (uint64_t)n + 1, is_device_ptr, s, tr, &dr));
+    TIGR_TRY(stage(col, m, is_device_ptr, s, tc, &dc));
+    TIGR_TRY(stage(w, m, is_device_ptr, s, tw, &dw));
+    TIGR_TRY(graph_from_csr_device(n, m, dr, dc, dw, symmetric_hint, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_rmat_coo(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed, uint64_t wseed,
+                          uint32_t wmin, uint32_t wmax, uint32_t* src, uint32_t* dst, uint32_t* w, void* stream) {
+    if (m && (!src || !dst)) return fail(TIGR_EINVAL, "rmat_coo: src/dst NULL");
+    TIGR_TRY(need_device());
+    return rmat_range(n, 0, m, a, b, c, seed, wseed, wmin, wmax, src, dst, w, (cudaStream_t)stream);
+}
+
+tigr_status tigr_graph_rmat(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed, uint64_t wseed,
+                            uint32_t wmin, uint32_t wmax, int weighted, int symmetrize, void* stream,
+                            tigr_graph** out) {
+    if (!out) return fail(TIGR_EINVAL, "graph_rmat: out is NULL");
+    *out = nullptr;
+    TIGR_TRY(need_device());
+    cudaStream_t s = (cudaStream_t)stream;
+    TIGR_TRY(graph_rmat_device(n, m, a, b, c, seed, wseed, wmin, wmax, weighted, symmetrize, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* weighted, int* symmetric,
+                            uint64_t* device_bytes) {
+    if (!g) return fail(TIGR_EINVAL, "graph_info: NULL graph");
+    if (n) *n = g->n;
+    if (m) *m = g->m;
+    if (weighted) *weighted = g->weighted;
+    if (symmetric) *symmetric = g->symmetric;
+    if (device_bytes) *device_bytes = g->row_ptr.bytes + g->deg.bytes + g->cptr.bytes + g->col.bytes + g->wt.bytes;
+    return TIGR_OK;
+}
+
+tigr_status tigr_graph_export_csr(const tigr_graph* g, int64_t* row_ptr, uint32_t* col, uint32_t* w,
+                                  int is_device_ptr, void* stream) {
+    if (!g) return fail(TIGR_EINVAL, "graph_export_csr: NULL graph");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (is_device_ptr) {
+        TIGR_TRY(graph_export_csr_device(g, row_ptr, col, w, s));
+        TIGR_CK(cudaStreamSynchronize(s));
+        return TIGR_OK;
+    }
+    TmpBuf dr, dc, dw;
+    if (row_ptr) TIGR_TRY(dr.alloc(sizeof(int64_t) * ((size_t)g->n + 1), s));
+    if (col) TIGR_TRY(dc.alloc(sizeof(uint32_t) * (g->m ? g->m : 1), s));
+    if (w && g->weighted) TIGR_TRY(dw.alloc(sizeof(uint32_t) * (g->m ? g->m : 1), s));
+    TIGR_TRY(graph_export_csr_device(g, dr.as<int64_t>(), dc.as<uint32_t>(), dw.as<uint32_t>(), s));
+    if (row_ptr) TIGR_CK(cudaMemcpyAsync(row_ptr, dr.p, sizeof(int64_t) * ((size_t)g->n + 1), cudaMemcpyDeviceToHost, s));
+    if (col && g->m) TIGR_CK(cudaMemcpyAsync(col, dc.p, sizeof(uint32_t) * g->m, cudaMemcpyDeviceToHost, s));
+    if (w && g->weighted && g->m) TIGR_CK(cudaMemcpyAsync(w, dw.p, sizeof(uint32_t) * g->m, cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+void tigr_graph_free(tigr_graph* g) { delete g; }
+
+tigr_status tigr_virtualize(const tigr_graph* g, uint32_t K, tigr_layout layout, void* stream, tigr_vgraph** out) {
+    if (!g || !out) return fail(TIGR_EINVAL, "virtualize: NULL argument");
+    *out = nullptr;
+    return virtualize_device(g, K, layout, (cudaStream_t)stream, out);
+}
+
+tigr_status tigr_vgraph_info(const tigr_vgraph* vg, uint64_t* nv, uint64_t* bytes, double* ms_build, uint32_t* lo,
+                             uint32_t* hi) {
+    if (!vg) return fail(TIGR_EINVAL, "vgraph_info: NULL vgraph");
+    if (nv) *nv = vg->nv;
+    if (bytes) *bytes = vg->vnode_ptr.bytes + vg->vn_phys.bytes + vg->vinfo.bytes;
+    if (ms_build) *ms_build = vg->ms_build;
+    if (lo) *lo = vg->lo;
+    if (hi) *hi = vg->hi;
+    return TIGR_OK;
+}
+
+tigr_status tigr_vgraph_export(const tigr_vgraph* vg, uint32_t* vnode_ptr, uint32_t* vn_phys, int is_device_ptr,
+                               void* stream) {
+    if (!vg) return fail(TIGR_EINVAL, "vgraph_export: NULL vgraph");
+    cudaStream_t s = (cudaStream_t)stream;
+    const cudaMemcpyKind k = is_device_ptr ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
+    if (vnode_ptr)
+        TIGR_CK(cudaMemcpyAsync(vnode_ptr, vg->vnode_ptr.p, sizeof(uint32_t) * ((size_t)vg->g->n + 1), k, s));
+    if (vn_phys && vg->nv) TIGR_CK(cudaMemcpyAsync(vn_phys, vg->vn_phys.p, sizeof(uint32_t) * vg->nv, k, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_vgraph_assignment(const tigr_vgraph* vg, uint32_t* counts, uint32_t* nbr, uint32_t* w,
+                                   int is_device_ptr, void* stream) {
+    if (!vg || !counts || !nbr) return fail(TIGR_EINVAL, "vgraph_assignment: NULL argument");
+    cudaStream_t s = (cudaStream_t)stream;
+    const uint64_t m = vg->g->m;
+    if (is_device_ptr) {
+        TIGR_TRY(assignment_device(vg, counts, nbr, w, s));
+        TIGR_CK(cudaStreamSynchronize(s));
+        return TIGR_OK;
+    }
+    TmpBuf dc, dn, dw;
+    TIGR_TRY(dc.alloc(sizeof(uint32_t) * (vg->nv ? vg->nv : 1), s));
+    TIGR_TRY(dn.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    if (w) TIGR_TRY(dw.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    TIGR_TRY(assignment_device(vg, dc.as<uint32_t>(), dn.as<uint32_t>(), dw.as<uint32_t>(), s));
+    if (vg->nv) TIGR_CK(cudaMemcpyAsync(counts, dc.p, sizeof(uint32_t) * vg->nv, cudaMemcpyDeviceToHost, s));
+    if (m) TIGR_CK(cudaMemcpyAsync(nbr, dn.p, sizeof(uint32_t) * m, cudaMemcpyDeviceToHost, s));
+    if (w && m) TIGR_CK(cudaMemcpyAsync(w, dw.p, sizeof(uint32_t) * m, cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_vgraph_partition(tigr_vgraph* vg, int nranks, int rank) {
+    if (!vg) return fail(TIGR_EINVAL, "vgraph_partition: NULL vgraph");
+    return partition_host(vg, nranks, rank);
+}
+
+void tigr_vgraph_free(tigr_vgraph* vg) { delete vg; }
+
+tigr_status tigr_run(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tigr_run_opts* opts, void* out_values,
+                     int out_is_device, tigr_stats* stats) {
+    if (!vg) return fail(TIGR_EINVAL, "run: NULL vgraph");
+    tigr_run_opts o;
+    if (opts) o = *opts; else tigr_run_opts_default(&o);
+    return run_device(vg, algo, source, o, out_values, out_is_device, stats);
+}
+
+tigr_status tigr_comm_unique_id(uint8_t id[128]) {
+    if (!id) return fail(TIGR_EINVAL, "comm_unique_id: NULL");
+    return comm_unique_id(id);
+}
+
+tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out) {
+    if (!id || !out) return fail(TIGR_EINVAL, "comm_init: NULL");
+    *out = nullptr;
+    return comm_init(nranks, rank, id, out);
+}
+
+void tigr_comm_free(tigr_comm* c) { comm_free(c); }
+
+const char* tigr_last_error(void) { return t_err.c_str(); }
+
+uint64_t tigr_launch_count(void) { return g_launches.load(); }
+
+const char* tigr_version(void) { return "tigr-b200 0.1 (sm_100a)"; }
+
+}  // extern "C"

@@ -1,0 +1,299 @@
+// csr.cu -- device CSR construction.
+//
+// CSR = node array (exclusive scan of out-degrees) + edge array grouped by source
+// (Fig. 10a; "we reorder the edges during the construction of CSR",
+// L1131-1132).  B200 layout: every node's segment starts on a 16-byte boundary and is
+// padded to a multiple of 4 slots (pads = 0xFFFFFFFF), so the relax kernels can move
+// edges (and, in a separate array, weights) as 128-bit chunks; cptr[v] is the first chunk.
+// The arc order inside a segment is whatever the atomic scatter produced (the paper's
+// results do not depend on it; tests compare segments as multisets).
+#include "internal.cuh"
+
+namespace tigr {
+
+tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double b, double c,
+                       uint64_t seed, uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src,
+                       uint32_t* dst, uint32_t* w, cudaStream_t s);
+
+namespace {
+
+__global__ void k_maxid(const uint32_t* __restrict__ a, const uint32_t* __restrict__ b, uint64_t m,
+                        uint32_t* out) {
+    uint32_t mx = 0;
+    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
+         i += (uint64_t)gridDim.x * blockDim.x)
+        mx = max(mx, max(a[i], b[i]));
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
+}
+
+// out-degree histogram; warp-aggregated so hub sources cost one atomic per warp
+__device__ __forceinline__ void agg_add(uint32_t* cnt, uint32_t key, bool valid) {
+    const uint32_t active = __ballot_sync(0xffffffffu, valid);
+    if (!valid) return;
+    const uint32_t peers = __match_any_sync(active, key);
+    const int lane = threadIdx.x & 31;
+    if (lane == __ffs(peers) - 1) atomicAdd(&cnt[key], (uint32_t)__popc(peers));
+}
+
+__global__ void k_hist(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
+                       int sym, uint32_t* deg) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t start = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t rounds = (m + stride - 1) / stride;
+    for (uint64_t r = 0; r < rounds; ++r) {
+        const uint64_t i = start + r * stride;
+        const bool v = i < m;
+        agg_add(deg, v ? src[i] : 0, v);
+        if (sym) agg_add(deg, v ? dst[i] : 0, v);
+    }
+}
+
+// warp-aggregated slot reservation: returns this lane's position within its source segment
+__device__ __forceinline__ uint32_t agg_reserve(uint32_t* cursor, uint32_t key, bool valid) {
+    const uint32_t active = __ballot_sync(0xffffffffu, valid);
+    if (!valid) return 0;
+    const uint32_t peers = __match_any_sync(active, key);
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(peers) - 1;
+    uint32_t base = 0;
+    if (lane == leader) base = atomicAdd(&cursor[key], (uint32_t)__popc(peers));
+    base = __shfl_sync(peers, base, leader);
+    return base + __popc(peers & ((1u << lane) - 1));
+}
+
+__global__ void k_scatter(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst,
+                          const uint32_t* __restrict__ w, uint64_t m, int sym,
+                          const uint32_t* __restrict__ cptr, uint32_t* cursor, uint32_t* __restrict__ col,
+                          uint32_t* __restrict__ wt) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const uint64_t start = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t rounds = (m + stride - 1) / stride;
+    for (uint64_t r = 0; r < rounds; ++r) {
+        const uint64_t i = start + r * stride;
+        const bool v = i < m;
+        const uint32_t s = v ? src[i] : 0, d = v ? dst[i] : 0;
+        const uint32_t x = (v && w) ? w[i] : 0;
+        {
+            const uint32_t p = agg_reserve(cursor, s, v);
+            if (v) {
+                const uint64_t slot = (uint64_t)cptr[s] * kChunk + p;
+                col[slot] = d;
+                if (wt) wt[slot] = x;
+            }
+        }
+        if (sym) {
+            const uint32_t p = agg_reserve(cursor, d, v);
+            if (v) {
+                const uint64_t slot = (uint64_t)cptr[d] * kChunk + p;
+                col[slot] = s;
+                if (wt) wt[slot] = x;
+            }
+        }
+    }
+}
+
+__global__ void k_pad(const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cptr, uint32_t n,
+                      uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    const uint64_t base = (uint64_t)cptr[v] * kChunk;
+    const uint32_t d = deg[v];
+    const uint64_t end = (uint64_t)cptr[v + 1] * kChunk;
+    for (uint64_t s = base + d; s < end; ++s) {
+        col[s] = kPad;
+        if (wt) wt[s] = 0;
+    }
+}
+
+__global__ void k_deg_from_rowptr(const int64_t* __restrict__ rp, uint32_t n, uint64_t m,
+                                  uint32_t* __restrict__ deg, uint32_t* bad) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v == 0 && (rp[0] != 0 || rp[n] != (int64_t)m)) *bad = 1;
+    if (v >= n) return;
+    const int64_t d = rp[v + 1] - rp[v];
+    if (d < 0 || d > 0xFFFFFFFFll) { *bad = 1; deg[v] = 0; return; }
+    deg[v] = (uint32_t)d;
+}
+
+__device__ __forceinline__ uint32_t owner_of(const int64_t* __restrict__ rp, uint32_t n, uint64_t e) {
+    uint32_t lo = 0, hi = n;  // last v with rp[v] <= e
+    while (hi - lo > 1) {
+        const uint32_t mid = lo + (hi - lo) / 2;
+        if ((uint64_t)rp[mid] <= e) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+// canonical (row_ptr-indexed) arrays <-> padded segments
+__global__ void k_csr_to_padded(const int64_t* __restrict__ rp, uint32_t n, uint64_t m,
+                                const uint32_t* __restrict__ cin, const uint32_t* __restrict__ win,
+                                const uint32_t* __restrict__ cptr, uint32_t* __restrict__ col,
+                                uint32_t* __restrict__ wt, uint32_t* bad) {
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m;
+         e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = owner_of(rp, n, e);
+        const uint64_t slot = (uint64_t)cptr[v] * kChunk + (e - rp[v]);
+        const uint32_t c = cin[e];
+        if (c >= n) *bad = 1;
+        col[slot] = c;
+        if (wt) wt[slot] = win[e];
+    }
+}
+
+__global__ void k_padded_to_csr(const int64_t* __restrict__ rp, uint32_t n, uint64_t m,
+                                const uint32_t* __restrict__ cptr, const uint32_t* __restrict__ col,
+                                const uint32_t* __restrict__ wt, uint32_t* __restrict__ cout,
+                                uint32_t* __restrict__ wout) {
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m;
+         e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = owner_of(rp, n, e);
+        const uint64_t slot = (uint64_t)cptr[v] * kChunk + (e - rp[v]);
+        if (cout) cout[e] = col[slot];
+        if (wout) wout[e] = wt[slot];
+    }
+}
+
+unsigned capped_grid(uint64_t items) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t want = (items + kBlock - 1) / kBlock;
+    const uint64_t cap = (uint64_t)sms * 16;
+    return (unsigned)(want == 0 ? 1 : (want < cap ? want : cap));
+}
+
+// degrees known -> row_ptr, cptr, edge buffers
+tigr_status layout_from_degrees(tigr_graph* g, cudaStream_t s) {
+    TIGR_TRY(g->row_ptr.alloc(sizeof(int64_t) * ((size_t)g->n + 1)));
+    TIGR_TRY(exclusive_scan_u64(g->deg.as<uint32_t>(), g->n, SCAN_U32, 1,
+                                reinterpret_cast<uint64_t*>(g->row_ptr.p), s));
+    TIGR_TRY(g->cptr.alloc(sizeof(uint32_t) * ((size_t)g->n + 1)));
+    uint64_t nch = 0;
+    TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), g->n, SCAN_CEIL_DIV, kChunk, g->cptr.as<uint32_t>(),
+                                s, &nch));
+    if (nch >= (1ull << 32)) return fail(TIGR_ERANGE, "graph: padded edge chunks exceed 2^32");
+    g->nchunks = nch;
+    TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1)));
+    if (g->weighted) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1)));
+    return TIGR_OK;
+}
+
+}  // namespace
+
+tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                  const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out) {
+    const uint64_t arcs = symmetrize ? 2 * m : m;
+    if (arcs >= (1ull << 32) * 3) return fail(TIGR_ERANGE, "graph: too many arcs");
+    if (m) {
+        TmpBuf mx;
+        TIGR_TRY(mx.alloc(sizeof(uint32_t), s));
+        TIGR_CK(cudaMemsetAsync(mx.p, 0, sizeof(uint32_t), s));
+        k_maxid<<<capped_grid(m), kBlock, 0, s>>>(src, dst, m, mx.as<uint32_t>());
+        TIGR_CKL("maxid");
+        uint32_t hmax = 0;
+        TIGR_CK(cudaMemcpyAsync(&hmax, mx.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        TIGR_CK(cudaStreamSynchronize(s));
+        if (hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
+    }
+    tigr_graph* g = new tigr_graph();
+    g->n = n;
+    g->m = arcs;
+    g->weighted = w != nullptr;
+    g->symmetric = symmetrize != 0;
+    auto bail = [&](tigr_status st) { delete g; return st; };
+    tigr_status st = g->deg.alloc(sizeof(uint32_t) * n);
+    if (st) return bail(st);
+    if (cudaMemsetAsync(g->deg.p, 0, sizeof(uint32_t) * n, s) != cudaSuccess)
+        return bail(cuda_fail(cudaGetLastError(), "memset deg", __FILE__, __LINE__));
+    if (m) {
+        k_hist<<<capped_grid(m), kBlock, 0, s>>>(src, dst, m, symmetrize, g->deg.as<uint32_t>());
+        count_launch();
+    }
+    if ((st = layout_from_degrees(g, s))) return bail(st);
+    if (m) {
+        TmpBuf cursor;
+        if ((st = cursor.alloc(sizeof(uint32_t) * n, s))) return bail(st);
+        cudaMemsetAsync(cursor.p, 0, sizeof(uint32_t) * n, s);
+        k_scatter<<<capped_grid(m), kBlock, 0, s>>>(src, dst, w, m, symmetrize, g->cptr.as<uint32_t>(),
+                                                    cursor.as<uint32_t>(), g->col.as<uint32_t>(),
+                                                    g->wt.as<uint32_t>());
+        count_launch();
+    }
+    k_pad<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), g->cptr.as<uint32_t>(), n,
+                                          g->col.as<uint32_t>(), g->wt.as<uint32_t>());
+    count_launch();
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return bail(cuda_fail(e, "graph_from_coo kernels", __FILE__, __LINE__));
+    *out = g;
+    return TIGR_OK;
+}
+
+tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col,
+                                  const uint32_t* w, int symmetric_hint, cudaStream_t s, tigr_graph** out) {
+    tigr_graph* g = new tigr_graph();
+    g->n = n;
+    g->m = m;
+    g->weighted = w != nullptr;
+    g->symmetric = symmetric_hint != 0;
+    auto bail = [&](tigr_status st) { delete g; return st; };
+    tigr_status st;
+    TmpBuf bad;
+    if ((st = bad.alloc(sizeof(uint32_t), s))) return bail(st);
+    cudaMemsetAsync(bad.p, 0, sizeof(uint32_t), s);
+    if ((st = g->deg.alloc(sizeof(uint32_t) * n))) return bail(st);
+    k_deg_from_rowptr<<<grid_for(n), kBlock, 0, s>>>(rp, n, m, g->deg.as<uint32_t>(), bad.as<uint32_t>());
+    count_launch();
+    uint32_t hbad = 0;
+    cudaMemcpyAsync(&hbad, bad.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return bail(cuda_fail(e, "from_csr validate", __FILE__, __LINE__));
+    if (hbad) return bail(fail(TIGR_EINVAL, "graph_from_csr: row_ptr not monotone / row_ptr[0] != 0 / row_ptr[n] != m"));
+    if ((st = layout_from_degrees(g, s))) return bail(st);
+    if (m) {
+        k_csr_to_padded<<<capped_grid(m), kBlock, 0, s>>>(rp, n, m, col, w, g->cptr.as<uint32_t>(),
+                                                          g->col.as<uint32_t>(), g->wt.as<uint32_t>(),
+                                                          bad.as<uint32_t>());
+        count_launch();
+    }
+    k_pad<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), g->cptr.as<uint32_t>(), n,
+                                          g->col.as<uint32_t>(), g->wt.as<uint32_t>());
+    count_launch();
+    cudaMemcpyAsync(&hbad, bad.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return bail(cuda_fail(e, "from_csr kernels", __FILE__, __LINE__));
+    if (hbad) return bail(fail(TIGR_EINVAL, "graph_from_csr: col id >= n"));
+    *out = g;
+    return TIGR_OK;
+}
+
+tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w,
+                                    cudaStream_t s) {
+    if (rp)
+        TIGR_CK(cudaMemcpyAsync(rp, g->row_ptr.p, sizeof(int64_t) * ((size_t)g->n + 1),
+                                cudaMemcpyDeviceToDevice, s));
+    if ((col || (w && g->weighted)) && g->m) {
+        k_padded_to_csr<<<capped_grid(g->m), kBlock, 0, s>>>(
+            g->row_ptr.as<int64_t>(), g->n, g->m, g->cptr.as<uint32_t>(), g->col.as<uint32_t>(),
+            g->wt.as<uint32_t>(), col, g->weighted ? w : nullptr);
+        TIGR_CKL("export csr");
+    }
+    return TIGR_OK;
+}
+
+tigr_status graph_rmat_device(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed,
+                              uint64_t wseed, uint32_t wmin, uint32_t wmax, int weighted, int symmetrize,
+                              cudaStream_t s, tigr_graph** out) {
+    TmpBuf src, dst, w;
+    const size_t bytes = sizeof(uint32_t) * (m ? m : 1);
+    TIGR_TRY(src.alloc(bytes, s));
+    TIGR_TRY(dst.alloc(bytes, s));
+    if (weighted) TIGR_TRY(w.alloc(bytes, s));
+    TIGR_TRY(rmat_range(n, 0, m, a, b, c, seed, wseed, wmin, wmax, src.as<uint32_t>(), dst.as<uint32_t>(),
+                        weighted ? w.as<uint32_t>() : nullptr, s));
+    return graph_from_coo_device(n, m, src.as<uint32_t>(), dst.as<uint32_t>(),
+                                 weighted ? w.as<uint32_t>() : nullptr, symmetrize, s, out);
+}
+
+}  // namespace tigr

@@ -1,0 +1,103 @@
+// internal.cuh -- shared internals of libtigr (CUDA, sm_100a).  Not part of the ABI.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <string>
+
+#include "tigr.h"
+
+namespace tigr {
+
+constexpr uint32_t kInf = 0xFFFFFFFFu;
+constexpr uint32_t kChunk = 4;          // edges per 16-byte chunk (col and weight arrays)
+constexpr uint32_t kPad = 0xFFFFFFFFu;  // column value of padding slots
+constexpr int kBlock = 256;
+
+// ---- error state (tigr_last_error) -------------------------------------------------------
+void set_error(const std::string& msg);
+tigr_status fail(tigr_status st, const std::string& msg);
+tigr_status cuda_fail(cudaError_t e, const char* what, const char* file, int line);
+
+extern std::atomic<uint64_t> g_launches;
+inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+#define TIGR_CK(call)                                                         \
+    do {                                                                      \
+        cudaError_t _e = (call);                                              \
+        if (_e != cudaSuccess) return ::tigr::cuda_fail(_e, #call, __FILE__, __LINE__); \
+    } while (0)
+
+#define TIGR_CKL(what)                                                        \
+    do {                                                                      \
+        ::tigr::count_launch();                                               \
+        cudaError_t _e = cudaGetLastError();                                  \
+        if (_e != cudaSuccess) return ::tigr::cuda_fail(_e, what, __FILE__, __LINE__); \
+    } while (0)
+
+#define TIGR_TRY(expr)                                                        \
+    do {                                                                      \
+        tigr_status _s = (expr);                                              \
+        if (_s != TIGR_OK) return _s;                                         \
+    } while (0)
+
+inline unsigned grid_for(uint64_t items, int block = kBlock) {
+    uint64_t g = (items + block - 1) / block;
+    return (unsigned)(g ? g : 1);
+}
+
+// ---- device buffers ------------------------------------------------------------------------
+// Owning device allocation (cudaMalloc; persistent structures) or stream-ordered temporary.
+struct DevBuf {
+    void* p = nullptr;
+    size_t bytes = 0;
+    tigr_status alloc(size_t nbytes);
+    void release();
+    ~DevBuf() { release(); }
+    template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+struct TmpBuf {  // cudaMallocAsync / cudaFreeAsync on a stream
+    void* p = nullptr;
+    cudaStream_t s = nullptr;
+    tigr_status alloc(size_t nbytes, cudaStream_t stream);
+    ~TmpBuf();
+    template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// ---- scan (scan.cu) ----------------------------------------------------------------------
+// out[i] = sum_{k<i} f(k) for i in [0, count], where f is selected by `kind` over `in`:
+enum ScanKind : int {
+    SCAN_U32 = 0,        // f(k) = in[k]
+    SCAN_CEIL_DIV = 1,   // f(k) = ceil(in[k] / div)
+};
+tigr_status exclusive_scan_u64(const uint32_t* in, uint64_t count, ScanKind kind, uint32_t div,
+                               uint64_t* out, cudaStream_t s);
+tigr_status exclusive_scan_u32(const uint32_t* in, uint64_t count, ScanKind kind, uint32_t div,
+                               uint32_t* out, cudaStream_t s, uint64_t* total_host);
+
+}  // namespace tigr
+
+// ---- handles -----------------------------------------------------------------------------
+struct tigr_graph {
+    uint32_t n = 0;
+    uint64_t m = 0;          // arcs (after symmetrisation)
+    uint64_t nchunks = 0;    // 16-byte chunks per edge array (padded segments)
+    bool weighted = false;
+    bool symmetric = false;
+    tigr::DevBuf row_ptr;    // int64[n+1], canonical offsets
+    tigr::DevBuf deg;        // uint32[n]
+    tigr::DevBuf cptr;       // uint32[n+1], first chunk of each node's segment
+    tigr::DevBuf col;        // uint32[4 * nchunks], padded segments, pads = 0xFFFFFFFF
+    tigr::DevBuf wt;         // uint32[4 * nchunks] or empty
+};
+
+struct tigr_comm {
+    void* nccl = nullptr;    // ncclComm_t
+    int nranks = 1;
+    int rank = 0;
+};
+
+struct tigr_vgraph;  // defined in vgraph.cuh

@@ -1,0 +1,354 @@
+// relax.cu -- relax kernels and iteration control.
+//
+// One thread per virtual node (the paper's scheduling unit: "threads are scheduled based on
+// the virtually transformed graph ... each thread is assigned to process a virtual node",
+// §4.4; Alg. 2, Alg. 3):
+//   v = vn_phys[i]                                   (Alg. 2 line 2, "main difference")
+//   x = value[v]                                     (Alg. 2 line 3; BSP: previous iteration)
+//   for its <= K edges e (stride order, Alg. 3 line 7):
+//       alt = f(x, w_e);  if better(alt, value[nbr]) then atomic{Min,Max}(&value[nbr], alt)
+//                                                     and mark nbr active (worklist, §5)
+// PageRank pushes contrib[v] = x[v]/d_v with a float64 atomic add (fn. 7 L1078: the vertex
+// function is split into an associative accumulate and a separate apply; Thm. 3).
+// B200 specifics: edges and weights move as 16-byte chunks through the non-coherent read-only
+// path; the value gathers of a thread's edges are issued together before its atomics; all of
+// a family's virtual nodes share one 16-byte node record; the worklist is an iteration stamp
+// per node (no per-iteration clearing pass); the loop runs on the device as a CUDA graph.
+#include "internal.cuh"
+#include "vgraph.cuh"
+#include "relax.cuh"
+
+namespace tigr {
+
+// ------------------------------------------------------------------------------------------
+// edge walk: the set of (nbr, w) slots a virtual node owns, in the layout's order
+// ------------------------------------------------------------------------------------------
+__device__ __forceinline__ uint4 ldg_chunk(const uint4* p) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    return r;
+}
+
+__device__ __forceinline__ uint32_t ldg_u32(const uint32_t* p) {
+    uint32_t r;
+    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    return r;
+}
+
+// Calls f(nbr[8], w[8]) on batches of up to 8 slots (pads/absent = kPad).
+template <int LAYOUT, bool VEC, bool W, class F>
+__device__ __forceinline__ void walk(const uint32_t* __restrict__ col, const uint32_t* __restrict__ wt,
+                                     uint32_t cbase, uint32_t d, uint32_t j, uint32_t mv, uint32_t K, F&& f) {
+    uint32_t nb[8], ww[8];
+    if (VEC) {
+        const uint4* c4 = reinterpret_cast<const uint4*>(col) + cbase;
+        const uint4* w4 = reinterpret_cast<const uint4*>(wt) + cbase;
+        const uint32_t q = (d + kChunk - 1) / kChunk;  // chunks of this node
+        uint32_t k, step, kend;
+        if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = j; step = mv; kend = q; }
+        else {
+            const uint32_t per = (K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : K / kChunk;
+            k = j * per; step = 1;
+            kend = (per >= q - k) ? q : k + per;
+        }
+        for (; k < kend; k += 2 * step) {
+            const bool has2 = k + step < kend;
+            const uint4 a = ldg_chunk(c4 + k);
+            const uint4 b = has2 ? ldg_chunk(c4 + k + step) : make_uint4(kPad, kPad, kPad, kPad);
+            uint4 wa = make_uint4(0, 0, 0, 0), wb = wa;
+            if (W) { wa = ldg_chunk(w4 + k); if (has2) wb = ldg_chunk(w4 + k + step); }
+            nb[0] = a.x; nb[1] = a.y; nb[2] = a.z; nb[3] = a.w;
+            nb[4] = b.x; nb[5] = b.y; nb[6] = b.z; nb[7] = b.w;
+            ww[0] = wa.x; ww[1] = wa.y; ww[2] = wa.z; ww[3] = wa.w;
+            ww[4] = wb.x; ww[5] = wb.y; ww[6] = wb.z; ww[7] = wb.w;
+            f(nb, ww);
+        }
+    } else {
+        const uint32_t* cs = col + (uint64_t)cbase * kChunk;
+        const uint32_t* ws = wt + (uint64_t)cbase * kChunk;
+        uint32_t p, step, pend;
+        if (LAYOUT == TIGR_LAYOUT_STRIDED) { p = j; step = mv; pend = d; }
+        else { p = j * K; step = 1; pend = (K >= d - p) ? d : p + K; }
+        while (p < pend) {
+#pragma unroll
+            for (int t = 0; t < 8; ++t) {
+                const uint32_t pt = p + t * step;
+                const bool ok = pt < pend;
+                nb[t] = ok ? ldg_u32(cs + pt) : kPad;
+                ww[t] = (W && ok) ? ldg_u32(ws + pt) : 0;
+            }
+            f(nb, ww);
+            p += 8 * step;
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// relax kernel
+// ------------------------------------------------------------------------------------------
+template <int A>
+__device__ __forceinline__ bool better(uint32_t alt, uint32_t cur) {
+    return A == TIGR_SSWP ? alt > cur : alt < cur;
+}
+
+template <int A>
+__device__ __forceinline__ uint32_t combine(uint32_t x, uint32_t w) {
+    if (A == TIGR_BFS) return x + 1;
+    if (A == TIGR_SSSP) {
+        const uint64_t s = (uint64_t)x + w;
+        return s >= kInf ? kInf - 1 : (uint32_t)s;
+    }
+    if (A == TIGR_CC) return x;
+    return x < w ? x : w;  // SSWP
+}
+
+template <int A, int LAYOUT, bool VEC, int FRONT, bool BSP, bool STATS>
+__global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
+    constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    const uint64_t i = (uint64_t)a.lo + (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
+    const uint32_t it = (FRONT == TIGR_FRONTIER_DENSE) ? a.ctl->it : 0;
+    bool touched = false;
+    uint32_t n_edges = 0, n_upd = 0, n_vn = 0;
+    if (i < a.hi) {
+        const uint32_t v = a.vn_phys[i];
+        bool act = true;
+        if (FRONT == TIGR_FRONTIER_DENSE) act = a.stamp[(uint64_t)(it & 1u) * a.n + v] == it;
+        uint32_t x = 0;
+        if (act) {
+            x = BSP ? a.prev[v] : a.val[v];
+            if (FRONT == TIGR_FRONTIER_NONE) {
+                if ((A == TIGR_BFS || A == TIGR_SSSP) && x == kInf) act = false;
+                if (A == TIGR_SSWP && x == 0) act = false;
+            }
+        }
+        if (act) {
+            const uint4 info = a.vinfo[v];  // {chunk base, degree, first vnode, family size}
+            const uint32_t j = (uint32_t)(i - info.z);
+            if (STATS) n_vn = 1;
+            walk<LAYOUT, VEC, W>(a.col, a.wt, info.x, info.y, j, info.w, a.K,
+                                 [&](const uint32_t* nb, const uint32_t* ww) {
+                uint32_t cur[8];
+#pragma unroll
+                for (int t = 0; t < 8; ++t) cur[t] = (nb[t] != kPad) ? a.val[nb[t]] : 0u;
+#pragma unroll
+                for (int t = 0; t < 8; ++t) {
+                    if (nb[t] == kPad) continue;
+                    if (STATS) ++n_edges;
+                    const uint32_t alt = combine<A>(x, ww[t]);
+                    if (better<A>(alt, cur[t])) {
+                        if (A == TIGR_SSWP) atomicMax(a.val + nb[t], alt);
+                        else atomicMin(a.val + nb[t], alt);
+                        if (FRONT == TIGR_FRONTIER_DENSE) a.stamp[(uint64_t)((it + 1) & 1u) * a.n + nb[t]] = it + 1;
+                        touched = true;
+                        if (STATS) ++n_upd;
+                    }
+                }
+            });
+        }
+    }
+    if (__any_sync(0xffffffffu, touched) && (threadIdx.x & 31) == 0) a.ctl->changed = 1;
+    if (STATS) {
+        unsigned long long e = n_edges, u = n_upd, q = n_vn;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            e += __shfl_xor_sync(0xffffffffu, e, o);
+            u += __shfl_xor_sync(0xffffffffu, u, o);
+            q += __shfl_xor_sync(0xffffffffu, q, o);
+        }
+        if ((threadIdx.x & 31) == 0) {
+            if (e) atomicAdd(&a.ctl->edges, e);
+            if (u) atomicAdd(&a.ctl->updates, u);
+            if (q) atomicAdd(&a.ctl->vnodes, q);
+        }
+    }
+}
+
+template <int LAYOUT, bool VEC, bool STATS>
+__global__ void __launch_bounds__(kRelaxThreads) k_relax_pr(RelaxArgs a) {
+    const uint64_t i = (uint64_t)a.lo + (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
+    uint32_t n_edges = 0;
+    if (i < a.hi) {
+        const uint32_t v = a.vn_phys[i];
+        const double x = a.contrib[v];
+        const uint4 info = a.vinfo[v];
+        const uint32_t j = (uint32_t)(i - info.z);
+        walk<LAYOUT, VEC, false>(a.col, a.wt, info.x, info.y, j, info.w, a.K,
+                                 [&](const uint32_t* nb, const uint32_t*) {
+#pragma unroll
+            for (int t = 0; t < 8; ++t) {
+                if (nb[t] == kPad) continue;
+                atomicAdd(a.acc + nb[t], x);  // RED.ADD.F64 (result unused)
+                if (STATS) ++n_edges;
+            }
+        });
+    }
+    if (STATS) {
+        unsigned long long e = n_edges;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(0xffffffffu, e, o);
+        if ((threadIdx.x & 31) == 0 && e) atomicAdd(&a.ctl->edges, e);
+        if (threadIdx.x == 0 && blockIdx.x == 0) atomicAdd(&a.ctl->vnodes, (unsigned long long)(a.hi - a.lo));
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// dispatch
+// ------------------------------------------------------------------------------------------
+template <int A, int LAYOUT, bool VEC>
+static RelaxFn pick_front(int front, bool bsp, bool stats) {
+#define TIGR_PICK(F, B, S) if (front == F && bsp == B && stats == S) return &k_relax<A, LAYOUT, VEC, F, B, S>;
+    TIGR_PICK(TIGR_FRONTIER_DENSE, false, false)
+    TIGR_PICK(TIGR_FRONTIER_DENSE, false, true)
+    TIGR_PICK(TIGR_FRONTIER_DENSE, true, false)
+    TIGR_PICK(TIGR_FRONTIER_DENSE, true, true)
+    TIGR_PICK(TIGR_FRONTIER_NONE, false, false)
+    TIGR_PICK(TIGR_FRONTIER_NONE, false, true)
+    TIGR_PICK(TIGR_FRONTIER_NONE, true, false)
+    TIGR_PICK(TIGR_FRONTIER_NONE, true, true)
+#undef TIGR_PICK
+    return nullptr;
+}
+
+template <int A>
+static RelaxFn pick_layout(int layout, bool vec, int front, bool bsp, bool stats) {
+    if (layout == TIGR_LAYOUT_STRIDED)
+        return vec ? pick_front<A, TIGR_LAYOUT_STRIDED, true>(front, bsp, stats)
+                   : pick_front<A, TIGR_LAYOUT_STRIDED, false>(front, bsp, stats);
+    return vec ? pick_front<A, TIGR_LAYOUT_CONSECUTIVE, true>(front, bsp, stats)
+               : pick_front<A, TIGR_LAYOUT_CONSECUTIVE, false>(front, bsp, stats);
+}
+
+RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats) {
+    switch (algo) {
+        case TIGR_BFS: return pick_layout<TIGR_BFS>(layout, vec, front, bsp, stats);
+        case TIGR_SSSP: return pick_layout<TIGR_SSSP>(layout, vec, front, bsp, stats);
+        case TIGR_CC: return pick_layout<TIGR_CC>(layout, vec, front, bsp, stats);
+        case TIGR_SSWP: return pick_layout<TIGR_SSWP>(layout, vec, front, bsp, stats);
+        case TIGR_PR:
+            if (layout == TIGR_LAYOUT_STRIDED)
+                return vec ? (stats ? &k_relax_pr<TIGR_LAYOUT_STRIDED, true, true> : &k_relax_pr<TIGR_LAYOUT_STRIDED, true, false>)
+                           : (stats ? &k_relax_pr<TIGR_LAYOUT_STRIDED, false, true> : &k_relax_pr<TIGR_LAYOUT_STRIDED, false, false>);
+            return vec ? (stats ? &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, true, true> : &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, true, false>)
+                       : (stats ? &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, false, true> : &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, false, false>);
+    }
+    return nullptr;
+}
+
+// ------------------------------------------------------------------------------------------
+// init / control / PR apply / multi-GPU diff / assignment dump
+// ------------------------------------------------------------------------------------------
+__global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
+                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v < n) {
+        uint32_t x = kInf;
+        if (algo == TIGR_CC) x = v;
+        else if (algo == TIGR_SSWP) x = 0;
+        if (v == source && algo != TIGR_CC) x = (algo == TIGR_SSWP) ? kInf : 0;
+        val[v] = x;
+        stamp[v] = 0u;                                                   // parity 0
+        stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == source) ? 1u : 0u;  // parity 1: it = 1
+    }
+    if (v == 0) {
+        ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
+        ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
+    }
+}
+
+// end of one iteration: decide whether to continue; sets the graph's WHILE condition
+__global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle) {
+    const uint32_t changed = ctl->changed;
+    uint32_t cont = changed ? 1u : 0u;
+    if (changed && ctl->it >= ctl->max_iters) { cont = 0; ctl->notconv = 1; }
+    ctl->changed = 0;
+    if (cont) ctl->it += 1;
+    ctl->cont = cont;
+    if (use_handle) cudaGraphSetConditional(h, cont);
+}
+
+// multi-GPU: after the all-reduce, activate every node whose replica value moved
+__global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
+                       uint32_t* __restrict__ stamp, Ctl* ctl) {
+    const uint32_t it = ctl->it;
+    bool moved = false;
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v < n) {
+        const uint32_t x = val[v];
+        if (x != prev[v]) { prev[v] = x; stamp[(uint64_t)((it + 1) & 1u) * n + v] = it + 1; moved = true; }
+    }
+    if (__any_sync(0xffffffffu, moved) && (threadIdx.x & 31) == 0) ctl->changed = 1;
+}
+
+__global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
+                          double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    double dang = 0.0;
+    if (v < n) {
+        const double x0 = 1.0 / (double)n;
+        const uint32_t d = deg[v];
+        x[v] = x0;
+        contrib[v] = d ? __ddiv_rn(x0, (double)d) : 0.0;
+        acc[v] = 0.0;
+        if (!d) dang = x0;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) dang += __shfl_xor_sync(0xffffffffu, dang, o);
+    if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(&ctl->dsum[0], dang);
+}
+
+// x = (1-d)/n + d*(acc + dsum/n);  contrib = x/deg;  acc = 0;  next dangling mass -> dsum_next
+__global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double base, double damping,
+                           int dangling, double* __restrict__ x, double* __restrict__ contrib,
+                           double* __restrict__ acc, const double* dsum_cur, double* dsum_next) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    double dang = 0.0;
+    if (v < n) {
+        double s = acc[v];
+        if (dangling) s = __dadd_rn(s, __ddiv_rn(*dsum_cur, (double)n));
+        const double r = __dadd_rn(base, __dmul_rn(damping, s));  // no FMA: matches the oracle
+        const uint32_t d = deg[v];
+        x[v] = r;
+        contrib[v] = d ? __ddiv_rn(r, (double)d) : 0.0;
+        acc[v] = 0.0;
+        if (!d) dang = r;
+    }
+    if (dangling) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) dang += __shfl_xor_sync(0xffffffffu, dang, o);
+        if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(dsum_next, dang);
+    }
+}
+
+// per-vnode edge lists, walked with the relax kernels' own arithmetic (layout parity tests)
+template <int LAYOUT, bool VEC>
+__global__ void k_assign(RelaxArgs a, const uint32_t* __restrict__ offs, uint32_t* __restrict__ counts,
+                         uint32_t* __restrict__ nbr, uint32_t* __restrict__ wout, int weighted, int pass) {
+    const uint64_t i = (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
+    if (i >= a.hi) return;
+    const uint32_t v = a.vn_phys[i];
+    const uint4 info = a.vinfo[v];
+    const uint32_t j = (uint32_t)(i - info.z);
+    uint32_t c = 0;
+    const uint32_t base = pass ? offs[i] : 0;
+    const uint32_t* wt = weighted ? a.wt : a.col;
+    walk<LAYOUT, VEC, true>(a.col, wt, info.x, info.y, j, info.w, a.K,
+                            [&](const uint32_t* nb, const uint32_t* ww) {
+        for (int t = 0; t < 8; ++t) {
+            if (nb[t] == kPad) continue;
+            if (pass) {
+                nbr[base + c] = nb[t];
+                if (wout && weighted) wout[base + c] = ww[t];
+            }
+            ++c;
+        }
+    });
+    if (!pass) counts[i] = c;
+}
+
+AssignFn assign_kernel(int layout, bool vec) {
+    if (layout == TIGR_LAYOUT_STRIDED) return vec ? &k_assign<TIGR_LAYOUT_STRIDED, true> : &k_assign<TIGR_LAYOUT_STRIDED, false>;
+    return vec ? &k_assign<TIGR_LAYOUT_CONSECUTIVE, true> : &k_assign<TIGR_LAYOUT_CONSECUTIVE, false>;
+}
+
+}  // namespace tigr

@@ -1,0 +1,42 @@
+// relax.cuh -- kernel argument block and kernel-pointer dispatch for relax.cu (internal).
+#pragma once
+
+#include "internal.cuh"
+#include "vgraph.cuh"
+
+namespace tigr {
+
+constexpr int kRelaxThreads = 256;
+
+struct RelaxArgs {
+    const uint32_t* __restrict__ vn_phys;
+    const uint4* __restrict__ vinfo;
+    const uint32_t* __restrict__ col;
+    const uint32_t* __restrict__ wt;
+    uint32_t lo, hi, K, n;
+    uint32_t* val;               // values, updated in place with atomics
+    const uint32_t* prev;        // BSP snapshot
+    uint32_t* stamp;             // uint32[2n] worklist stamps
+    double* acc;                 // PR accumulator (RED.ADD.F64 target)
+    const double* contrib;       // PR x/deg
+    Ctl* ctl;
+};
+
+typedef void (*RelaxFn)(RelaxArgs);
+typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
+
+RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats);
+AssignFn assign_kernel(int layout, bool vec);
+
+__global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
+                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters);
+__global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle);
+__global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
+                       uint32_t* __restrict__ stamp, Ctl* ctl);
+__global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
+                          double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl);
+__global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double base, double damping,
+                           int dangling, double* __restrict__ x, double* __restrict__ contrib,
+                           double* __restrict__ acc, const double* dsum_cur, double* dsum_next);
+
+}  // namespace tigr

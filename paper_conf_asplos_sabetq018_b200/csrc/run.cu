@@ -1,0 +1,359 @@
+// run.cu -- host orchestration of one algorithm run (SURVEY.md §3 "Build entry points" 3).
+//
+// Frontier algorithms (BFS/SSSP/CC/SSWP) iterate  [BSP snapshot] -> relax -> [all-reduce ->
+// diff] -> control  until no value changes (the paper's `finished` flag, Alg. 2/3, and the
+// BSP halting rule, §2.1).  By default the loop is ONE CUDA graph launch: the body is
+// captured into the body graph of a conditional WHILE node and k_control sets the condition
+// on the device, so there is no host round trip per iteration (the paper copies `finished`
+// back every iteration).  PageRank runs pr_iters x (relax -> [all-reduce] -> apply).
+#include <algorithm>
+#include <vector>
+
+#include "internal.cuh"
+#include "relax.cuh"
+#include "vgraph.cuh"
+
+namespace tigr {
+
+tigr_status comm_allreduce(tigr_comm* c, void* buf, size_t count, int algo, cudaStream_t s);
+
+Workspace::~Workspace() {
+    for (auto& kv : graphs) {
+        if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
+        if (kv.second.stream) cudaStreamDestroy(kv.second.stream);
+    }
+    for (auto& e : ev)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : tev) cudaEventDestroy(e);
+    if (ctl_host) cudaFreeHost(ctl_host);
+}
+
+namespace {
+
+tigr_status ensure_ws(tigr_vgraph* vg, bool pr) {
+    Workspace& ws = vg->ws;
+    const size_t n = vg->g->n ? vg->g->n : 1;
+    if (!ws.ctl.p) {
+        TIGR_TRY(ws.ctl.alloc(sizeof(Ctl)));
+        TIGR_CK(cudaMallocHost(&ws.ctl_host, sizeof(Ctl)));
+        for (auto& e : ws.ev) TIGR_CK(cudaEventCreate(&e));
+    }
+    if (pr) {
+        if (!ws.x.p) {
+            TIGR_TRY(ws.x.alloc(sizeof(double) * n));
+            TIGR_TRY(ws.contrib.alloc(sizeof(double) * n));
+            TIGR_TRY(ws.acc.alloc(sizeof(double) * n));
+        }
+    } else if (!ws.val.p) {
+        TIGR_TRY(ws.val.alloc(sizeof(uint32_t) * n));
+        TIGR_TRY(ws.prev.alloc(sizeof(uint32_t) * n));
+        TIGR_TRY(ws.stamp.alloc(sizeof(uint32_t) * 2 * n));
+    }
+    return TIGR_OK;
+}
+
+RelaxArgs make_args(tigr_vgraph* vg) {
+    const tigr_graph* g = vg->g;
+    RelaxArgs a;
+    a.vn_phys = vg->vn_phys.as<uint32_t>();
+    a.vinfo = vg->vinfo.as<uint4>();
+    a.col = g->col.as<uint32_t>();
+    a.wt = g->weighted ? g->wt.as<uint32_t>() : g->col.as<uint32_t>();
+    a.lo = vg->lo;
+    a.hi = vg->hi;
+    a.K = vg->K;
+    a.n = g->n;
+    a.val = vg->ws.val.as<uint32_t>();
+    a.prev = vg->ws.prev.as<uint32_t>();
+    a.stamp = vg->ws.stamp.as<uint32_t>();
+    a.acc = vg->ws.acc.as<double>();
+    a.contrib = vg->ws.contrib.as<double>();
+    a.ctl = vg->ws.ctl.as<Ctl>();
+    return a;
+}
+
+struct FrontierPlan {
+    RelaxFn relax;
+    RelaxArgs args;
+    unsigned grid;
+    bool bsp, comm;
+    int algo;
+    tigr_comm* c;
+    uint32_t n;
+};
+
+// enqueue one iteration body; returns number of kernels it launches
+tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditionalHandle h, int use_handle,
+                         int* kernels, cudaEvent_t ev_a = nullptr, cudaEvent_t ev_b = nullptr) {
+    int k = 0;
+    if (p.bsp && !p.comm)
+        TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * p.n, cudaMemcpyDeviceToDevice, s));
+    if (ev_a) TIGR_CK(cudaEventRecord(ev_a, s));
+    if (p.grid) {
+        p.relax<<<p.grid, kRelaxThreads, 0, s>>>(p.args);
+        TIGR_CK(cudaGetLastError());
+        ++k;
+    }
+    if (ev_b) TIGR_CK(cudaEventRecord(ev_b, s));
+    if (p.comm) {
+        TIGR_TRY(comm_allreduce(p.c, p.args.val, p.n, p.algo, s));
+        // the local `changed` flag is rank-local: reset it so k_control only sees k_diff's verdict
+        TIGR_CK(cudaMemsetAsync(&p.args.ctl->changed, 0, sizeof(uint32_t), s));
+        k_diff<<<grid_for(p.n), kBlock, 0, s>>>(p.n, p.args.val, (uint32_t*)p.args.prev, p.args.stamp, p.args.ctl);
+        TIGR_CK(cudaGetLastError());
+        ++k;
+    }
+    k_control<<<1, 1, 0, s>>>(p.args.ctl, h, use_handle);
+    TIGR_CK(cudaGetLastError());
+    ++k;
+    *kernels = k;
+    return TIGR_OK;
+}
+
+tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_run_opts& o, cudaStream_t s,
+                         tigr_stats* st) {
+    Workspace& ws = vg->ws;
+    const uint32_t n = vg->g->n;
+    int front = o.frontier == TIGR_FRONTIER_AUTO ? TIGR_FRONTIER_DENSE : o.frontier;
+    FrontierPlan p;
+    p.bsp = o.schedule == 1;
+    p.comm = o.comm != nullptr && o.comm->nranks > 1;
+    p.c = o.comm;
+    p.algo = algo;
+    p.n = n;
+    p.relax = relax_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0);
+    if (!p.relax) return fail(TIGR_EUNSUPPORTED, "no relax kernel for this option combination");
+    p.args = make_args(vg);
+    p.grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + kRelaxThreads - 1) / kRelaxThreads);
+    const uint32_t max_iters = o.max_iters ? o.max_iters : (n + 1 > n ? n + 1 : n);
+
+    cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
+    TIGR_CK(cudaEventRecord(t0, s));
+    k_init<<<grid_for(n), kBlock, 0, s>>>(algo, n, source, p.args.val, p.args.stamp, p.args.ctl, max_iters);
+    TIGR_CKL("init");
+    if (p.bsp || p.comm)
+        TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
+
+    int kpi = 0;
+    uint32_t launches = 0;
+    double ms_relax = 0.0;
+    // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
+    const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
+    if (use_graph) {
+        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0), front, p.bsp ? 1 : 0, o.collect_stats ? 1 : 0,
+                     p.comm ? 1 : 0, vg->lo, vg->hi};
+        auto itg = ws.graphs.find(key);
+        if (itg == ws.graphs.end()) {
+            CachedGraph cg;
+            TIGR_CK(cudaStreamCreateWithFlags(&cg.stream, cudaStreamNonBlocking));
+            cudaGraph_t g;
+            TIGR_CK(cudaGraphCreate(&g, 0));
+            cudaGraphConditionalHandle h;
+            TIGR_CK(cudaGraphConditionalHandleCreate(&h, g, 1, cudaGraphCondAssignDefault));
+            cudaGraphNodeParams cp = {};
+            cp.type = cudaGraphNodeTypeConditional;
+            cp.conditional.handle = h;
+            cp.conditional.type = cudaGraphCondTypeWhile;
+            cp.conditional.size = 1;
+            cudaGraphNode_t node;
+            TIGR_CK(cudaGraphAddNode(&node, g, nullptr, 0, &cp));
+            cudaGraph_t body = cp.conditional.phGraph_out[0];
+            TIGR_CK(cudaStreamBeginCaptureToGraph(cg.stream, body, nullptr, nullptr, 0,
+                                                  cudaStreamCaptureModeThreadLocal));
+            tigr_status bst = enqueue_body(p, cg.stream, h, 1, &cg.kernels_per_iter);
+            cudaGraph_t captured = nullptr;
+            cudaError_t ce = cudaStreamEndCapture(cg.stream, &captured);
+            if (bst != TIGR_OK) { cudaGraphDestroy(g); return bst; }
+            if (ce != cudaSuccess) { cudaGraphDestroy(g); return cuda_fail(ce, "graph capture", __FILE__, __LINE__); }
+            ce = cudaGraphInstantiate(&cg.exec, g, 0);
+            cudaGraphDestroy(g);
+            if (ce != cudaSuccess) return cuda_fail(ce, "graph instantiate", __FILE__, __LINE__);
+            itg = ws.graphs.emplace(key, cg).first;
+        }
+        CachedGraph& cg = itg->second;
+        kpi = cg.kernels_per_iter;
+        TIGR_CK(cudaEventRecord(ws.ev[2], s));
+        TIGR_CK(cudaStreamWaitEvent(cg.stream, ws.ev[2], 0));
+        TIGR_CK(cudaGraphLaunch(cg.exec, cg.stream));
+        TIGR_CK(cudaEventRecord(ws.ev[3], cg.stream));
+        TIGR_CK(cudaStreamWaitEvent(s, ws.ev[3], 0));
+    } else {
+        for (;;) {
+            int k = 0;
+            TIGR_TRY(enqueue_body(p, s, 0, 0, &k, o.time_kernels ? ws.ev[2] : nullptr,
+                                  o.time_kernels ? ws.ev[3] : nullptr));
+            count_launch(k);
+            launches += p.grid ? 1 : 0;
+            TIGR_CK(cudaMemcpyAsync(ws.ctl_host, p.args.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+            TIGR_CK(cudaStreamSynchronize(s));
+            if (o.time_kernels && p.grid) {
+                float ms = 0.f;
+                TIGR_CK(cudaEventElapsedTime(&ms, ws.ev[2], ws.ev[3]));
+                ms_relax += ms;
+            }
+            if (!ws.ctl_host->cont) break;
+        }
+    }
+    TIGR_CK(cudaEventRecord(t1, s));
+    TIGR_CK(cudaMemcpyAsync(ws.ctl_host, p.args.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    const Ctl& c = *ws.ctl_host;
+    if (use_graph) {
+        count_launch((uint64_t)c.it * kpi);
+        launches = p.grid ? c.it : 0;
+    }
+    if (st) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, t0, t1);
+        st->iterations = c.it;
+        st->relax_launches = launches;
+        st->edges_processed = c.edges;
+        st->updates = c.updates;
+        st->active_vnodes = c.vnodes;
+        st->ms_total = ms;
+        st->ms_relax = ms_relax;
+    }
+    if (c.notconv) return fail(TIGR_ENOTCONV, "max_iters reached before the fixed point");
+    return TIGR_OK;
+}
+
+tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr_stats* st) {
+    Workspace& ws = vg->ws;
+    const uint32_t n = vg->g->n;
+    RelaxArgs a = make_args(vg);
+    RelaxFn relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
+    const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + kRelaxThreads - 1) / kRelaxThreads);
+    const bool comm = o.comm != nullptr && o.comm->nranks > 1;
+    const double base = (1.0 - o.pr_damping) / (double)n;
+    cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
+    TIGR_CK(cudaEventRecord(t0, s));
+    TIGR_CK(cudaMemsetAsync(a.ctl, 0, sizeof(Ctl), s));
+    k_pr_init<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), ws.x.as<double>(), ws.contrib.as<double>(),
+                                             ws.acc.as<double>(), a.ctl);
+    TIGR_CKL("pr init");
+    double ms_relax = 0.0, ms_ex = 0.0;
+    uint32_t launches = 0;
+    if (o.time_kernels) {  // 3 events per iteration: relax start / relax end / exchange end
+        while (ws.tev.size() < 3 * (size_t)o.pr_iters) {
+            cudaEvent_t e;
+            TIGR_CK(cudaEventCreate(&e));
+            ws.tev.push_back(e);
+        }
+    }
+    for (uint32_t t = 0; t < o.pr_iters; ++t) {
+        if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t], s));
+        if (grid) {
+            relax<<<grid, kRelaxThreads, 0, s>>>(a);
+            TIGR_CKL("pr relax");
+            ++launches;
+        }
+        if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t + 1], s));
+        if (comm) TIGR_TRY(comm_allreduce(o.comm, ws.acc.p, n, TIGR_PR, s));
+        if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t + 2], s));
+        double* dcur = &a.ctl->dsum[t & 1];
+        double* dnext = &a.ctl->dsum[(t + 1) & 1];
+        if (o.pr_dangling) TIGR_CK(cudaMemsetAsync(dnext, 0, sizeof(double), s));
+        k_pr_apply<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), base, o.pr_damping, o.pr_dangling,
+                                                  ws.x.as<double>(), ws.contrib.as<double>(), ws.acc.as<double>(),
+                                                  dcur, dnext);
+        TIGR_CKL("pr apply");
+    }
+    TIGR_CK(cudaEventRecord(t1, s));
+    TIGR_CK(cudaMemcpyAsync(ws.ctl_host, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    if (o.time_kernels) {
+        for (uint32_t t = 0; t < o.pr_iters; ++t) {
+            float ms = 0.f;
+            TIGR_CK(cudaEventElapsedTime(&ms, ws.tev[3 * t], ws.tev[3 * t + 1]));
+            ms_relax += ms;
+            TIGR_CK(cudaEventElapsedTime(&ms, ws.tev[3 * t + 1], ws.tev[3 * t + 2]));
+            ms_ex += ms;
+        }
+    }
+    if (st) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, t0, t1);
+        st->iterations = o.pr_iters;
+        st->relax_launches = launches;
+        st->edges_processed = ws.ctl_host->edges;
+        st->updates = 0;
+        st->active_vnodes = ws.ctl_host->vnodes;
+        st->ms_total = ms;
+        st->ms_relax = ms_relax;
+        st->ms_exchange = ms_ex;
+    }
+    return TIGR_OK;
+}
+
+}  // namespace
+
+tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tigr_run_opts& o, void* out,
+                       int out_is_device, tigr_stats* st) {
+    const tigr_graph* g = vg->g;
+    if ((int)algo < TIGR_BFS || (int)algo > TIGR_PR) return fail(TIGR_EINVAL, "run: unknown algorithm");
+    if ((algo == TIGR_BFS || algo == TIGR_SSSP || algo == TIGR_SSWP) && source >= g->n)
+        return fail(TIGR_EINVAL, "run: source >= n");
+    if ((algo == TIGR_SSSP || algo == TIGR_SSWP) && !g->weighted)
+        return fail(TIGR_EINVAL, "run: SSSP/SSWP need a weighted graph");
+    if (algo == TIGR_CC && !g->symmetric)
+        return fail(TIGR_EINVAL, "run: CC needs a symmetric graph (build with symmetrize=1)");
+    if (algo == TIGR_PR && !(o.pr_damping >= 0.0 && o.pr_damping <= 1.0))
+        return fail(TIGR_EINVAL, "run: pr_damping outside [0, 1]");
+    if (o.frontier < TIGR_FRONTIER_AUTO || o.frontier > TIGR_FRONTIER_NONE)
+        return fail(TIGR_EINVAL, "run: unknown frontier mode");
+    cudaStream_t s = (cudaStream_t)o.stream;
+    if (st) *st = tigr_stats{};
+    if (g->n == 0) return TIGR_OK;
+    TIGR_TRY(ensure_ws(vg, algo == TIGR_PR));
+    tigr_status rs = (algo == TIGR_PR) ? run_pr(vg, o, s, st) : run_frontier(vg, algo, source, o, s, st);
+    if (rs != TIGR_OK && rs != TIGR_ENOTCONV) return rs;
+    const void* res = (algo == TIGR_PR) ? vg->ws.x.p : vg->ws.val.p;
+    const size_t bytes = (size_t)g->n * (algo == TIGR_PR ? sizeof(double) : sizeof(uint32_t));
+    if (out) {
+        TIGR_CK(cudaMemcpyAsync(out, res, bytes, out_is_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
+        TIGR_CK(cudaStreamSynchronize(s));
+    }
+    return rs;
+}
+
+// per-vnode edge lists through the relax kernels' walk (layout parity)
+tigr_status assignment_device(const tigr_vgraph* vgc, uint32_t* counts, uint32_t* nbr, uint32_t* w,
+                              cudaStream_t s) {
+    tigr_vgraph* vg = const_cast<tigr_vgraph*>(vgc);
+    if (vg->nv == 0) return TIGR_OK;
+    RelaxArgs a = make_args(vg);
+    a.lo = 0;
+    a.hi = (uint32_t)vg->nv;
+    AssignFn f = assign_kernel(vg->layout, vg->vec);
+    const unsigned grid = (unsigned)((vg->nv + kRelaxThreads - 1) / kRelaxThreads);
+    TmpBuf offs;
+    TIGR_TRY(offs.alloc(sizeof(uint32_t) * (vg->nv + 1), s));
+    f<<<grid, kRelaxThreads, 0, s>>>(a, nullptr, counts, nullptr, nullptr, vg->g->weighted, 0);
+    TIGR_CKL("assign count");
+    TIGR_TRY(exclusive_scan_u32(counts, vg->nv, SCAN_U32, 1, offs.as<uint32_t>(), s, nullptr));
+    f<<<grid, kRelaxThreads, 0, s>>>(a, offs.as<uint32_t>(), counts, nbr, w, vg->g->weighted, 1);
+    TIGR_CKL("assign fill");
+    return TIGR_OK;
+}
+
+// contiguous, family-aligned vnode ranges with ~equal edge counts
+tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank) {
+    if (nranks < 1 || rank < 0 || rank >= nranks) return fail(TIGR_EINVAL, "partition: bad rank/nranks");
+    const tigr_graph* g = vg->g;
+    if (nranks == 1 || g->n == 0) { vg->lo = 0; vg->hi = (uint32_t)vg->nv; return TIGR_OK; }
+    std::vector<int64_t> rp((size_t)g->n + 1);
+    std::vector<uint32_t> vp((size_t)g->n + 1);
+    TIGR_CK(cudaMemcpy(rp.data(), g->row_ptr.p, sizeof(int64_t) * rp.size(), cudaMemcpyDeviceToHost));
+    TIGR_CK(cudaMemcpy(vp.data(), vg->vnode_ptr.p, sizeof(uint32_t) * vp.size(), cudaMemcpyDeviceToHost));
+    auto cut = [&](int r) -> uint32_t {  // first vertex whose edge prefix reaches r/nranks of m
+        if (r <= 0) return 0;
+        if (r >= nranks) return g->n;
+        const int64_t target = (int64_t)((__int128)g->m * r / nranks);
+        return (uint32_t)(std::lower_bound(rp.begin(), rp.end() - 1, target) - rp.begin());
+    };
+    vg->lo = vp[cut(rank)];
+    vg->hi = vp[cut(rank + 1)];
+    return TIGR_OK;
+}
+
+}  // namespace tigr

@@ -1,0 +1,69 @@
+// vgraph.cuh -- the virtual graph handle and its run workspace (internal).
+#pragma once
+
+#include <map>
+#include <vector>
+#include <tuple>
+
+#include "internal.cuh"
+
+namespace tigr {
+
+// Device-side control block of one run (one per vgraph workspace).
+struct Ctl {
+    uint32_t changed;      // set by relax when any value improved this iteration
+    uint32_t it;           // current iteration (1-based; node v is active iff stamp[v] == it)
+    uint32_t max_iters;
+    uint32_t cont;         // 1 while the loop should continue (host-loop mode reads it)
+    uint32_t notconv;      // 1 if the cap was hit while values still changed
+    uint32_t pad[3];
+    unsigned long long edges, updates, vnodes;
+    double dsum[2];        // PR: dangling mass of the iterate (parity of the iteration)
+};
+
+struct GraphKey {
+    int algo, layout_vec, frontier, schedule, stats, comm;
+    uint32_t lo, hi;
+    bool operator<(const GraphKey& o) const {
+        return std::tie(algo, layout_vec, frontier, schedule, stats, comm, lo, hi) <
+               std::tie(o.algo, o.layout_vec, o.frontier, o.schedule, o.stats, o.comm, o.lo, o.hi);
+    }
+};
+
+struct CachedGraph {
+    cudaGraphExec_t exec = nullptr;
+    cudaStream_t stream = nullptr;
+    int kernels_per_iter = 0;
+};
+
+struct Workspace {
+    DevBuf val;      // uint32[n] values (BFS/SSSP/CC/SSWP)
+    DevBuf prev;     // uint32[n] BSP snapshot / multi-GPU pre-exchange copy
+    DevBuf stamp;    // uint32[2n] worklist: node v active in iteration it iff stamp[(it&1)n + v] == it;
+                     // relax(it) writes only the other parity, so activations never race reads
+    DevBuf x;        // double[n] PR rank
+    DevBuf contrib;  // double[n] PR x/deg
+    DevBuf acc;      // double[n] PR accumulator
+    DevBuf ctl;      // Ctl
+    Ctl* ctl_host = nullptr;  // pinned mirror for the host loop
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    std::vector<cudaEvent_t> tev;  // per-relax-launch timing events (time_kernels)
+    std::map<GraphKey, CachedGraph> graphs;
+    ~Workspace();
+};
+
+}  // namespace tigr
+
+struct tigr_vgraph {
+    const tigr_graph* g = nullptr;
+    uint32_t K = 8;
+    tigr_layout layout = TIGR_LAYOUT_STRIDED;
+    bool vec = true;             // 16-byte chunk units (4 | K)
+    uint64_t nv = 0;
+    tigr::DevBuf vnode_ptr;      // uint32[n+1]
+    tigr::DevBuf vn_phys;        // uint32[nv]
+    tigr::DevBuf vinfo;          // uint4[n] = {chunk base, degree, first vnode, family size}
+    uint32_t lo = 0, hi = 0;     // this rank's vnode range
+    double ms_build = 0.0;
+    tigr::Workspace ws;
+};

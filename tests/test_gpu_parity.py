@@ -1,0 +1,307 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded
+inputs.  Bit-exact for generator / CSR / virtual split / BFS / SSSP / CC / SSWP; PageRank
+within 1e-6 max abs per vertex (BASELINE.json north_star).  Where several results are
+correct (the order of arcs inside a CSR segment, hence which arcs a virtual node owns) the
+unique part is compared exactly and the rest is checked for validity."""
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+INF = 0xFFFFFFFF
+
+
+@pytest.fixture(scope="module")
+def tigr():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_asplos_sabetq018_b200 as t
+    return t
+
+
+def _u32(t):
+    return t.cpu().numpy().view(np.uint32)
+
+
+def _dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a).view(np.int32)).cuda()
+
+
+# ------------------------------------------------------------------------------------ a0
+@pytest.mark.parametrize("cfg", ["cfg1", "cfg2", "cfg3"])
+def test_generator_bit_exact(tigr, cfg):
+    rec = graphgen.recipe(cfg)
+    m = min(rec.m, 1 << 24)
+    src, dst, w = graphgen.rmat(rec.n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax)
+    ds = torch.empty(m, dtype=torch.int32, device="cuda")
+    dd, dw = torch.empty_like(ds), torch.empty_like(ds)
+    tigr.tigr_rmat_coo(rec.n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, ds, dd, dw)
+    torch.cuda.synchronize()
+    assert np.array_equal(_u32(ds), src) and np.array_equal(_u32(dd), dst) and np.array_equal(_u32(dw), w)
+
+
+def test_generator_full_scale_sampled(tigr):
+    """cfg5 (1.47B arcs): a prefix and a far slice, drawn on both sides (counter-based)."""
+    rec = graphgen.recipe("cfg5")
+    m = 1 << 20
+    ds = torch.empty(m, dtype=torch.int32, device="cuda")
+    dd, dw = torch.empty_like(ds), torch.empty_like(ds)
+    tigr.tigr_rmat_coo(rec.n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, ds, dd, dw)
+    src, dst, w = graphgen.rmat(rec.n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax)
+    assert np.array_equal(_u32(ds), src) and np.array_equal(_u32(dd), dst) and np.array_equal(_u32(dw), w)
+
+
+# ------------------------------------------------------------------------------------ a1
+def _canon(rp, col, w):
+    """Per-segment sort by (col, w): the unique content of a CSR with unordered segments."""
+    n = len(rp) - 1
+    seg = np.repeat(np.arange(n), np.diff(rp))
+    keys = (col, seg) if w is None else (w, col, seg)
+    order = np.lexsort(keys)
+    return col[order], (None if w is None else w[order])
+
+
+@pytest.mark.parametrize("sym", [False, True])
+def test_csr_build_matches_oracle(tigr, sym):
+    rec = graphgen.recipe("cfg2")
+    src, dst, w = graphgen.rmat(rec.n, rec.m // 2, rec.a, rec.b, rec.c, rec.seed, rec.wseed)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w, symmetrize=sym)
+    rp, col, wt = tigr.tigr_graph_export_csr(g)
+    o = oracle.csr_build(rec.n, *(oracle.symmetrize(src, dst, w) if sym else (src, dst, w)))
+    assert np.array_equal(rp, o.row_ptr)
+    c1, w1 = _canon(rp, col, wt)
+    c2, w2 = _canon(o.row_ptr, o.col, o.wt)
+    assert np.array_equal(c1, c2) and np.array_equal(w1, w2)
+
+
+def test_csr_from_csr_roundtrip(tigr):
+    src, dst, w = graphgen.random_small(300, 4000, 5)
+    o = oracle.csr_build(300, src, dst, w)
+    g = tigr.tigr_graph_from_csr(300, o.row_ptr, o.col, o.wt)
+    rp, col, wt = tigr.tigr_graph_export_csr(g)
+    assert np.array_equal(rp, o.row_ptr) and np.array_equal(col, o.col) and np.array_equal(wt, o.wt)
+
+
+# ------------------------------------------------------------------------------------ a2-a5
+@pytest.mark.parametrize("K", [1, 3, 4, 8, 32, 0xFFFFFFFF])
+@pytest.mark.parametrize("layout", ["consecutive", "strided"])
+def test_virtual_split_and_assignment(tigr, K, layout):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(g, K, layout)
+    vp, ph = tigr.tigr_vgraph_export(vg)
+    rp, col, wt = tigr.tigr_graph_export_csr(g)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    ov = oracle.Virtual(o, K)
+    assert np.array_equal(vp, ov.vnode_ptr.astype(np.uint32)) and np.array_equal(ph, ov.vn_phys)
+    counts, nbr, ww = tigr.tigr_vgraph_assignment(vg)
+    # the unit of the layout: 16-byte chunks (4 edges) when 4 | K
+    chunk = 4 if (K % 4 == 0 or K == 0xFFFFFFFF) else 1
+    lay = 0 if layout == "consecutive" else 1
+    want = np.array([len(ov.edges(i, lay, chunk)) for i in range(ov.nv)], dtype=np.uint32)
+    assert np.array_equal(counts, want)
+    assert counts.max() <= K
+    # every arc exactly once: a family's arcs are its node's segment (as multisets)
+    offs = np.concatenate([[0], np.cumsum(counts.astype(np.int64))])
+    for v in np.flatnonzero(np.diff(o.row_ptr)):
+        a, b = offs[vp[v]], offs[vp[v + 1]]
+        got = sorted(zip(nbr[a:b].tolist(), ww[a:b].tolist()))
+        exp = sorted(zip(o.col[o.row_ptr[v]:o.row_ptr[v + 1]].tolist(), o.wt[o.row_ptr[v]:o.row_ptr[v + 1]].tolist()))
+        assert got == exp, v
+    # the device's own segment order: vnode i owns exactly the oracle's positions in it
+    for i in range(0, ov.nv, max(1, ov.nv // 200)):
+        v = int(ph[i])
+        pos = ov.edges(i, lay, chunk) - o.row_ptr[v]
+        seg = col[rp[v]:rp[v + 1]]
+        assert sorted(nbr[offs[i]:offs[i + 1]].tolist()) == sorted(seg[pos].tolist()), i
+
+
+# ------------------------------------------------------------------------------------ a6-a9
+def _oracle_all(n, src, dst, w, source=0):
+    o = oracle.csr_build(n, src, dst, w)
+    return {"bfs": oracle.bfs(o, source), "sssp": oracle.sssp(o, source), "sswp": oracle.sswp(o, source),
+            "cc": oracle.cc(n, src, dst), "pr": oracle.pagerank(o, 20)}
+
+
+def _run_all(tigr, n, src, dst, w, K=8, layout="strided", source=0, **kw):
+    g = tigr.tigr_graph_from_coo(n, src, dst, w)
+    gs = tigr.tigr_graph_from_coo(n, src, dst, None, symmetrize=True)
+    vg = tigr.tigr_virtualize(g, K, layout)
+    vgs = tigr.tigr_virtualize(gs, K, layout)
+    out = {a: tigr.tigr_run(vg, a, source, **kw) for a in ("bfs", "sssp", "sswp")}
+    out["cc"] = tigr.tigr_run(vgs, "cc", **kw)
+    prkw = {k: v for k, v in kw.items() if k not in ("schedule", "frontier")}
+    out["pr"] = tigr.tigr_run(vg, "pr", **prkw)
+    return out
+
+
+def _assert_parity(got, want):
+    for a in ("bfs", "sssp", "sswp", "cc"):
+        assert np.array_equal(got[a], want[a]), a
+    err = np.abs(got["pr"] - want["pr"]).max() if len(want["pr"]) else 0.0
+    assert err <= 1e-6, err
+
+
+@pytest.mark.parametrize("K", [1, 4, 8, 32, 0xFFFFFFFF])
+@pytest.mark.parametrize("layout", ["consecutive", "strided"])
+def test_cfg1_all_algorithms(tigr, K, layout):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    _assert_parity(_run_all(tigr, rec.n, src, dst, w, K, layout), _oracle_all(rec.n, src, dst, w))
+
+
+@pytest.mark.parametrize("schedule,frontier,use_graph", [(0, 1, 1), (1, 1, 1), (0, 2, 1), (1, 2, 0), (0, 1, 0)])
+def test_cfg1_schedules(tigr, schedule, frontier, use_graph):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    got = _run_all(tigr, rec.n, src, dst, w, schedule=schedule, frontier=frontier, use_graph=use_graph)
+    _assert_parity(got, _oracle_all(rec.n, src, dst, w))
+
+
+def test_bsp_iterations_match_paper_literal_push(tigr):
+    """Table 8 (L1480-1486): BSP #iterations are the same for the original graph and every
+    virtual split; and equal to the oracle's paper-literal sequential push (BSP, worklist)."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    for algo, code in (("bfs", oracle.BFS), ("sssp", oracle.SSSP), ("sswp", oracle.SSWP)):
+        _, want_it, _ = oracle.push_virtual(o, oracle.Virtual(o, 8), code, 0, schedule=1, worklist=1)
+        for K in (1, 8, 0xFFFFFFFF):
+            g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+            vg = tigr.tigr_virtualize(g, K, "strided")
+            vals, st = tigr.tigr_run(vg, algo, 0, schedule=1, return_stats=True)
+            assert st["iterations"] == want_it, (algo, K, st["iterations"], want_it)
+
+
+def test_cfg2_bfs_cc(tigr):
+    rec = graphgen.recipe("cfg2")
+    src, dst, _ = graphgen.generate(rec, weighted=False)
+    g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False)
+    gs = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False,
+                              symmetrize=True)
+    vg = tigr.tigr_virtualize(g, 8)
+    vgs = tigr.tigr_virtualize(gs, 8)
+    o = oracle.csr_build(rec.n, src, dst)
+    assert np.array_equal(tigr.tigr_run(vg, "bfs", 0), oracle.bfs(o, 0))
+    assert np.array_equal(tigr.tigr_run(vgs, "cc"), oracle.cc(rec.n, src, dst))
+
+
+# ------------------------------------------------------------------------------------ edge cases
+def _edge_cases():
+    cases = {}
+    cases["single_vertex"] = (1, [], [], [])
+    cases["no_edges"] = (5, [], [], [])
+    cases["self_loops_dups"] = (4, [0, 0, 0, 1, 1, 2], [0, 1, 1, 1, 2, 2], [3, 5, 2, 1, 7, 4])
+    cases["source_deg0"] = (4, [1, 2], [2, 3], [1, 1])
+    cases["two_components"] = (6, [0, 1, 3, 4], [1, 2, 4, 5], [2, 2, 9, 9])
+    cases["cycle"] = (7, list(range(7)), [(i + 1) % 7 for i in range(7)], [1, 2, 3, 4, 5, 6, 7])
+    star = 70000  # hub with d >> 32K
+    cases["hub"] = (star + 1, [0] * star + list(range(1, star + 1)), list(range(1, star + 1)) + [0] * star,
+                    [(i % 64) + 1 for i in range(2 * star)])
+    for d in (7, 8, 9, 16, 17, 257):  # d around K and 32K+1 for K = 8
+        cases[f"deg{d}"] = (d + 2, [0] * d + [1], list(range(1, d + 1)) + [d + 1], [(3 * i) % 64 + 1 for i in range(d + 1)])
+    k = 12
+    cases["complete"] = (k, [i for i in range(k) for j in range(k) if i != j],
+                         [j for i in range(k) for j in range(k) if i != j], [((i * 7 + j) % 64) + 1 for i in range(k) for j in range(k) if i != j])
+    return cases
+
+
+@pytest.mark.parametrize("name", list(_edge_cases()))
+@pytest.mark.parametrize("K", [1, 8])
+def test_edge_cases(tigr, name, K):
+    n, src, dst, w = _edge_cases()[name]
+    src, dst, w = (np.asarray(x, dtype=np.uint32) for x in (src, dst, w))
+    _assert_parity(_run_all(tigr, n, src, dst, w, K), _oracle_all(n, src, dst, w))
+
+
+def test_unit_weights_sssp_equals_bfs(tigr):
+    src, dst, _ = graphgen.random_small(500, 3000, 11)
+    g = tigr.tigr_graph_from_coo(500, src, dst, np.ones(len(src), np.uint32))
+    vg = tigr.tigr_virtualize(g, 8)
+    assert np.array_equal(tigr.tigr_run(vg, "sssp", 3), tigr.tigr_run(vg, "bfs", 3))
+
+
+def test_pr_dangling_redistribute(tigr):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, None)
+    vg = tigr.tigr_virtualize(g, 8)
+    got = tigr.tigr_run(vg, "pr", pr_dangling=1)
+    want = oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20, 0.85, 1)
+    assert np.abs(got - want).max() <= 1e-6
+    assert abs(got.sum() - 1.0) < 1e-9  # redistribute conserves mass
+
+
+def test_errors(tigr):
+    src, dst, w = graphgen.random_small(10, 30, 1)
+    g = tigr.tigr_graph_from_coo(10, src, dst, None)
+    vg = tigr.tigr_virtualize(g, 8)
+    for bad in (lambda: tigr.tigr_run(vg, "sssp", 0),          # unweighted
+                lambda: tigr.tigr_run(vg, "cc"),                # not symmetric
+                lambda: tigr.tigr_run(vg, "bfs", 10),           # source >= n
+                lambda: tigr.tigr_virtualize(g, 0),             # K = 0
+                lambda: tigr.tigr_graph_from_coo(10, [0, 10], [1, 2]),  # id >= n
+                lambda: tigr.tigr_graph_from_csr(3, np.array([0, 2, 1, 3]), np.array([0, 1, 2]))):
+        with pytest.raises(tigr.TigrError) as ei:
+            bad()
+        assert ei.value.status == tigr.TIGR_EINVAL
+    gw = tigr.tigr_graph_from_coo(10, src, dst, w)
+    vgw = tigr.tigr_virtualize(gw, 8)
+    with pytest.raises(tigr.TigrError) as ei:
+        tigr.tigr_run(vgw, "sssp", 0, max_iters=1)
+    assert ei.value.status == tigr.TIGR_ENOTCONV
+
+
+def test_device_buffers_and_streams(tigr):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        g = tigr.tigr_graph_from_coo(rec.n, _dev(src), _dev(dst), _dev(w), stream=s)
+        vg = tigr.tigr_virtualize(g, 8, stream=s)
+        out = torch.empty(rec.n, dtype=torch.int32, device="cuda")
+        tigr.tigr_run(vg, "sssp", 0, out=out, stream=s)
+        s.synchronize()
+    assert np.array_equal(_u32(out), oracle.sssp(oracle.csr_build(rec.n, src, dst, w), 0))
+    prd = torch.empty(rec.n, dtype=torch.float64, device="cuda")
+    tigr.tigr_run(vg, "pr", out=prd, stream=s)
+    assert np.abs(prd.cpu().numpy() - oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20)).max() <= 1e-6
+
+
+def test_stats_counts(tigr):
+    """collect_stats: PR processes every arc every iteration; frontier runs count edges of
+    active vnodes (BFS in BSP mode = arcs out of each level, i.e. all arcs of reached nodes)."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(g, 8)
+    _, st = tigr.tigr_run(vg, "pr", collect_stats=1, return_stats=True)
+    assert st["edges_processed"] == 20 * rec.m
+    lv, st = tigr.tigr_run(vg, "bfs", 0, schedule=1, collect_stats=1, return_stats=True)
+    deg = np.bincount(src, minlength=rec.n)
+    assert st["edges_processed"] == int(deg[lv != INF].sum())
+
+
+def test_partition_ranges(tigr):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(g, 8)
+    vp, _ = tigr.tigr_vgraph_export(vg)
+    nv = vg.info()["nv"]
+    for P in (2, 3, 8):
+        bounds = []
+        for r in range(P):
+            tigr.tigr_vgraph_partition(vg, P, r)
+            i = vg.info()
+            bounds.append((i["lo"], i["hi"]))
+            assert i["lo"] in set(vp.tolist()) and i["hi"] in set(vp.tolist())  # family-aligned
+        assert bounds[0][0] == 0 and bounds[-1][1] == nv
+        assert all(bounds[r][1] == bounds[r + 1][0] for r in range(P - 1))
+    tigr.tigr_vgraph_partition(vg, 1, 0)
+    assert vg.info()["hi"] == nv

@@ -32,6 +32,54 @@ def build_c_shared(sources: list[str], target: str, extra: list[str] | None = No
     return target
 
 
+NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def _nccl_include() -> list[str]:
+    cands = ["/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/include", "/usr/include"]
+    for c in cands:
+        if os.path.exists(os.path.join(c, "nccl.h")):
+            return ["-I", c]
+    return []
+
+
+def build_tigr(force: bool = False, verbose: bool = False) -> str:
+    """nvcc -gencode arch=compute_100a,code=sm_100a every csrc/*.cu -> libtigr.so (in-tree)."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    pkg = os.path.join(ROOT, "paper_conf_asplos_sabetq018_b200")
+    csrc = os.path.join(pkg, "csrc")
+    target = os.path.join(pkg, "libtigr.so")
+    objdir = os.path.join(ROOT, "build", "obj")
+    os.makedirs(objdir, exist_ok=True)
+    sources = sorted(os.path.join(csrc, f) for f in os.listdir(csrc) if f.endswith(".cu"))
+    headers = sorted(os.path.join(csrc, f) for f in os.listdir(csrc) if f.endswith((".cuh", ".h")))
+    headers.append(os.path.join(ROOT, "include", "tigr.h"))
+    flags = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
+             "--expt-relaxed-constexpr", "--extended-lambda", *ARCH, "-I", os.path.join(ROOT, "include"),
+             *_nccl_include()]
+    if os.environ.get("TIGR_PTXAS_VERBOSE"):
+        flags += ["-Xptxas", "-v"]
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
+        if force or _stale(obj, [src, *headers]):
+            cmd = [NVCC, *flags, "-c", src, "-o", obj]
+            if verbose:
+                print(" ".join(cmd), flush=True)
+            subprocess.run(cmd, check=True)
+        return obj
+
+    with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
+        objs = list(ex.map(compile_one, sources))
+    if force or _stale(target, objs):
+        cmd = [NVCC, *ARCH, "-shared", "-o", target + ".tmp", *objs, "-ldl"]
+        subprocess.run(cmd, check=True)
+        os.replace(target + ".tmp", target)
+    return target
+
+
 if __name__ == "__main__":
     sys.path.insert(0, ROOT)
     import __graft_entry__  # noqa: E402
