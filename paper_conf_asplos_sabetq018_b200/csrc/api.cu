@@ -2,6 +2,7 @@
 // host<->device staging, error state; every compute step runs in the kernels of the other
 // translation units.
 #include <cstdio>
+#include <mutex>
 #include <cstring>
 #include <string>
 
@@ -27,21 +28,36 @@ tigr_status cuda_fail(cudaError_t e, const char* what, const char* file, int lin
     return (e == cudaErrorMemoryAllocation) ? TIGR_ENOMEM : TIGR_ECUDA;
 }
 
-tigr_status DevBuf::alloc(size_t nbytes) {
+void init_pool() {
+    static std::once_flag once;
+    std::call_once(once, [] {
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess) return;
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) != cudaSuccess) return;
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    });
+}
+
+tigr_status DevBuf::alloc(size_t nbytes, cudaStream_t stream) {
     release();
-    cudaError_t e = cudaMalloc(&p, nbytes ? nbytes : 16);
-    if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMalloc", __FILE__, __LINE__); }
+    init_pool();
+    s = stream;
+    cudaError_t e = cudaMallocAsync(&p, nbytes ? nbytes : 16, stream);
+    if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMallocAsync", __FILE__, __LINE__); }
     bytes = nbytes;
     return TIGR_OK;
 }
 
 void DevBuf::release() {
-    if (p) cudaFree(p);
+    if (p) cudaFreeAsync(p, s);
     p = nullptr;
     bytes = 0;
 }
 
 tigr_status TmpBuf::alloc(size_t nbytes, cudaStream_t stream) {
+    init_pool();
     s = stream;
     cudaError_t e = cudaMallocAsync(&p, nbytes ? nbytes : 16, stream);
     if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMallocAsync", __FILE__, __LINE__); }

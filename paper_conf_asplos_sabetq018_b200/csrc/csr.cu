@@ -5,8 +5,9 @@
 // L1131-1132).  B200 layout: every node's segment starts on a 16-byte boundary and is
 // padded to a multiple of 4 slots (pads = 0xFFFFFFFF), so the relax kernels can move
 // edges (and, in a separate array, weights) as 128-bit chunks; cptr[v] is the first chunk.
-// The arc order inside a segment is whatever the atomic scatter produced (the paper's
-// results do not depend on it; tests compare segments as multisets).
+// From an arc list the CSR is built by a stable radix sort on the source (sort.cu), so the
+// arcs of a source keep their input order: the canonical CSR, element-identical to a stable
+// counting sort.
 #include "internal.cuh"
 
 namespace tigr {
@@ -14,6 +15,8 @@ namespace tigr {
 tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double b, double c,
                        uint64_t seed, uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src,
                        uint32_t* dst, uint32_t* w, cudaStream_t s);
+tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
+                             int symmetrize, cudaStream_t s, tigr_graph* g);
 
 namespace {
 
@@ -26,72 +29,6 @@ __global__ void k_maxid(const uint32_t* __restrict__ a, const uint32_t* __restri
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
     if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
-}
-
-// out-degree histogram; warp-aggregated so hub sources cost one atomic per warp
-__device__ __forceinline__ void agg_add(uint32_t* cnt, uint32_t key, bool valid) {
-    const uint32_t active = __ballot_sync(0xffffffffu, valid);
-    if (!valid) return;
-    const uint32_t peers = __match_any_sync(active, key);
-    const int lane = threadIdx.x & 31;
-    if (lane == __ffs(peers) - 1) atomicAdd(&cnt[key], (uint32_t)__popc(peers));
-}
-
-__global__ void k_hist(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
-                       int sym, uint32_t* deg) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    const uint64_t start = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const uint64_t rounds = (m + stride - 1) / stride;
-    for (uint64_t r = 0; r < rounds; ++r) {
-        const uint64_t i = start + r * stride;
-        const bool v = i < m;
-        agg_add(deg, v ? src[i] : 0, v);
-        if (sym) agg_add(deg, v ? dst[i] : 0, v);
-    }
-}
-
-// warp-aggregated slot reservation: returns this lane's position within its source segment
-__device__ __forceinline__ uint32_t agg_reserve(uint32_t* cursor, uint32_t key, bool valid) {
-    const uint32_t active = __ballot_sync(0xffffffffu, valid);
-    if (!valid) return 0;
-    const uint32_t peers = __match_any_sync(active, key);
-    const int lane = threadIdx.x & 31;
-    const int leader = __ffs(peers) - 1;
-    uint32_t base = 0;
-    if (lane == leader) base = atomicAdd(&cursor[key], (uint32_t)__popc(peers));
-    base = __shfl_sync(peers, base, leader);
-    return base + __popc(peers & ((1u << lane) - 1));
-}
-
-__global__ void k_scatter(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst,
-                          const uint32_t* __restrict__ w, uint64_t m, int sym,
-                          const uint32_t* __restrict__ cptr, uint32_t* cursor, uint32_t* __restrict__ col,
-                          uint32_t* __restrict__ wt) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    const uint64_t start = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const uint64_t rounds = (m + stride - 1) / stride;
-    for (uint64_t r = 0; r < rounds; ++r) {
-        const uint64_t i = start + r * stride;
-        const bool v = i < m;
-        const uint32_t s = v ? src[i] : 0, d = v ? dst[i] : 0;
-        const uint32_t x = (v && w) ? w[i] : 0;
-        {
-            const uint32_t p = agg_reserve(cursor, s, v);
-            if (v) {
-                const uint64_t slot = (uint64_t)cptr[s] * kChunk + p;
-                col[slot] = d;
-                if (wt) wt[slot] = x;
-            }
-        }
-        if (sym) {
-            const uint32_t p = agg_reserve(cursor, d, v);
-            if (v) {
-                const uint64_t slot = (uint64_t)cptr[d] * kChunk + p;
-                col[slot] = s;
-                if (wt) wt[slot] = x;
-            }
-        }
-    }
 }
 
 __global__ void k_pad(const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cptr, uint32_t n,
@@ -166,17 +103,17 @@ unsigned capped_grid(uint64_t items) {
 
 // degrees known -> row_ptr, cptr, edge buffers
 tigr_status layout_from_degrees(tigr_graph* g, cudaStream_t s) {
-    TIGR_TRY(g->row_ptr.alloc(sizeof(int64_t) * ((size_t)g->n + 1)));
+    TIGR_TRY(g->row_ptr.alloc(sizeof(int64_t) * ((size_t)g->n + 1), s));
     TIGR_TRY(exclusive_scan_u64(g->deg.as<uint32_t>(), g->n, SCAN_U32, 1,
                                 reinterpret_cast<uint64_t*>(g->row_ptr.p), s));
-    TIGR_TRY(g->cptr.alloc(sizeof(uint32_t) * ((size_t)g->n + 1)));
+    TIGR_TRY(g->cptr.alloc(sizeof(uint32_t) * ((size_t)g->n + 1), s));
     uint64_t nch = 0;
     TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), g->n, SCAN_CEIL_DIV, kChunk, g->cptr.as<uint32_t>(),
                                 s, &nch));
     if (nch >= (1ull << 32)) return fail(TIGR_ERANGE, "graph: padded edge chunks exceed 2^32");
     g->nchunks = nch;
-    TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1)));
-    if (g->weighted) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1)));
+    TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));
+    if (g->weighted) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));
     return TIGR_OK;
 }
 
@@ -202,30 +139,15 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
     g->m = arcs;
     g->weighted = w != nullptr;
     g->symmetric = symmetrize != 0;
-    auto bail = [&](tigr_status st) { delete g; return st; };
-    tigr_status st = g->deg.alloc(sizeof(uint32_t) * n);
-    if (st) return bail(st);
-    if (cudaMemsetAsync(g->deg.p, 0, sizeof(uint32_t) * n, s) != cudaSuccess)
-        return bail(cuda_fail(cudaGetLastError(), "memset deg", __FILE__, __LINE__));
-    if (m) {
-        k_hist<<<capped_grid(m), kBlock, 0, s>>>(src, dst, m, symmetrize, g->deg.as<uint32_t>());
+    tigr_status st = csr_build_sorted(n, m, src, dst, w, symmetrize, s, g);
+    if (st == TIGR_OK) {
+        k_pad<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), g->cptr.as<uint32_t>(), n, g->col.as<uint32_t>(),
+                                              g->wt.as<uint32_t>());
         count_launch();
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) st = cuda_fail(e, "graph_from_coo pad", __FILE__, __LINE__);
     }
-    if ((st = layout_from_degrees(g, s))) return bail(st);
-    if (m) {
-        TmpBuf cursor;
-        if ((st = cursor.alloc(sizeof(uint32_t) * n, s))) return bail(st);
-        cudaMemsetAsync(cursor.p, 0, sizeof(uint32_t) * n, s);
-        k_scatter<<<capped_grid(m), kBlock, 0, s>>>(src, dst, w, m, symmetrize, g->cptr.as<uint32_t>(),
-                                                    cursor.as<uint32_t>(), g->col.as<uint32_t>(),
-                                                    g->wt.as<uint32_t>());
-        count_launch();
-    }
-    k_pad<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), g->cptr.as<uint32_t>(), n,
-                                          g->col.as<uint32_t>(), g->wt.as<uint32_t>());
-    count_launch();
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return bail(cuda_fail(e, "graph_from_coo kernels", __FILE__, __LINE__));
+    if (st != TIGR_OK) { delete g; return st; }
     *out = g;
     return TIGR_OK;
 }
@@ -242,7 +164,7 @@ tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, con
     TmpBuf bad;
     if ((st = bad.alloc(sizeof(uint32_t), s))) return bail(st);
     cudaMemsetAsync(bad.p, 0, sizeof(uint32_t), s);
-    if ((st = g->deg.alloc(sizeof(uint32_t) * n))) return bail(st);
+    if ((st = g->deg.alloc(sizeof(uint32_t) * n, s))) return bail(st);
     k_deg_from_rowptr<<<grid_for(n), kBlock, 0, s>>>(rp, n, m, g->deg.as<uint32_t>(), bad.as<uint32_t>());
     count_launch();
     uint32_t hbad = 0;

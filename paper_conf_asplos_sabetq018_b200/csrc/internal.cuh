@@ -49,15 +49,21 @@ inline unsigned grid_for(uint64_t items, int block = kBlock) {
 }
 
 // ---- device buffers ------------------------------------------------------------------------
-// Owning device allocation (cudaMalloc; persistent structures) or stream-ordered temporary.
+// Owning device allocation of a persistent structure.  Stream-ordered (cudaMallocAsync from the
+// device's default pool, whose release threshold libtigr raises so that freed blocks stay cached:
+// rebuilding a graph every bench step costs no cudaMalloc/cudaFree synchronisation).  Freed on
+// the stream it was allocated on; callers synchronise before freeing a handle.
 struct DevBuf {
     void* p = nullptr;
     size_t bytes = 0;
-    tigr_status alloc(size_t nbytes);
+    cudaStream_t s = nullptr;
+    tigr_status alloc(size_t nbytes, cudaStream_t stream);
     void release();
     ~DevBuf() { release(); }
     template <class T> T* as() const { return static_cast<T*>(p); }
 };
+
+void init_pool();  // raise the default pool's release threshold (once per process)
 
 struct TmpBuf {  // cudaMallocAsync / cudaFreeAsync on a stream
     void* p = nullptr;

@@ -23,17 +23,37 @@ namespace tigr {
 // ------------------------------------------------------------------------------------------
 // edge walk: the set of (nbr, w) slots a virtual node owns, in the layout's order
 // ------------------------------------------------------------------------------------------
+// Read-only streaming loads (edge / weight chunks): not allocated in L1, and marked
+// evict-first in L2 so that the 1+ GB edge stream does not push the value / accumulator
+// arrays out of the 126 MB L2.  Not volatile: the compiler may hoist them.
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
+__device__ __forceinline__ uint64_t policy_evict_last() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+
 __device__ __forceinline__ uint4 ldg_chunk(const uint4* p) {
     uint4 r;
-    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+        : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(policy_evict_first()));
     return r;
 }
 
 __device__ __forceinline__ uint32_t ldg_u32(const uint32_t* p) {
     uint32_t r;
-    asm volatile("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(policy_evict_first()));
     return r;
+}
+
+// fire-and-forget float64 add into the accumulator, kept resident in L2 (evict-last)
+__device__ __forceinline__ void red_add_f64(double* p, double v, uint64_t pol) {
+    asm volatile("red.global.add.L2::cache_hint.f64 [%0], %1, %2;" :: "l"(p), "d"(v), "l"(pol) : "memory");
 }
 
 // Calls f(nbr[8], w[8]) on batches of up to 8 slots (pads/absent = kPad).
@@ -192,6 +212,103 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_pr(RelaxArgs a) {
     }
 }
 
+// PageRank push, B virtual nodes per thread, loads of every stage issued for all B vnodes
+// before the first atomic (memory-level parallelism: the per-vnode chain vn_phys -> node
+// record -> edge chunks is three dependent latencies; B independent chains overlap them).
+// Thread t of block b handles vnodes b*B*T + r*T + t (r < B), so each stage stays coalesced.
+template <int LAYOUT, int B, bool HINT>
+__global__ void __launch_bounds__(kRelaxThreads) k_relax_pr_mlp(RelaxArgs a) {
+    const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * kRelaxThreads) + threadIdx.x;
+    const uint64_t pol = HINT ? policy_evict_last() : 0;
+    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
+    uint32_t v[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+        v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
+    }
+    uint4 info[B];
+    double x[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        info[r] = make_uint4(0, 0, 0, 1);
+        x[r] = 0.0;
+        if (v[r] != kPad) { info[r] = __ldg(a.vinfo + v[r]); x[r] = __ldg(a.contrib + v[r]); }
+    }
+    uint4 c0[B], c1[B];
+    uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+        const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
+        uint32_t k;
+        if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
+        else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
+        else {
+            const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
+            k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
+            kend[r] = (per >= q - k) ? q : k + per;
+        }
+        const uint4* cb = c4 + info[r].x;
+        c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
+        c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
+        kn[r] = k + 2 * step[r];
+    }
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+            if (nb[t] == kPad) continue;
+            if (HINT) red_add_f64(a.acc + nb[t], x[r], pol);
+            else atomicAdd(a.acc + nb[t], x[r]);
+        }
+    }
+    // chunks beyond the first two (K > 8, or K = no-split): rare, plain loop
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint4* cb = c4 + info[r].x;
+        for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
+            const uint4 c = ldg_chunk(cb + k);
+            const uint32_t nb[4] = {c.x, c.y, c.z, c.w};
+#pragma unroll
+            for (int t = 0; t < 4; ++t) {
+                if (nb[t] == kPad) continue;
+                if (HINT) red_add_f64(a.acc + nb[t], x[r], pol);
+                else atomicAdd(a.acc + nb[t], x[r]);
+            }
+        }
+    }
+}
+
+// kernel variant (development knob, TIGR_PR_VARIANT): 0 = one vnode per thread (k_relax_pr),
+// 1/2/3/4 = 1/2/4/8 vnodes per thread with L2 hints, 5 = 4 per thread without the RED hint
+int pr_variant() {
+    const char* e = getenv("TIGR_PR_VARIANT");
+    return e ? atoi(e) : 3;
+}
+
+int pr_vnodes_per_thread(int layout, bool vec, bool stats) {
+    const int var = pr_variant();
+    if (!vec || stats || var == 0) return 1;
+    return var == 1 ? 1 : (var == 2 ? 2 : (var == 3 ? 4 : (var == 4 ? 8 : (var == 5 ? 4 : 1))));
+}
+
+RelaxFn relax_pr_mlp_kernel(int layout, bool vec, bool stats) {
+    const int var = pr_variant();
+    if (!vec || stats || var == 0) return nullptr;
+    const bool st = layout == TIGR_LAYOUT_STRIDED;
+#define TIGR_PR_PICK(VAR, B, H) \
+    if (var == VAR) return st ? &k_relax_pr_mlp<TIGR_LAYOUT_STRIDED, B, H> : &k_relax_pr_mlp<TIGR_LAYOUT_CONSECUTIVE, B, H>;
+    TIGR_PR_PICK(1, 1, true)
+    TIGR_PR_PICK(2, 2, true)
+    TIGR_PR_PICK(3, 4, true)
+    TIGR_PR_PICK(4, 8, true)
+    TIGR_PR_PICK(5, 4, false)
+#undef TIGR_PR_PICK
+    return nullptr;
+}
+
 // ------------------------------------------------------------------------------------------
 // dispatch
 // ------------------------------------------------------------------------------------------
@@ -280,6 +397,20 @@ __global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* _
     if (__any_sync(0xffffffffu, moved) && (threadIdx.x & 31) == 0) ctl->changed = 1;
 }
 
+// block-reduce a double and add it to *dst with one atomic per block (kBlock threads)
+__device__ __forceinline__ void block_add(double v, double* dst) {
+    __shared__ double part[kBlock / 32];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        double t = 0.0;
+        for (int w = 0; w < kBlock / 32; ++w) t += part[w];
+        if (t != 0.0) atomicAdd(dst, t);
+    }
+}
+
 __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
                           double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
@@ -292,9 +423,7 @@ __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* 
         acc[v] = 0.0;
         if (!d) dang = x0;
     }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) dang += __shfl_xor_sync(0xffffffffu, dang, o);
-    if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(&ctl->dsum[0], dang);
+    block_add(dang, &ctl->dsum[0]);
 }
 
 // x = (1-d)/n + d*(acc + dsum/n);  contrib = x/deg;  acc = 0;  next dangling mass -> dsum_next
@@ -313,11 +442,7 @@ __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double 
         acc[v] = 0.0;
         if (!d) dang = r;
     }
-    if (dangling) {
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) dang += __shfl_xor_sync(0xffffffffu, dang, o);
-        if ((threadIdx.x & 31) == 0 && dang != 0.0) atomicAdd(dsum_next, dang);
-    }
+    if (dangling) block_add(dang, dsum_next);
 }
 
 // per-vnode edge lists, walked with the relax kernels' own arithmetic (layout parity tests)

@@ -30,24 +30,24 @@ Workspace::~Workspace() {
 
 namespace {
 
-tigr_status ensure_ws(tigr_vgraph* vg, bool pr) {
+tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
     Workspace& ws = vg->ws;
     const size_t n = vg->g->n ? vg->g->n : 1;
     if (!ws.ctl.p) {
-        TIGR_TRY(ws.ctl.alloc(sizeof(Ctl)));
+        TIGR_TRY(ws.ctl.alloc(sizeof(Ctl), s));
         TIGR_CK(cudaMallocHost(&ws.ctl_host, sizeof(Ctl)));
         for (auto& e : ws.ev) TIGR_CK(cudaEventCreate(&e));
     }
     if (pr) {
         if (!ws.x.p) {
-            TIGR_TRY(ws.x.alloc(sizeof(double) * n));
-            TIGR_TRY(ws.contrib.alloc(sizeof(double) * n));
-            TIGR_TRY(ws.acc.alloc(sizeof(double) * n));
+            TIGR_TRY(ws.x.alloc(sizeof(double) * n, s));
+            TIGR_TRY(ws.contrib.alloc(sizeof(double) * n, s));
+            TIGR_TRY(ws.acc.alloc(sizeof(double) * n, s));
         }
     } else if (!ws.val.p) {
-        TIGR_TRY(ws.val.alloc(sizeof(uint32_t) * n));
-        TIGR_TRY(ws.prev.alloc(sizeof(uint32_t) * n));
-        TIGR_TRY(ws.stamp.alloc(sizeof(uint32_t) * 2 * n));
+        TIGR_TRY(ws.val.alloc(sizeof(uint32_t) * n, s));
+        TIGR_TRY(ws.prev.alloc(sizeof(uint32_t) * n, s));
+        TIGR_TRY(ws.stamp.alloc(sizeof(uint32_t) * 2 * n, s));
     }
     return TIGR_OK;
 }
@@ -221,8 +221,11 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     Workspace& ws = vg->ws;
     const uint32_t n = vg->g->n;
     RelaxArgs a = make_args(vg);
-    RelaxFn relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
-    const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + kRelaxThreads - 1) / kRelaxThreads);
+    RelaxFn relax = relax_pr_mlp_kernel(vg->layout, vg->vec, o.collect_stats != 0);
+    uint64_t per_block = kRelaxThreads;
+    if (relax) per_block *= pr_vnodes_per_thread(vg->layout, vg->vec, o.collect_stats != 0);
+    else relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
+    const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
     const bool comm = o.comm != nullptr && o.comm->nranks > 1;
     const double base = (1.0 - o.pr_damping) / (double)n;
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
@@ -304,7 +307,7 @@ tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const t
     cudaStream_t s = (cudaStream_t)o.stream;
     if (st) *st = tigr_stats{};
     if (g->n == 0) return TIGR_OK;
-    TIGR_TRY(ensure_ws(vg, algo == TIGR_PR));
+    TIGR_TRY(ensure_ws(vg, algo == TIGR_PR, s));
     tigr_status rs = (algo == TIGR_PR) ? run_pr(vg, o, s, st) : run_frontier(vg, algo, source, o, s, st);
     if (rs != TIGR_OK && rs != TIGR_ENOTCONV) return rs;
     const void* res = (algo == TIGR_PR) ? vg->ws.x.p : vg->ws.val.p;

@@ -62,7 +62,7 @@ tigr_status virtualize_device(const tigr_graph* g, uint32_t K, tigr_layout layou
     cudaEventCreate(&e1);
     cudaEventRecord(e0, s);
     tigr_status st;
-    if ((st = vg->vnode_ptr.alloc(sizeof(uint32_t) * ((size_t)g->n + 1)))) return bail(st);
+    if ((st = vg->vnode_ptr.alloc(sizeof(uint32_t) * ((size_t)g->n + 1), s))) return bail(st);
     uint64_t nv = 0;
     if ((st = exclusive_scan_u32(g->deg.as<uint32_t>(), g->n, SCAN_CEIL_DIV, K, vg->vnode_ptr.as<uint32_t>(),
                                  s, &nv)))
@@ -71,8 +71,8 @@ tigr_status virtualize_device(const tigr_graph* g, uint32_t K, tigr_layout layou
     vg->nv = nv;
     vg->lo = 0;
     vg->hi = (uint32_t)nv;
-    if ((st = vg->vn_phys.alloc(sizeof(uint32_t) * (nv ? nv : 1)))) return bail(st);
-    if ((st = vg->vinfo.alloc(sizeof(uint4) * (g->n ? g->n : 1)))) return bail(st);
+    if ((st = vg->vn_phys.alloc(sizeof(uint32_t) * (nv ? nv : 1), s))) return bail(st);
+    if ((st = vg->vinfo.alloc(sizeof(uint4) * (g->n ? g->n : 1), s))) return bail(st);
     k_emit<<<grid_for(g->n), kBlock, 0, s>>>(vg->vnode_ptr.as<uint32_t>(), g->n, vg->vn_phys.as<uint32_t>());
     count_launch();
     k_vinfo<<<grid_for(g->n), kBlock, 0, s>>>(g->cptr.as<uint32_t>(), g->deg.as<uint32_t>(),

@@ -1,0 +1,82 @@
+"""Kernel micro-benchmark on the GPU box: build the cfg4 graph once per process and time the
+phases / relax-kernel variants with CUDA events.  Development tool (not the driver bench)."""
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import graphgen  # noqa: E402
+import paper_conf_asplos_sabetq018_b200 as tigr  # noqa: E402
+
+
+def main():
+    cfg = os.environ.get("CFG", "cfg4")
+    K = int(os.environ.get("K", "8"))
+    layout = os.environ.get("LAYOUT", "strided")
+    reps = int(os.environ.get("REPS", "3"))
+    rec = graphgen.recipe(cfg)
+    s = torch.cuda.current_stream()
+    src = torch.empty(rec.m, dtype=torch.int32, device="cuda")
+    dst = torch.empty_like(src)
+    tigr.tigr_rmat_coo(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, 1, 64, src, dst, None, stream=s)
+    torch.cuda.synchronize()
+    res = {"variant": os.environ.get("TIGR_PR_VARIANT", "default"), "cfg": cfg, "K": K, "layout": layout}
+    csr, vir = [], []
+    for _ in range(reps):
+        e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        e[0].record(s)
+        g = tigr.tigr_graph_from_coo(rec.n, src, dst, None, stream=s)
+        e[1].record(s)
+        vg = tigr.tigr_virtualize(g, K, layout, stream=s)
+        e[2].record(s)
+        torch.cuda.synchronize()
+        csr.append(e[0].elapsed_time(e[1]))
+        vir.append(e[1].elapsed_time(e[2]))
+    res["csr_ms"] = min(csr)
+    res["virt_ms"] = min(vir)
+    out = torch.empty(rec.n, dtype=torch.float64, device="cuda")
+    best = None
+    for _ in range(reps):
+        _, st = tigr.tigr_run(vg, "pr", out=out, stream=s, time_kernels=1, return_stats=True)
+        if best is None or st["ms_relax"] < best["ms_relax"]:
+            best = st
+    res["pr_ms_total"] = best["ms_total"]
+    res["relax_ms_per_launch"] = best["ms_relax"] / max(best["relax_launches"], 1)
+    nv = vg.info()["nv"]
+    n_out = int(torch.count_nonzero(torch.bincount(src, minlength=rec.n)).item())
+    bytes_alg = rec.m * 20 + nv * 4 + n_out * 16
+    res["relax_GBps_alg"] = bytes_alg / (res["relax_ms_per_launch"] * 1e-3) / 1e9
+    res["relax_frac"] = res["relax_GBps_alg"] / 6541.8
+    res["gteps_relax"] = rec.m / (res["relax_ms_per_launch"] * 1e-3) / 1e9
+    if os.environ.get("FRONTIER", "1") == "1" and cfg == "cfg4":
+        gw = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=True, stream=s)
+        vgw = tigr.tigr_virtualize(gw, K, layout, stream=s)
+        o32 = torch.empty(rec.n, dtype=torch.int32, device="cuda")
+        for algo in ("bfs", "sssp", "sswp"):
+            ts = []
+            for _ in range(reps):
+                _, st = tigr.tigr_run(vgw, algo, 0, out=o32, stream=s, return_stats=True)
+                ts.append(st["ms_total"])
+            res[algo + "_ms"] = min(ts)
+            res[algo + "_iters"] = st["iterations"]
+        del vgw, gw
+        gs = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False,
+                                  symmetrize=True, stream=s)
+        vgs = tigr.tigr_virtualize(gs, K, layout, stream=s)
+        ts = []
+        for _ in range(reps):
+            _, st = tigr.tigr_run(vgs, "cc", 0, out=o32, stream=s, return_stats=True)
+            ts.append(st["ms_total"])
+        res["cc_ms"] = min(ts)
+        res["cc_iters"] = st["iterations"]
+    print(json.dumps(res), flush=True)
+
+
+if __name__ == "__main__":
+    main()
