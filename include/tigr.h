@@ -200,6 +200,9 @@ void tigr_comm_free(tigr_comm* comm);
 /* ----------------------------------------------------------------- misc ---- */
 
 const char* tigr_last_error(void);
+/* libtigr caches freed device blocks for reuse (graph rebuilds allocate GBs); return them all
+ * to the driver.  Synchronises the device. */
+void tigr_release_cached_memory(void);
 /* Number of CUDA kernels this library launched in this process (graph-launched ones
  * included, counted per executed node). */
 uint64_t tigr_launch_count(void);

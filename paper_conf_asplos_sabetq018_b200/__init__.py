@@ -83,6 +83,7 @@ _SIGS = {
     "tigr_comm_free": (None, [_P]),
     "tigr_last_error": (ctypes.c_char_p, []),
     "tigr_launch_count": (_U64, []),
+    "tigr_release_cached_memory": (None, []),
     "tigr_version": (ctypes.c_char_p, []),
 }
 for _name, (_res, _args) in _SIGS.items():
@@ -337,6 +338,10 @@ def tigr_last_error() -> str:
 
 def tigr_launch_count() -> int:
     return int(_lib.tigr_launch_count())
+
+
+def tigr_release_cached_memory() -> None:
+    _lib.tigr_release_cached_memory()
 
 
 def tigr_version() -> str:

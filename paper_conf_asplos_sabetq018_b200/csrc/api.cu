@@ -1,7 +1,10 @@
 // api.cu -- the extern "C" boundary of libtigr.so (include/tigr.h).  Argument checking,
 // host<->device staging, error state; every compute step runs in the kernels of the other
 // translation units.
+#include <chrono>
 #include <cstdio>
+#include <cstdlib>
+#include <map>
 #include <mutex>
 #include <cstring>
 #include <string>
@@ -16,6 +19,25 @@ static thread_local std::string t_err;
 
 void set_error(const std::string& msg) { t_err = msg; }
 
+void trace(cudaStream_t s, const char* what) {
+    static const bool on = getenv("TIGR_TRACE") != nullptr;
+    if (!on) return;
+    static thread_local std::chrono::steady_clock::time_point last = std::chrono::steady_clock::now();
+    cudaStreamSynchronize(s);
+    const auto now = std::chrono::steady_clock::now();
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaMemPool_t pool;
+    uint64_t reserved = 0, used = 0;
+    if (cudaDeviceGetMemPool(&pool, dev) == cudaSuccess) {
+        cudaMemPoolGetAttribute(pool, cudaMemPoolAttrReservedMemCurrent, &reserved);
+        cudaMemPoolGetAttribute(pool, cudaMemPoolAttrUsedMemCurrent, &used);
+    }
+    fprintf(stderr, "[tigr trace] %-28s %9.3f ms  (pool reserved %.2f GB, used %.2f GB)\n", what,
+            std::chrono::duration<double, std::milli>(now - last).count(), reserved / 1e9, used / 1e9);
+    last = now;
+}
+
 tigr_status fail(tigr_status st, const std::string& msg) {
     t_err = msg;
     return st;
@@ -28,44 +50,105 @@ tigr_status cuda_fail(cudaError_t e, const char* what, const char* file, int lin
     return (e == cudaErrorMemoryAllocation) ? TIGR_ENOMEM : TIGR_ECUDA;
 }
 
-void init_pool() {
-    static std::once_flag once;
-    std::call_once(once, [] {
-        int dev = 0;
-        if (cudaGetDevice(&dev) != cudaSuccess) return;
-        cudaMemPool_t pool;
-        if (cudaDeviceGetDefaultMemPool(&pool, dev) != cudaSuccess) return;
-        uint64_t thr = UINT64_MAX;
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    });
+// ---- caching device allocator ------------------------------------------------------------
+// cudaMallocAsync of multi-GB blocks measured 15-100 ms on B200 even with a raised pool
+// release threshold, and a graph build allocates ~6 GB of sort buffers; so libtigr keeps its
+// own cache of cudaMalloc'ed blocks (2 MiB granularity, best fit within +25%).  A freed block
+// records an event on the stream that last used it; reuse from another stream waits on it.
+namespace {
+struct CachedBlock {
+    void* p;
+    size_t size;
+    cudaStream_t s;
+    cudaEvent_t ev;
+};
+std::mutex g_cache_mu;
+std::multimap<size_t, CachedBlock> g_free;       // size -> block
+std::map<void*, size_t> g_live;                 // live block -> size
+constexpr size_t kGran = 2u << 20;
+
+void release_cached_locked() {
+    for (auto& kv : g_free) {
+        cudaFree(kv.second.p);
+        if (kv.second.ev) cudaEventDestroy(kv.second.ev);
+    }
+    g_free.clear();
+}
+}  // namespace
+
+void init_pool() {}
+
+void* cache_alloc(size_t nbytes, cudaStream_t s, cudaError_t* err) {
+    const size_t size = ((nbytes ? nbytes : 1) + kGran - 1) / kGran * kGran;
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_free.lower_bound(size);
+    if (it != g_free.end() && it->first <= size + size / 4 + kGran) {
+        CachedBlock b = it->second;
+        g_free.erase(it);
+        if (b.s != s && b.ev) cudaStreamWaitEvent(s, b.ev, 0);
+        if (b.ev) cudaEventDestroy(b.ev);
+        g_live[b.p] = b.size;
+        *err = cudaSuccess;
+        return b.p;
+    }
+    void* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, size);
+    if (e != cudaSuccess) {  // give the cache back to the driver and retry once
+        cudaGetLastError();
+        cudaDeviceSynchronize();
+        release_cached_locked();
+        e = cudaMalloc(&p, size);
+    }
+    *err = e;
+    if (e != cudaSuccess) return nullptr;
+    g_live[p] = size;
+    return p;
+}
+
+void cache_free(void* p, cudaStream_t s) {
+    if (!p) return;
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_live.find(p);
+    if (it == g_live.end()) return;
+    CachedBlock b{p, it->second, s, nullptr};
+    g_live.erase(it);
+    if (cudaEventCreateWithFlags(&b.ev, cudaEventDisableTiming) == cudaSuccess) cudaEventRecord(b.ev, s);
+    else b.ev = nullptr;
+    g_free.emplace(b.size, b);
+}
+
+void cache_release_all() {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    cudaDeviceSynchronize();
+    release_cached_locked();
 }
 
 tigr_status DevBuf::alloc(size_t nbytes, cudaStream_t stream) {
     release();
-    init_pool();
     s = stream;
-    cudaError_t e = cudaMallocAsync(&p, nbytes ? nbytes : 16, stream);
-    if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMallocAsync", __FILE__, __LINE__); }
+    cudaError_t e = cudaSuccess;
+    p = cache_alloc(nbytes, stream, &e);
+    if (!p) return cuda_fail(e, "cudaMalloc", __FILE__, __LINE__);
     bytes = nbytes;
     return TIGR_OK;
 }
 
 void DevBuf::release() {
-    if (p) cudaFreeAsync(p, s);
+    if (p) cache_free(p, s);
     p = nullptr;
     bytes = 0;
 }
 
 tigr_status TmpBuf::alloc(size_t nbytes, cudaStream_t stream) {
-    init_pool();
     s = stream;
-    cudaError_t e = cudaMallocAsync(&p, nbytes ? nbytes : 16, stream);
-    if (e != cudaSuccess) { p = nullptr; return cuda_fail(e, "cudaMallocAsync", __FILE__, __LINE__); }
+    cudaError_t e = cudaSuccess;
+    p = cache_alloc(nbytes, stream, &e);
+    if (!p) return cuda_fail(e, "cudaMalloc", __FILE__, __LINE__);
     return TIGR_OK;
 }
 
 TmpBuf::~TmpBuf() {
-    if (p) cudaFreeAsync(p, s);
+    if (p) cache_free(p, s);
 }
 
 // other translation units
@@ -143,8 +226,10 @@ tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, con
     TIGR_TRY(stage(src, m, is_device_ptr, s, ts, &ds));
     TIGR_TRY(stage(dst, m, is_device_ptr, s, td, &dd));
     TIGR_TRY(stage(w, m, is_device_ptr, s, tw, &dw));
+    trace(s, "coo: stage");
     TIGR_TRY(graph_from_coo_device(n, m, ds, dd, dw, symmetrize, s, out));
     TIGR_CK(cudaStreamSynchronize(s));
+    trace(s, "coo: done");
     return TIGR_OK;
 }
 
@@ -303,6 +388,8 @@ void tigr_comm_free(tigr_comm* c) { comm_free(c); }
 const char* tigr_last_error(void) { return t_err.c_str(); }
 
 uint64_t tigr_launch_count(void) { return g_launches.load(); }
+
+void tigr_release_cached_memory(void) { cache_release_all(); }
 
 const char* tigr_version(void) { return "tigr-b200 0.1 (sm_100a)"; }
 

@@ -133,6 +133,7 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
         TIGR_CK(cudaMemcpyAsync(&hmax, mx.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         TIGR_CK(cudaStreamSynchronize(s));
         if (hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
+        trace(s, "coo: validate ids");
     }
     tigr_graph* g = new tigr_graph();
     g->n = n;

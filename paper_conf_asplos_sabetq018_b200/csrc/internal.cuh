@@ -43,6 +43,10 @@ inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_o
         if (_s != TIGR_OK) return _s;                                         \
     } while (0)
 
+// Development tracing: with TIGR_TRACE=1 in the environment, trace(s, "phase") synchronises
+// the stream and prints the host wall time since the previous trace point (stderr).
+void trace(cudaStream_t s, const char* what);
+
 inline unsigned grid_for(uint64_t items, int block = kBlock) {
     uint64_t g = (items + block - 1) / block;
     return (unsigned)(g ? g : 1);

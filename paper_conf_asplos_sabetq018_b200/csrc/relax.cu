@@ -18,6 +18,8 @@
 #include "vgraph.cuh"
 #include "relax.cuh"
 
+#include <algorithm>
+
 namespace tigr {
 
 // ------------------------------------------------------------------------------------------
@@ -281,11 +283,216 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_pr_mlp(RelaxArgs a) {
     }
 }
 
+// ------------------------------------------------------------------------------------------
+// PageRank push with the hottest destinations privatised in shared memory.
+//
+// Power-law in-degrees make the RED traffic collide on a few L2 sectors (cfg4: the top vertex
+// receives 0.14% of all arcs, and the 4 vertices of its 32-byte sector ~0.24%); B200 serialises
+// same-sector reductions, which caps skewed f64 REDs at ~70 G/s versus ~190 G/s spread
+// (tools/micro/red_bench.cu).  Each persistent block keeps an open-addressing table of the
+// hottest destinations (sampled in-degree, chosen on the device) in shared memory, adds their
+// contributions there, and flushes one RED per hot vertex at the end.  All other arcs RED
+// straight to L2.  Same sums, different association order (PR parity is 1e-6).
+// ------------------------------------------------------------------------------------------
+int pr_variant();
+
+constexpr int kHotMaxSlots = 8192;        // largest table (power of two)
+constexpr int kHotMaxIds = kHotMaxSlots / 4;  // load factor <= 1/4: ~1.4 probes for a miss
+constexpr int kHotSampleStride = 16;      // sample every 16th 16-byte chunk of the arc array
+
+template <int LOGS>
+__device__ __forceinline__ uint32_t hot_hash(uint32_t v) { return (v * 0x9E3779B1u) >> (32 - LOGS); }
+
+// sampled in-degree: every kHotSampleStride-th chunk of the arc array
+__global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uint32_t* __restrict__ cnt) {
+    for (uint64_t k = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) * kHotSampleStride; k < nchunks;
+         k += (uint64_t)gridDim.x * blockDim.x * kHotSampleStride) {
+        const uint4 c = __ldg(c4 + k);
+        if (c.x != kPad) atomicAdd(cnt + c.x, 1u);
+        if (c.y != kPad) atomicAdd(cnt + c.y, 1u);
+        if (c.z != kPad) atomicAdd(cnt + c.z, 1u);
+        if (c.w != kPad) atomicAdd(cnt + c.w, 1u);
+    }
+}
+
+// histogram of floor(log2(count)) (bucket 0 = count 0)
+__global__ void k_hot_loghist(const uint32_t* __restrict__ cnt, uint32_t n, uint32_t* __restrict__ hist) {
+    __shared__ uint32_t h[33];
+    if (threadIdx.x < 33) h[threadIdx.x] = 0;
+    __syncthreads();
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        const uint32_t c = cnt[v];
+        if (c) atomicAdd(&h[32 - __clz(c)], 1u);
+    }
+    __syncthreads();
+    if (threadIdx.x < 33 && h[threadIdx.x]) atomicAdd(&hist[threadIdx.x], h[threadIdx.x]);
+}
+
+// hot = sampled count >= 2^(b-1) for the smallest bucket b keeping #hot <= max_ids (and >= 2)
+__global__ void k_hot_compact(const uint32_t* __restrict__ cnt, uint32_t n, const uint32_t* __restrict__ hist,
+                              uint32_t max_ids, uint32_t* __restrict__ hot_ids, uint32_t* __restrict__ n_hot) {
+    __shared__ uint32_t thr;
+    if (threadIdx.x == 0) {
+        uint32_t acc = 0, b = 33;
+        while (b > 2 && acc + hist[b - 1] <= max_ids) { acc += hist[b - 1]; --b; }
+        thr = (b >= 33) ? 0xFFFFFFFFu : (1u << (b - 1));  // bucket b holds counts in [2^(b-1), 2^b)
+    }
+    __syncthreads();
+    const uint32_t t = thr;
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        if (cnt[v] >= t && cnt[v] >= 2) {
+            const uint32_t h = atomicAdd(n_hot, 1u);
+            if (h < max_ids) hot_ids[h] = v;
+        }
+    }
+}
+
+// LOGS: log2 of the table size (2^LOGS slots, at most 2^LOGS / 4 hot ids); MINB: blocks/SM
+template <int LAYOUT, int B, int LOGS, int MINB>
+__global__ void __launch_bounds__(kRelaxThreads, MINB) k_relax_pr_hot(RelaxArgs a, const uint32_t* __restrict__ hot_ids,
+                                                                     const uint32_t* __restrict__ n_hot_p, uint32_t tiles) {
+    constexpr int kSlots = 1 << LOGS;
+    extern __shared__ __align__(16) unsigned char hsm[];
+    double* s_acc = reinterpret_cast<double*>(hsm);
+    uint32_t* s_key = reinterpret_cast<uint32_t*>(hsm + sizeof(double) * kSlots);
+    const int t = threadIdx.x;
+    for (int i = t; i < kSlots; i += kRelaxThreads) { s_key[i] = kPad; s_acc[i] = 0.0; }
+    __syncthreads();
+    const uint32_t n_hot = min(*n_hot_p, (uint32_t)(kSlots / 4));
+    for (uint32_t h = t; h < n_hot; h += kRelaxThreads) {
+        const uint32_t id = hot_ids[h];
+        uint32_t s = hot_hash<LOGS>(id);
+        while (atomicCAS(&s_key[s], kPad, id) != kPad) s = (s + 1) & (kSlots - 1);
+    }
+    __syncthreads();
+    const uint64_t pol = policy_evict_last();
+    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
+    auto push = [&](uint32_t nb, double x) {
+        uint32_t s = hot_hash<LOGS>(nb);
+        for (;;) {
+            const uint32_t k = s_key[s];
+            if (k == nb) { atomicAdd(&s_acc[s], x); return; }
+            if (k == kPad) { red_add_f64(a.acc + nb, x, pol); return; }
+            s = (s + 1) & (kSlots - 1);
+        }
+    };
+    for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        const uint64_t base = (uint64_t)a.lo + (uint64_t)tile * (B * kRelaxThreads) + t;
+        uint32_t v[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+            v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
+        }
+        uint4 info[B];
+        double x[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            info[r] = make_uint4(0, 0, 0, 1);
+            x[r] = 0.0;
+            if (v[r] != kPad) { info[r] = __ldg(a.vinfo + v[r]); x[r] = __ldg(a.contrib + v[r]); }
+        }
+        uint4 c0[B], c1[B];
+        uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+            const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
+            uint32_t k;
+            if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
+            else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
+            else {
+                const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
+                k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
+                kend[r] = (per >= q - k) ? q : k + per;
+            }
+            const uint4* cb = c4 + info[r].x;
+            c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
+            c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
+            kn[r] = k + 2 * step[r];
+        }
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                if (nb[q] != kPad) push(nb[q], x[r]);
+        }
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint4* cb = c4 + info[r].x;
+            for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
+                const uint4 c = ldg_chunk(cb + k);
+                const uint32_t nb[4] = {c.x, c.y, c.z, c.w};
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (nb[q] != kPad) push(nb[q], x[r]);
+            }
+        }
+    }
+    __syncthreads();
+    for (int i = t; i < kSlots; i += kRelaxThreads) {
+        const uint32_t k = s_key[i];
+        if (k != kPad && s_acc[i] != 0.0) red_add_f64(a.acc + k, s_acc[i], pol);
+    }
+}
+
+uint32_t pr_hot_max() { return kHotMaxIds; }
+
+// sampled in-degrees -> device list of at most max_ids hottest destinations (no host sync)
+tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uint32_t max_ids, uint32_t* cnt_tmp,
+                          uint32_t* hist_tmp, uint32_t* hot_ids, uint32_t* n_hot, cudaStream_t s) {
+    TIGR_CK(cudaMemsetAsync(cnt_tmp, 0, sizeof(uint32_t) * n, s));
+    TIGR_CK(cudaMemsetAsync(hist_tmp, 0, sizeof(uint32_t) * 33, s));
+    TIGR_CK(cudaMemsetAsync(n_hot, 0, sizeof(uint32_t), s));
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t samples = (nchunks + kHotSampleStride - 1) / kHotSampleStride;
+    if (samples) {
+        k_hot_sample<<<grid_for(samples < (uint64_t)sms * 2048 ? samples : (uint64_t)sms * 2048), kBlock, 0, s>>>(
+            reinterpret_cast<const uint4*>(col), nchunks, cnt_tmp);
+        TIGR_CKL("hot sample");
+    }
+    const unsigned g = (unsigned)std::min<uint64_t>(grid_for(n), (uint64_t)sms * 8);
+    k_hot_loghist<<<g, kBlock, 0, s>>>(cnt_tmp, n, hist_tmp);
+    TIGR_CKL("hot loghist");
+    k_hot_compact<<<g, kBlock, 0, s>>>(cnt_tmp, n, hist_tmp, max_ids, hot_ids, n_hot);
+    TIGR_CKL("hot compact");
+    return TIGR_OK;
+}
+
+template <int B, int LOGS, int MINB>
+static PrHotConfig make_hot(int layout) {
+    PrHotConfig c;
+    c.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_hot<TIGR_LAYOUT_STRIDED, B, LOGS, MINB>
+                                         : &k_relax_pr_hot<TIGR_LAYOUT_CONSECUTIVE, B, LOGS, MINB>;
+    c.vnodes_per_thread = B;
+    c.smem = (sizeof(double) + sizeof(uint32_t)) << LOGS;
+    c.max_ids = (1u << LOGS) / 4;
+    return c;
+}
+
+// variants (TIGR_PR_VARIANT): 6 = 8192 slots, 4 vnodes/thread; 7 = 8192, 2/thread;
+// 8 = 4096 slots, 4/thread; 9 = 2048 slots, 4/thread; 10 = 4096 slots, 2/thread
+PrHotConfig relax_pr_hot_config(int layout, bool vec) {
+    PrHotConfig none;
+    if (!vec) return none;
+    switch (pr_variant()) {
+        case 6: return make_hot<4, 13, 2>(layout);
+        case 7: return make_hot<2, 13, 2>(layout);
+        case 8: return make_hot<4, 12, 3>(layout);
+        case 9: return make_hot<4, 11, 3>(layout);
+        case 10: return make_hot<2, 12, 4>(layout);
+        default: return none;
+    }
+}
+
 // kernel variant (development knob, TIGR_PR_VARIANT): 0 = one vnode per thread (k_relax_pr),
 // 1/2/3/4 = 1/2/4/8 vnodes per thread with L2 hints, 5 = 4 per thread without the RED hint
 int pr_variant() {
     const char* e = getenv("TIGR_PR_VARIANT");
-    return e ? atoi(e) : 3;
+    return e ? atoi(e) : 6;
 }
 
 int pr_vnodes_per_thread(int layout, bool vec, bool stats) {

@@ -29,6 +29,18 @@ RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool s
 // PageRank push with several virtual nodes per thread (nullptr: use relax_kernel's); B per thread
 RelaxFn relax_pr_mlp_kernel(int layout, bool vec, bool stats);
 int pr_vnodes_per_thread(int layout, bool vec, bool stats);
+// PageRank push with shared-memory privatisation of the hottest destinations (persistent grid)
+typedef void (*RelaxHotFn)(RelaxArgs, const uint32_t*, const uint32_t*, uint32_t);
+struct PrHotConfig {
+    RelaxHotFn fn = nullptr;
+    int vnodes_per_thread = 1;
+    size_t smem = 0;          // dynamic shared memory per block
+    uint32_t max_ids = 0;     // hot destinations the table holds
+};
+PrHotConfig relax_pr_hot_config(int layout, bool vec);
+uint32_t pr_hot_max();        // capacity of the workspace's hot-id list (>= any config's max_ids)
+tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uint32_t max_ids, uint32_t* cnt_tmp,
+                          uint32_t* hist_tmp, uint32_t* hot_ids, uint32_t* n_hot, cudaStream_t s);
 AssignFn assign_kernel(int layout, bool vec);
 
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,

@@ -43,6 +43,7 @@ tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
             TIGR_TRY(ws.x.alloc(sizeof(double) * n, s));
             TIGR_TRY(ws.contrib.alloc(sizeof(double) * n, s));
             TIGR_TRY(ws.acc.alloc(sizeof(double) * n, s));
+            TIGR_TRY(ws.hot.alloc(sizeof(uint32_t) * (n + 34 + pr_hot_max()), s));
         }
     } else if (!ws.val.p) {
         TIGR_TRY(ws.val.alloc(sizeof(uint32_t) * n, s));
@@ -221,6 +222,26 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     Workspace& ws = vg->ws;
     const uint32_t n = vg->g->n;
     RelaxArgs a = make_args(vg);
+    // preferred: persistent kernel with the hottest destinations privatised in shared memory
+    const PrHotConfig hc = o.collect_stats ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
+    const RelaxHotFn hot = hc.fn;
+    uint32_t* hot_cnt = ws.hot.as<uint32_t>();
+    uint32_t* hot_hist = hot_cnt + n;
+    uint32_t* hot_n = hot_hist + 33;
+    uint32_t* hot_ids = hot_n + 1;
+    unsigned hot_grid = 0, hot_tiles = 0;
+    if (hot) {
+        TIGR_CK(cudaFuncSetAttribute(hot, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hc.smem));
+        int per_sm = 0, dev = 0, sms = 148;
+        TIGR_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hot, kRelaxThreads, hc.smem));
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        const uint64_t per_tile = (uint64_t)kRelaxThreads * hc.vnodes_per_thread;
+        hot_tiles = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_tile - 1) / per_tile);
+        hot_grid = (unsigned)std::min<uint64_t>(hot_tiles, (uint64_t)sms * (per_sm > 0 ? per_sm : 1));
+        TIGR_TRY(pr_hot_select(vg->g->col.as<uint32_t>(), vg->g->nchunks, n, hc.max_ids, hot_cnt, hot_hist, hot_ids,
+                               hot_n, s));
+    }
     RelaxFn relax = relax_pr_mlp_kernel(vg->layout, vg->vec, o.collect_stats != 0);
     uint64_t per_block = kRelaxThreads;
     if (relax) per_block *= pr_vnodes_per_thread(vg->layout, vg->vec, o.collect_stats != 0);
@@ -245,7 +266,11 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     }
     for (uint32_t t = 0; t < o.pr_iters; ++t) {
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t], s));
-        if (grid) {
+        if (hot && hot_tiles) {
+            hot<<<hot_grid, kRelaxThreads, hc.smem, s>>>(a, hot_ids, hot_n, hot_tiles);
+            TIGR_CKL("pr relax (hot)");
+            ++launches;
+        } else if (grid) {
             relax<<<grid, kRelaxThreads, 0, s>>>(a);
             TIGR_CKL("pr relax");
             ++launches;

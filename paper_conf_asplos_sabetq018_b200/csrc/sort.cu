@@ -89,7 +89,7 @@ __global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ k
     extern __shared__ __align__(16) unsigned char smem[];
     VT* s_val = reinterpret_cast<VT*>(smem);
     uint32_t* s_key = reinterpret_cast<uint32_t*>(smem + sizeof(VT) * kTileItems);
-    __shared__ uint16_t s_wcnt[kSW][kMaxRadix + 1];
+    __shared__ uint32_t s_wcnt[kSW][kMaxRadix + 1];
     __shared__ uint32_t s_dstart[kMaxRadix + 1];
     __shared__ uint64_t s_gofs[kMaxRadix];
     __shared__ uint32_t s_tile;
@@ -121,16 +121,23 @@ __global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ k
             dig[r] = (uint32_t)radix;  // dummy bin
         }
     }
-    // stable ranking within the warp's 512 items (item order = round-major, then lane)
+    // stable ranking within the warp's 512 items (item order = round-major, then lane): the
+    // lowest lane of each digit group reserves popc(peers) slots with a shared atomic; the
+    // warp issues the rounds' atomics in order, so reservations follow item order; the
+    // results are broadcast after all rounds are issued (no per-round round trip).
     const uint32_t lt = (1u << lane) - 1;
+    uint32_t peers[kSI];
 #pragma unroll
     for (int r = 0; r < kSI; ++r) {
-        const uint32_t peers = __match_any_sync(0xffffffffu, dig[r]);
-        const uint32_t before = s_wcnt[wp][dig[r]];
-        rank[r] = (uint16_t)(before + __popc(peers & lt));
-        __syncwarp();
-        if ((peers & lt) == 0) s_wcnt[wp][dig[r]] = (uint16_t)(before + __popc(peers));
-        __syncwarp();
+        peers[r] = __match_any_sync(0xffffffffu, dig[r]);
+        uint32_t got = 0;
+        if ((peers[r] & lt) == 0) got = atomicAdd(&s_wcnt[wp][dig[r]], (uint32_t)__popc(peers[r]));
+        rank[r] = (uint16_t)got;
+    }
+#pragma unroll
+    for (int r = 0; r < kSI; ++r) {
+        const uint32_t base = __shfl_sync(0xffffffffu, (uint32_t)rank[r], __ffs(peers[r]) - 1);
+        rank[r] = (uint16_t)(base + __popc(peers[r] & lt));
     }
     __syncthreads();
     // per digit: exclusive prefix over warps, tile count, publish the aggregate
@@ -140,7 +147,7 @@ __global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ k
 #pragma unroll
         for (int wi = 0; wi < kSW; ++wi) {
             const uint32_t c = s_wcnt[wi][t];
-            s_wcnt[wi][t] = (uint16_t)s;
+            s_wcnt[wi][t] = s;
             s += c;
         }
         tile_cnt = s;
@@ -252,10 +259,12 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     const uint64_t tiles = (M + kTileItems - 1) / kTileItems;
 
     TmpBuf kb[2], vb[2], hist, dbase, status, counters;
+    trace(s, "sort: enter");
     for (int i = 0; i < 2; ++i) {
         TIGR_TRY(kb[i].alloc(sizeof(uint32_t) * (M ? M : 1), s));
         TIGR_TRY(vb[i].alloc(sizeof(VT) * (M ? M : 1), s));
     }
+    trace(s, "sort: alloc ping-pong");
     TIGR_TRY(hist.alloc(sizeof(unsigned long long) * 4 * kMaxRadix, s));
     TIGR_TRY(dbase.alloc(sizeof(uint64_t) * 4 * kMaxRadix, s));
     TIGR_TRY(status.alloc(sizeof(uint64_t) * kMaxRadix * (tiles ? tiles : 1), s));
@@ -263,6 +272,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     TIGR_CK(cudaMemsetAsync(hist.p, 0, sizeof(unsigned long long) * 4 * kMaxRadix, s));
     TIGR_CK(cudaMemsetAsync(status.p, 0, sizeof(uint64_t) * kMaxRadix * (tiles ? tiles : 1), s));
     TIGR_CK(cudaMemsetAsync(counters.p, 0, sizeof(uint32_t) * 4, s));
+    trace(s, "sort: alloc+memset");
     if (M) {
         k_digit_hist<true><<<sort_grid(M), kBlock, 0, s>>>(src, dst, m, M, passes, bits,
                                                             hist.as<unsigned long long>());
@@ -270,6 +280,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     }
     k_digit_base<<<1, kMaxRadix, 0, s>>>(hist.as<unsigned long long>(), passes, dbase.as<uint64_t>());
     TIGR_CKL("digit base");
+    trace(s, "sort: digit histograms");
     const size_t smem = (sizeof(VT) + sizeof(uint32_t)) * kTileItems;
     int cur = 0;
     for (int p = 0; p < passes && M; ++p) {
@@ -281,6 +292,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
                                                 counters.as<uint32_t>() + p, (uint64_t)(p + 1), kb[out].as<uint32_t>(),
                                                 vb[out].as<VT>());
         TIGR_CKL("onesweep");
+        trace(s, "sort: onesweep pass");
         cur = out;
     }
     std::swap(keys_out.p, kb[cur].p);
@@ -308,6 +320,7 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
         k_runs<<<sort_grid(M), kBlock, 0, s>>>(keys.as<uint32_t>(), M, st.as<uint32_t>(), en.as<uint32_t>());
         TIGR_CKL("runs");
     }
+    trace(s, "csr: runs");
     TIGR_TRY(g->deg.alloc(sizeof(uint32_t) * n, s));
     k_deg_from_runs<<<grid_for(n), kBlock, 0, s>>>(st.as<uint32_t>(), en.as<uint32_t>(), n, g->deg.as<uint32_t>());
     TIGR_CKL("deg");
@@ -319,6 +332,7 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), n, SCAN_CEIL_DIV, kChunk, g->cptr.as<uint32_t>(), s, &nch));
     if (nch >= (1ull << 32)) return fail(TIGR_ERANGE, "graph: padded edge chunks exceed 2^32");
     g->nchunks = nch;
+    trace(s, "csr: deg+scans");
     TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));
     if (W) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));
     if (M) {
@@ -327,6 +341,7 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
                                                     W ? g->wt.as<uint32_t>() : nullptr);
         TIGR_CKL("place");
     }
+    trace(s, "csr: place");
     return TIGR_OK;
 }
 

@@ -44,6 +44,7 @@ struct Workspace {
     DevBuf x;        // double[n] PR rank
     DevBuf contrib;  // double[n] PR x/deg
     DevBuf acc;      // double[n] PR accumulator
+    DevBuf hot;      // uint32: PR hot-destination selection {count[n], hist[33], n_hot, ids[max]}
     DevBuf ctl;      // Ctl
     Ctl* ctl_host = nullptr;  // pinned mirror for the host loop
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
