@@ -186,6 +186,148 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
     }
 }
 
+// Frontier relax with B virtual nodes per thread (16-byte-chunk layouts, no stats): every
+// stage -- vnode -> node id, activity stamp, node record + value, the first two edge (and
+// weight) chunks, the target-value gathers -- is issued for all B vnodes before the first
+// use, so a warp keeps ~8B independent loads in flight instead of one dependent chain.
+template <int A, int LAYOUT, int FRONT, bool BSP, int B>
+__global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
+    constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * kRelaxThreads) + threadIdx.x;
+    const uint32_t it = (FRONT == TIGR_FRONTIER_DENSE) ? a.ctl->it : 0;
+    const uint32_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;   // not written in this launch
+    uint32_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
+    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
+    const uint4* w4 = reinterpret_cast<const uint4*>(a.wt);
+    bool touched = false;
+
+    uint32_t v[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+        v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
+    }
+    bool act[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        act[r] = v[r] != kPad;
+        if (FRONT == TIGR_FRONTIER_DENSE && act[r]) act[r] = __ldg(stamp_cur + v[r]) == it;
+    }
+    uint32_t x[B];
+    uint4 info[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        x[r] = 0;
+        info[r] = make_uint4(0, 0, 0, 1);
+        if (act[r]) {
+            x[r] = BSP ? __ldg(a.prev + v[r]) : a.val[v[r]];
+            info[r] = __ldg(a.vinfo + v[r]);
+        }
+    }
+    uint4 c0[B], c1[B], w0[B], w1[B];
+    uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        if (FRONT == TIGR_FRONTIER_NONE) {
+            if ((A == TIGR_BFS || A == TIGR_SSSP) && x[r] == kInf) act[r] = false;
+            if (A == TIGR_SSWP && x[r] == 0) act[r] = false;
+        }
+        const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+        const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
+        uint32_t k;
+        if (!act[r]) { k = 0; step[r] = 1; kend[r] = 0; }
+        else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
+        else {
+            const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
+            k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
+            kend[r] = (per >= q - k) ? q : k + per;
+        }
+        const uint4 pad4 = make_uint4(kPad, kPad, kPad, kPad);
+        const bool h0 = k < kend[r], h1 = k + step[r] < kend[r];
+        c0[r] = h0 ? ldg_chunk(c4 + info[r].x + k) : pad4;
+        c1[r] = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : pad4;
+        if (W) {
+            w0[r] = h0 ? ldg_chunk(w4 + info[r].x + k) : make_uint4(0, 0, 0, 0);
+            w1[r] = h1 ? ldg_chunk(w4 + info[r].x + k + step[r]) : make_uint4(0, 0, 0, 0);
+        }
+        kn[r] = k + 2 * step[r];
+    }
+    auto relax8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv) {
+        uint32_t cur[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) cur[q] = (nb[q] != kPad) ? a.val[nb[q]] : 0u;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            if (nb[q] == kPad) continue;
+            const uint32_t alt = combine<A>(xv, W ? ww[q] : 0u);
+            if (better<A>(alt, cur[q])) {
+                if (A == TIGR_SSWP) atomicMax(a.val + nb[q], alt);
+                else atomicMin(a.val + nb[q], alt);
+                if (FRONT == TIGR_FRONTIER_DENSE) stamp_next[nb[q]] = it + 1;
+                touched = true;
+            }
+        }
+    };
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+        uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
+                 ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
+        relax8(nb, ww, x[r]);
+    }
+#pragma unroll
+    for (int r = 0; r < B; ++r) {  // chunks beyond the first two (K > 8 or no split)
+        for (uint32_t k = kn[r]; k < kend[r]; k += 2 * step[r]) {
+            const bool h1 = k + step[r] < kend[r];
+            const uint4 a0 = ldg_chunk(c4 + info[r].x + k);
+            const uint4 a1 = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
+            uint4 b0 = make_uint4(0, 0, 0, 0), b1 = b0;
+            if (W) { b0 = ldg_chunk(w4 + info[r].x + k); if (h1) b1 = ldg_chunk(w4 + info[r].x + k + step[r]); }
+            const uint32_t nb[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+            const uint32_t ww[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+            relax8(nb, ww, x[r]);
+        }
+    }
+    if (__any_sync(0xffffffffu, touched) && (threadIdx.x & 31) == 0) a.ctl->changed = 1;
+}
+
+int fr_variant() {
+    const char* e = getenv("TIGR_FR_VARIANT");
+    return e ? atoi(e) : 2;
+}
+
+template <int A, int LAYOUT>
+static RelaxFn pick_mlp(int front, bool bsp, int B) {
+#define TIGR_MLP(F, BS, BB) if (front == F && bsp == BS && B == BB) return &k_relax_mlp<A, LAYOUT, F, BS, BB>;
+    TIGR_MLP(TIGR_FRONTIER_DENSE, false, 2) TIGR_MLP(TIGR_FRONTIER_DENSE, true, 2)
+    TIGR_MLP(TIGR_FRONTIER_NONE, false, 2) TIGR_MLP(TIGR_FRONTIER_NONE, true, 2)
+    TIGR_MLP(TIGR_FRONTIER_DENSE, false, 4) TIGR_MLP(TIGR_FRONTIER_DENSE, true, 4)
+    TIGR_MLP(TIGR_FRONTIER_NONE, false, 4) TIGR_MLP(TIGR_FRONTIER_NONE, true, 4)
+#undef TIGR_MLP
+    return nullptr;
+}
+
+// multi-vnode frontier kernel, or nullptr (then relax_kernel's one-vnode-per-thread kernel)
+RelaxFn relax_mlp_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats, int* per_thread) {
+    const int var = fr_variant();
+    if (!vec || stats || var == 0 || algo == TIGR_PR) return nullptr;
+    const int B = var == 1 ? 2 : 4;
+    *per_thread = B;
+    const bool st = layout == TIGR_LAYOUT_STRIDED;
+    switch (algo) {
+        case TIGR_BFS: return st ? pick_mlp<TIGR_BFS, TIGR_LAYOUT_STRIDED>(front, bsp, B)
+                                 : pick_mlp<TIGR_BFS, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
+        case TIGR_SSSP: return st ? pick_mlp<TIGR_SSSP, TIGR_LAYOUT_STRIDED>(front, bsp, B)
+                                  : pick_mlp<TIGR_SSSP, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
+        case TIGR_CC: return st ? pick_mlp<TIGR_CC, TIGR_LAYOUT_STRIDED>(front, bsp, B)
+                                : pick_mlp<TIGR_CC, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
+        case TIGR_SSWP: return st ? pick_mlp<TIGR_SSWP, TIGR_LAYOUT_STRIDED>(front, bsp, B)
+                                  : pick_mlp<TIGR_SSWP, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
+    }
+    return nullptr;
+}
+
 template <int LAYOUT, bool VEC, bool STATS>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax_pr(RelaxArgs a) {
     const uint64_t i = (uint64_t)a.lo + (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
@@ -348,7 +490,7 @@ __global__ void k_hot_compact(const uint32_t* __restrict__ cnt, uint32_t n, cons
 }
 
 // LOGS: log2 of the table size (2^LOGS slots, at most 2^LOGS / 4 hot ids); MINB: blocks/SM
-template <int LAYOUT, int B, int LOGS, int MINB>
+template <int LAYOUT, int B, int LOGS, int MINB, int MASKBITS = 0>
 __global__ void __launch_bounds__(kRelaxThreads, MINB) k_relax_pr_hot(RelaxArgs a, const uint32_t* __restrict__ hot_ids,
                                                                      const uint32_t* __restrict__ n_hot_p, uint32_t tiles) {
     constexpr int kSlots = 1 << LOGS;
@@ -372,7 +514,10 @@ __global__ void __launch_bounds__(kRelaxThreads, MINB) k_relax_pr_hot(RelaxArgs 
         for (;;) {
             const uint32_t k = s_key[s];
             if (k == nb) { atomicAdd(&s_acc[s], x); return; }
-            if (k == kPad) { red_add_f64(a.acc + nb, x, pol); return; }
+            if (k == kPad) {  // MASKBITS: timing experiment only (folds targets into 2^MASKBITS slots)
+                red_add_f64(a.acc + (MASKBITS ? (nb & ((1u << MASKBITS) - 1)) : nb), x, pol);
+                return;
+            }
             s = (s + 1) & (kSlots - 1);
         }
     };
@@ -462,11 +607,11 @@ tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uin
     return TIGR_OK;
 }
 
-template <int B, int LOGS, int MINB>
+template <int B, int LOGS, int MINB, int MASKBITS = 0>
 static PrHotConfig make_hot(int layout) {
     PrHotConfig c;
-    c.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_hot<TIGR_LAYOUT_STRIDED, B, LOGS, MINB>
-                                         : &k_relax_pr_hot<TIGR_LAYOUT_CONSECUTIVE, B, LOGS, MINB>;
+    c.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_hot<TIGR_LAYOUT_STRIDED, B, LOGS, MINB, MASKBITS>
+                                         : &k_relax_pr_hot<TIGR_LAYOUT_CONSECUTIVE, B, LOGS, MINB, MASKBITS>;
     c.vnodes_per_thread = B;
     c.smem = (sizeof(double) + sizeof(uint32_t)) << LOGS;
     c.max_ids = (1u << LOGS) / 4;
@@ -484,6 +629,8 @@ PrHotConfig relax_pr_hot_config(int layout, bool vec) {
         case 8: return make_hot<4, 12, 3>(layout);
         case 9: return make_hot<4, 11, 3>(layout);
         case 10: return make_hot<2, 12, 4>(layout);
+        case 11: return make_hot<4, 13, 2, 23>(layout);   // timing experiment: wrong results
+        case 12: return make_hot<4, 13, 2, 22>(layout);   // timing experiment: wrong results
         default: return none;
     }
 }

@@ -26,6 +26,8 @@ typedef void (*RelaxFn)(RelaxArgs);
 typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
 
 RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats);
+// frontier relax with *per_thread virtual nodes per thread (nullptr: use relax_kernel's)
+RelaxFn relax_mlp_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats, int* per_thread);
 // PageRank push with several virtual nodes per thread (nullptr: use relax_kernel's); B per thread
 RelaxFn relax_pr_mlp_kernel(int layout, bool vec, bool stats);
 int pr_vnodes_per_thread(int layout, bool vec, bool stats);

@@ -125,7 +125,13 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     p.relax = relax_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0);
     if (!p.relax) return fail(TIGR_EUNSUPPORTED, "no relax kernel for this option combination");
     p.args = make_args(vg);
-    p.grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + kRelaxThreads - 1) / kRelaxThreads);
+    int per_thread = 1;
+    if (RelaxFn mlp = relax_mlp_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0, &per_thread))
+        p.relax = mlp;
+    else
+        per_thread = 1;
+    const uint64_t per_block = (uint64_t)kRelaxThreads * per_thread;
+    p.grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
     const uint32_t max_iters = o.max_iters ? o.max_iters : (n + 1 > n ? n + 1 : n);
 
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];

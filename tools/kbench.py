@@ -61,7 +61,8 @@ def main():
         for algo in ("bfs", "sssp", "sswp"):
             ts = []
             for _ in range(reps):
-                _, st = tigr.tigr_run(vgw, algo, 0, out=o32, stream=s, return_stats=True)
+                _, st = tigr.tigr_run(vgw, algo, 0, out=o32, stream=s, return_stats=True,
+                                      use_graph=int(os.environ.get("USE_GRAPH", "1")))
                 ts.append(st["ms_total"])
             res[algo + "_ms"] = min(ts)
             res[algo + "_iters"] = st["iterations"]
@@ -71,7 +72,8 @@ def main():
         vgs = tigr.tigr_virtualize(gs, K, layout, stream=s)
         ts = []
         for _ in range(reps):
-            _, st = tigr.tigr_run(vgs, "cc", 0, out=o32, stream=s, return_stats=True)
+            _, st = tigr.tigr_run(vgs, "cc", 0, out=o32, stream=s, return_stats=True,
+                                  use_graph=int(os.environ.get("USE_GRAPH", "1")))
             ts.append(st["ms_total"])
         res["cc_ms"] = min(ts)
         res["cc_iters"] = st["iterations"]
