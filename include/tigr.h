@@ -179,6 +179,13 @@ tigr_status tigr_vgraph_partition(tigr_vgraph* vg, int nranks, int rank);
 
 void tigr_vgraph_free(tigr_vgraph* vg);
 
+/* The range rule tigr_vgraph_partition applies, as a pure HOST computation (no device needed):
+ * from host row_ptr[n+1] (int64) and vnode_ptr[n+1] (uint32), rank r of nranks owns vnodes
+ * [lo[r], hi[r]) = the virtual nodes of nodes [cut(r), cut(r+1)), where cut(r) is the first node
+ * whose arc prefix reaches r*m/nranks.  Ranges are contiguous, family-aligned and cover [0, NV). */
+tigr_status tigr_partition_ranges(uint32_t n, const int64_t* row_ptr, const uint32_t* vnode_ptr, int nranks,
+                                  uint32_t* lo, uint32_t* hi);
+
 /* ------------------------------------------------------------------ runs ---- */
 
 /* Run `algo` from `source` (ignored by CC and PR) to the fixed point (PR: pr_iters

@@ -76,6 +76,7 @@ _SIGS = {
     "tigr_vgraph_export": (_I, [_P, _P, _P, _I, _P]),
     "tigr_vgraph_assignment": (_I, [_P, _P, _P, _P, _I, _P]),
     "tigr_vgraph_partition": (_I, [_P, _I, _I]),
+    "tigr_partition_ranges": (_I, [_U32, _P, _P, _I, _P, _P]),
     "tigr_vgraph_free": (None, [_P]),
     "tigr_run": (_I, [_P, _I, _U32, ctypes.POINTER(tigr_run_opts), _P, _I, ctypes.POINTER(tigr_stats)]),
     "tigr_comm_unique_id": (_I, [_P]),
@@ -294,6 +295,17 @@ def tigr_vgraph_assignment(vg: VGraph, stream=None):
 
 def tigr_vgraph_partition(vg: VGraph, nranks: int, rank: int):
     _check(_lib.tigr_vgraph_partition(vg.ptr, nranks, rank))
+
+
+def tigr_partition_ranges(row_ptr, vnode_ptr, nranks: int):
+    """Host-only: (lo[nranks], hi[nranks]) vnode ranges from host row_ptr / vnode_ptr arrays."""
+    rp = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    vp = np.ascontiguousarray(vnode_ptr, dtype=np.uint32)
+    lo = np.empty(nranks, dtype=np.uint32)
+    hi = np.empty(nranks, dtype=np.uint32)
+    _check(_lib.tigr_partition_ranges(len(rp) - 1, rp.ctypes.data, vp.ctypes.data, nranks, lo.ctypes.data,
+                                      hi.ctypes.data))
+    return lo, hi
 
 
 def tigr_run(vg: VGraph, algo, source=0, opts: tigr_run_opts | None = None, out=None, stream=None,

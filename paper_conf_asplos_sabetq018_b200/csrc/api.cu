@@ -168,6 +168,7 @@ tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const t
                        int out_is_device, tigr_stats* st);
 tigr_status assignment_device(const tigr_vgraph* vg, uint32_t* counts, uint32_t* nbr, uint32_t* w, cudaStream_t s);
 tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank);
+void partition_ranges(uint32_t n, const int64_t* rp, const uint32_t* vp, int nranks, uint32_t* lo, uint32_t* hi);
 tigr_status comm_unique_id(uint8_t id[128]);
 tigr_status comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
 void comm_free(tigr_comm* c);
@@ -363,6 +364,13 @@ tigr_status tigr_vgraph_partition(tigr_vgraph* vg, int nranks, int rank) {
 }
 
 void tigr_vgraph_free(tigr_vgraph* vg) { delete vg; }
+
+tigr_status tigr_partition_ranges(uint32_t n, const int64_t* row_ptr, const uint32_t* vnode_ptr, int nranks,
+                                  uint32_t* lo, uint32_t* hi) {
+    if (!row_ptr || !vnode_ptr || !lo || !hi || nranks < 1) return fail(TIGR_EINVAL, "partition_ranges: bad argument");
+    partition_ranges(n, row_ptr, vnode_ptr, nranks, lo, hi);
+    return TIGR_OK;
+}
 
 tigr_status tigr_run(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tigr_run_opts* opts, void* out_values,
                      int out_is_device, tigr_stats* stats) {

@@ -118,7 +118,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     int front = o.frontier == TIGR_FRONTIER_AUTO ? TIGR_FRONTIER_DENSE : o.frontier;
     FrontierPlan p;
     p.bsp = o.schedule == 1;
-    p.comm = o.comm != nullptr && o.comm->nranks > 1;
+    p.comm = o.comm != nullptr;  // a 1-rank communicator still runs the exchange path (tests)
     p.c = o.comm;
     p.algo = algo;
     p.n = n;
@@ -253,7 +253,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     if (relax) per_block *= pr_vnodes_per_thread(vg->layout, vg->vec, o.collect_stats != 0);
     else relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
     const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
-    const bool comm = o.comm != nullptr && o.comm->nranks > 1;
+    const bool comm = o.comm != nullptr;
     const double base = (1.0 - o.pr_damping) / (double)n;
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
     TIGR_CK(cudaEventRecord(t0, s));
@@ -370,7 +370,22 @@ tigr_status assignment_device(const tigr_vgraph* vgc, uint32_t* counts, uint32_t
     return TIGR_OK;
 }
 
-// contiguous, family-aligned vnode ranges with ~equal edge counts
+// contiguous, family-aligned vnode ranges with ~equal edge counts: rank r owns
+// the vnodes of nodes [cut(r), cut(r+1)), cut(r) = first node whose arc prefix reaches r*m/P
+void partition_ranges(uint32_t n, const int64_t* rp, const uint32_t* vp, int nranks, uint32_t* lo, uint32_t* hi) {
+    const uint64_t m = (uint64_t)rp[n];
+    auto cut = [&](int r) -> uint32_t {
+        if (r <= 0) return 0;
+        if (r >= nranks) return n;
+        const int64_t target = (int64_t)((unsigned __int128)m * (unsigned)r / (unsigned)nranks);
+        return (uint32_t)(std::lower_bound(rp, rp + n, target) - rp);
+    };
+    for (int r = 0; r < nranks; ++r) {
+        lo[r] = vp[cut(r)];
+        hi[r] = vp[cut(r + 1)];
+    }
+}
+
 tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank) {
     if (nranks < 1 || rank < 0 || rank >= nranks) return fail(TIGR_EINVAL, "partition: bad rank/nranks");
     const tigr_graph* g = vg->g;
@@ -379,14 +394,10 @@ tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank) {
     std::vector<uint32_t> vp((size_t)g->n + 1);
     TIGR_CK(cudaMemcpy(rp.data(), g->row_ptr.p, sizeof(int64_t) * rp.size(), cudaMemcpyDeviceToHost));
     TIGR_CK(cudaMemcpy(vp.data(), vg->vnode_ptr.p, sizeof(uint32_t) * vp.size(), cudaMemcpyDeviceToHost));
-    auto cut = [&](int r) -> uint32_t {  // first vertex whose edge prefix reaches r/nranks of m
-        if (r <= 0) return 0;
-        if (r >= nranks) return g->n;
-        const int64_t target = (int64_t)((__int128)g->m * r / nranks);
-        return (uint32_t)(std::lower_bound(rp.begin(), rp.end() - 1, target) - rp.begin());
-    };
-    vg->lo = vp[cut(rank)];
-    vg->hi = vp[cut(rank + 1)];
+    std::vector<uint32_t> lo(nranks), hi(nranks);
+    partition_ranges(g->n, rp.data(), vp.data(), nranks, lo.data(), hi.data());
+    vg->lo = lo[rank];
+    vg->hi = hi[rank];
     return TIGR_OK;
 }
 

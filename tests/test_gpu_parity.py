@@ -306,3 +306,23 @@ def test_partition_ranges(tigr):
         assert all(bounds[r][1] == bounds[r + 1][0] for r in range(P - 1))
     tigr.tigr_vgraph_partition(vg, 1, 0)
     assert vg.info()["hi"] == nv
+
+
+def test_exchange_path_single_rank_nccl(tigr):
+    """The multi-GPU code path (NCCL all-reduce every iteration, k_diff activation, host loop)
+    on a 1-rank communicator: results must not change."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    comm = tigr.tigr_comm_init(1, 0, tigr.tigr_comm_unique_id())
+    want = _oracle_all(rec.n, src, dst, w)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    gs = tigr.tigr_graph_from_coo(rec.n, src, dst, None, symmetrize=True)
+    vg = tigr.tigr_virtualize(g, 8)
+    vgs = tigr.tigr_virtualize(gs, 8)
+    tigr.tigr_vgraph_partition(vg, 1, 0)
+    for algo in ("bfs", "sssp", "sswp"):
+        assert np.array_equal(tigr.tigr_run(vg, algo, 0, comm=comm), want[algo]), algo
+        assert np.array_equal(tigr.tigr_run(vg, algo, 0, comm=comm, schedule=1), want[algo]), algo
+    assert np.array_equal(tigr.tigr_run(vgs, "cc", comm=comm), want["cc"])
+    assert np.abs(tigr.tigr_run(vg, "pr", comm=comm) - want["pr"]).max() <= 1e-6
+    comm.free()

@@ -1,0 +1,85 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times
+(K = 8, strided layout, default kernels: hot-destination PR, 4-vnodes-per-thread frontier
+kernels, CUDA-graph loop).  The oracle computes the full results on the host copy of the
+same seeded graph (graphgen/, bit-identical to the device generator), so the comparison is
+element by element: bit-exact for BFS/SSSP/CC/SSWP, max |diff| <= 1e-6 for PageRank."""
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+@pytest.fixture(scope="module")
+def tigr():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_asplos_sabetq018_b200 as t
+    return t
+
+
+@pytest.fixture(scope="module")
+def cfg4():
+    rec = graphgen.recipe("cfg4")
+    src, dst, w = graphgen.generate(rec)
+    return rec, src, dst, w
+
+
+def test_cfg4_pagerank_full(tigr, cfg4):
+    """The bench workload itself: R-MAT scale 24, PageRank 20 iterations, K=8 strided."""
+    rec, src, dst, _ = cfg4
+    g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False)
+    vg = tigr.tigr_virtualize(g, 8, "strided")
+    got = tigr.tigr_run(vg, "pr")
+    want = oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20)
+    err = np.abs(got - want).max()
+    assert err <= 1e-6, err
+    # normalised error too (values are ~6e-8, so also demand relative agreement)
+    assert np.abs(rec.n * got - rec.n * want).max() <= 1e-6
+
+
+def test_cfg4_frontier_algorithms_full(tigr, cfg4):
+    rec, src, dst, w = cfg4
+    g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax,
+                             weighted=True)
+    vg = tigr.tigr_virtualize(g, 8, "strided")
+    o = oracle.csr_build(rec.n, src, dst, w)
+    assert np.array_equal(tigr.tigr_run(vg, "bfs", 0), oracle.bfs(o, 0))
+    assert np.array_equal(tigr.tigr_run(vg, "sssp", 0), oracle.sssp(o, 0))
+    assert np.array_equal(tigr.tigr_run(vg, "sswp", 0), oracle.sswp(o, 0))
+    del vg, g, o
+    gs = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False,
+                              symmetrize=True)
+    vgs = tigr.tigr_virtualize(gs, 8, "strided")
+    assert np.array_equal(tigr.tigr_run(vgs, "cc"), oracle.cc(rec.n, src, dst))
+
+
+@pytest.mark.parametrize("K", [4, 8, 16, 32])
+def test_cfg3_sssp_sswp_k_sweep(tigr, K, cfg3_oracle):
+    rec, want_sssp, want_sswp = cfg3_oracle
+    g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax,
+                             weighted=True)
+    vg = tigr.tigr_virtualize(g, K, "strided")
+    assert np.array_equal(tigr.tigr_run(vg, "sssp", rec.source), want_sssp)
+    assert np.array_equal(tigr.tigr_run(vg, "sswp", rec.source), want_sswp)
+
+
+@pytest.fixture(scope="module")
+def cfg3_oracle():
+    rec = graphgen.recipe("cfg3")
+    src, dst, w = graphgen.generate(rec)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    return rec, oracle.sssp(o, rec.source), oracle.sswp(o, rec.source)
+
+
+def test_cfg4_pagerank_k_and_layout_invariance(tigr, cfg4):
+    """Thm. 2: the virtual split does not change the result (PR up to summation order)."""
+    rec = cfg4[0]
+    g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False)
+    ref = tigr.tigr_run(tigr.tigr_virtualize(g, 8, "strided"), "pr")
+    for K, lay in ((4, "strided"), (32, "consecutive"), (0xFFFFFFFF, "strided")):
+        got = tigr.tigr_run(tigr.tigr_virtualize(g, K, lay), "pr")
+        assert np.abs(got - ref).max() <= 1e-12, (K, lay)
