@@ -1,0 +1,273 @@
+// pr.cu -- PageRank push with an in-degree-ordered accumulator (PR).
+//
+// The push relax adds contrib[u] = x[u]/d_u into acc[v] for every arc u->v with a float64
+// reduction (fn. 7 L1078; Thm. 3).  At scale 24 the accumulator is 134 MB, which
+// does not fit the 126 MB L2, and power-law in-degrees make the reductions collide on a few
+// sectors.  Measured on B200 (tools/micro/red_bench.cu): spread REDs run at ~190 G/s on an
+// L2-resident array, ~61 G/s once the array exceeds L2, ~70 G/s under R-MAT skew.
+//
+// So, once per graph, destinations get a dense "accumulator id" cid in order of decreasing
+// (sampled) in-degree, vertices without in-arcs last:
+//   * every arc's reduction lands in the first n_in entries (59 MB at scale 24: L2-resident);
+//   * the S hottest destinations (cid < S) are accumulated in shared memory by each persistent
+//     block and flushed once per block -- no hashing, the test is cid < S;
+// and the PR-only arc array col_pr = cid[col] is built next to the CSR.  The sources, the
+// virtual split and its strided layout are untouched: thread i still owns virtual node i and
+// its <= K arcs, and reads contrib[v] of its physical node v.  Apply reads acc[cid[v]].
+// Same sums as the plain push, associated differently (PR parity is 1e-6).
+#include <algorithm>
+
+#include "devutil.cuh"
+#include "internal.cuh"
+#include "relax.cuh"
+#include "vgraph.cuh"
+
+namespace tigr {
+
+tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t count, uint32_t key_limit,
+                           cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out);
+__global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uint32_t* __restrict__ cnt);
+
+namespace {
+
+constexpr int kCidSlots = 8192;   // shared-memory accumulator entries (64 KB of f64)
+
+__global__ void k_indeg_flag(const uint4* __restrict__ c4, uint64_t nchunks, uint8_t* __restrict__ flag) {
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
+         k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 c = ldg_chunk(c4 + k);
+        if (c.x != kPad) flag[c.x] = 1;
+        if (c.y != kPad) flag[c.y] = 1;
+        if (c.z != kPad) flag[c.z] = 1;
+        if (c.w != kPad) flag[c.w] = 1;
+    }
+}
+
+// sort key: vertices with in-arcs first, by decreasing floor(log2(sampled count)); ties by id
+__global__ void k_pr_key(const uint8_t* __restrict__ flag, const uint32_t* __restrict__ cnt, uint32_t n,
+                         uint32_t* __restrict__ key, uint32_t* __restrict__ ids, uint32_t* __restrict__ n_in) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    bool in = false;
+    if (v < n) {
+        in = flag[v] != 0;
+        const uint32_t c = cnt[v];
+        const uint32_t b = c ? 32u - __clz(c) : 0u;  // 0..32
+        key[v] = in ? 32u - b : 33u;                 // 0..33
+        ids[v] = v;
+    }
+    const uint32_t ballot = __ballot_sync(0xffffffffu, in);
+    if ((threadIdx.x & 31) == 0 && ballot) atomicAdd(n_in, (uint32_t)__popc(ballot));
+}
+
+__global__ void k_cid_scatter(const uint32_t* __restrict__ order, uint32_t n, uint32_t* __restrict__ cid) {
+    const uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c < n) cid[order[c]] = c;
+}
+
+__global__ void k_build_col_pr(const uint4* __restrict__ c4, uint64_t nchunks, const uint32_t* __restrict__ cid,
+                               uint4* __restrict__ out) {
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
+         k += (uint64_t)gridDim.x * blockDim.x) {
+        uint4 c = ldg_chunk(c4 + k);
+        c.x = c.x == kPad ? kPad : __ldg(cid + c.x);
+        c.y = c.y == kPad ? kPad : __ldg(cid + c.y);
+        c.z = c.z == kPad ? kPad : __ldg(cid + c.z);
+        c.w = c.w == kPad ? kPad : __ldg(cid + c.w);
+        out[k] = c;
+    }
+}
+
+template <int LAYOUT, int B>
+__global__ void __launch_bounds__(kRelaxThreads, 2) k_relax_pr_cid(RelaxArgs a, const uint32_t* __restrict__ col_pr,
+                                                                   uint32_t tiles) {
+    extern __shared__ __align__(16) double s_acc[];  // kCidSlots entries (dynamic: 64 KB)
+    const int t = threadIdx.x;
+    for (int i = t; i < kCidSlots; i += kRelaxThreads) s_acc[i] = 0.0;
+    __syncthreads();
+    const uint64_t pol = policy_evict_last();
+    const uint4* c4 = reinterpret_cast<const uint4*>(col_pr);
+    auto push = [&](uint32_t c, double x) {
+        if (c < (uint32_t)kCidSlots) atomicAdd(&s_acc[c], x);
+        else red_add_f64(a.acc + c, x, pol);
+    };
+    for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        const uint64_t base = (uint64_t)a.lo + (uint64_t)tile * (B * kRelaxThreads) + t;
+        uint32_t v[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+            v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
+        }
+        uint4 info[B];
+        double x[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            info[r] = make_uint4(0, 0, 0, 1);
+            x[r] = 0.0;
+            if (v[r] != kPad) { info[r] = __ldg(a.vinfo + v[r]); x[r] = __ldg(a.contrib + v[r]); }
+        }
+        uint4 c0[B], c1[B];
+        uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+            const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
+            uint32_t k;
+            if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
+            else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
+            else {
+                const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
+                k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
+                kend[r] = (per >= q - k) ? q : k + per;
+            }
+            const uint4* cb = c4 + info[r].x;
+            c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
+            c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
+            kn[r] = k + 2 * step[r];
+        }
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+                if (nb[q] != kPad) push(nb[q], x[r]);
+        }
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint4* cb = c4 + info[r].x;
+            for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
+                const uint4 c = ldg_chunk(cb + k);
+                const uint32_t nb[4] = {c.x, c.y, c.z, c.w};
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    if (nb[q] != kPad) push(nb[q], x[r]);
+            }
+        }
+    }
+    __syncthreads();
+    for (int i = t; i < kCidSlots; i += kRelaxThreads)
+        if (s_acc[i] != 0.0) red_add_f64(a.acc + i, s_acc[i], pol);
+}
+
+// x = (1-d)/n + d*(acc[cid[v]] + dsum/n); contrib = x/deg; next dangling mass -> dsum_next
+__global__ void k_pr_apply_cid(uint32_t n, const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cid,
+                               uint32_t n_in, double base, double damping, int dangling, double* __restrict__ x,
+                               double* __restrict__ contrib, const double* __restrict__ acc,
+                               const double* dsum_cur, double* dsum_next) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    double dang = 0.0;
+    if (v < n) {
+        const uint32_t c = cid[v];
+        double s = c < n_in ? acc[c] : 0.0;
+        if (dangling) s = __dadd_rn(s, __ddiv_rn(*dsum_cur, (double)n));
+        const double r = __dadd_rn(base, __dmul_rn(damping, s));  // no FMA: matches the oracle
+        const uint32_t d = deg[v];
+        x[v] = r;
+        contrib[v] = d ? __ddiv_rn(r, (double)d) : 0.0;
+        if (!d) dang = r;
+    }
+    if (dangling) {
+        __shared__ double part[kBlock / 32];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) dang += __shfl_xor_sync(0xffffffffu, dang, o);
+        if ((threadIdx.x & 31) == 0) part[threadIdx.x >> 5] = dang;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            double tt = 0.0;
+            for (int w = 0; w < kBlock / 32; ++w) tt += part[w];
+            if (tt != 0.0) atomicAdd(dsum_next, tt);
+        }
+    }
+}
+
+unsigned grid_cap(uint64_t items, int per_sm) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t want = (items + kBlock - 1) / kBlock;
+    const uint64_t cap = (uint64_t)sms * per_sm;
+    return (unsigned)(want == 0 ? 1 : (want < cap ? want : cap));
+}
+
+}  // namespace
+
+bool pr_cid_enabled() {
+    const char* e = getenv("TIGR_PR_VARIANT");
+    return !e || atoi(e) == 13;
+}
+
+// once per vgraph: cid order, n_in, col_pr (workspace), all on the device
+tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
+    Workspace& ws = vg->ws;
+    if (ws.cid_ready) return TIGR_OK;
+    const tigr_graph* g = vg->g;
+    const uint32_t n = g->n;
+    TIGR_TRY(ws.cid.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(ws.col_pr.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
+    TmpBuf flag, cnt, key, ids, nin;
+    TIGR_TRY(flag.alloc(n ? n : 1, s));
+    TIGR_TRY(cnt.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(key.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(ids.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(nin.alloc(sizeof(uint32_t), s));
+    TIGR_CK(cudaMemsetAsync(flag.p, 0, n, s));
+    TIGR_CK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * n, s));
+    TIGR_CK(cudaMemsetAsync(nin.p, 0, sizeof(uint32_t), s));
+    const uint4* c4 = g->col.as<uint4>();
+    if (g->nchunks) {
+        k_indeg_flag<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, flag.as<uint8_t>());
+        TIGR_CKL("pr indeg flag");
+        k_hot_sample<<<grid_cap(g->nchunks / 16 + 1, 16), kBlock, 0, s>>>(c4, g->nchunks, cnt.as<uint32_t>());
+        TIGR_CKL("pr sample");
+    }
+    k_pr_key<<<grid_for(n), kBlock, 0, s>>>(flag.as<uint8_t>(), cnt.as<uint32_t>(), n, key.as<uint32_t>(),
+                                             ids.as<uint32_t>(), nin.as<uint32_t>());
+    TIGR_CKL("pr key");
+    TmpBuf skeys, order;
+    TIGR_TRY(sort_pairs_u32(key.as<uint32_t>(), ids.as<uint32_t>(), n, 34, s, skeys, order));
+    k_cid_scatter<<<grid_for(n), kBlock, 0, s>>>(order.as<uint32_t>(), n, ws.cid.as<uint32_t>());
+    TIGR_CKL("pr cid");
+    if (g->nchunks) {
+        k_build_col_pr<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, ws.cid.as<uint32_t>(),
+                                                                    ws.col_pr.as<uint4>());
+        TIGR_CKL("pr col_pr");
+    }
+    uint32_t h = 0;
+    TIGR_CK(cudaMemcpyAsync(&h, nin.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    ws.n_in = h;
+    ws.cid_ready = true;
+    return TIGR_OK;
+}
+
+PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
+    PrCidPlan p;
+    const int B = 4;
+    p.fn = vg->layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, B>
+                                             : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, B>;
+    p.smem = sizeof(double) * kCidSlots;
+    cudaFuncSetAttribute(p.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
+    int per_sm = 0, dev = 0, sms = 148;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, p.fn, kRelaxThreads, p.smem);
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t per_tile = (uint64_t)kRelaxThreads * B;
+    p.tiles = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_tile - 1) / per_tile);
+    p.grid = (unsigned)std::min<uint64_t>(p.tiles, (uint64_t)sms * (per_sm > 0 ? per_sm : 1));
+    return p;
+}
+
+tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,
+                         double* dsum_next, cudaStream_t s) {
+    Workspace& ws = vg->ws;
+    const uint32_t n = vg->g->n;
+    k_pr_apply_cid<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), ws.cid.as<uint32_t>(), ws.n_in, base,
+                                                  damping, dangling, ws.x.as<double>(), ws.contrib.as<double>(),
+                                                  ws.acc.as<double>(), dsum_cur, dsum_next);
+    TIGR_CKL("pr apply (cid)");
+    // only the first n_in accumulator entries are ever written
+    TIGR_CK(cudaMemsetAsync(ws.acc.p, 0, sizeof(double) * ws.n_in, s));
+    return TIGR_OK;
+}
+
+}  // namespace tigr

@@ -17,6 +17,7 @@
 #include "internal.cuh"
 #include "vgraph.cuh"
 #include "relax.cuh"
+#include "devutil.cuh"
 
 #include <algorithm>
 
@@ -25,39 +26,6 @@ namespace tigr {
 // ------------------------------------------------------------------------------------------
 // edge walk: the set of (nbr, w) slots a virtual node owns, in the layout's order
 // ------------------------------------------------------------------------------------------
-// Read-only streaming loads (edge / weight chunks): not allocated in L1, and marked
-// evict-first in L2 so that the 1+ GB edge stream does not push the value / accumulator
-// arrays out of the 126 MB L2.  Not volatile: the compiler may hoist them.
-__device__ __forceinline__ uint64_t policy_evict_first() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-
-__device__ __forceinline__ uint64_t policy_evict_last() {
-    uint64_t p;
-    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-    return p;
-}
-
-__device__ __forceinline__ uint4 ldg_chunk(const uint4* p) {
-    uint4 r;
-    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-        : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(policy_evict_first()));
-    return r;
-}
-
-__device__ __forceinline__ uint32_t ldg_u32(const uint32_t* p) {
-    uint32_t r;
-    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(policy_evict_first()));
-    return r;
-}
-
-// fire-and-forget float64 add into the accumulator, kept resident in L2 (evict-last)
-__device__ __forceinline__ void red_add_f64(double* p, double v, uint64_t pol) {
-    asm volatile("red.global.add.L2::cache_hint.f64 [%0], %1, %2;" :: "l"(p), "d"(v), "l"(pol) : "memory");
-}
-
 // Calls f(nbr[8], w[8]) on batches of up to 8 slots (pads/absent = kPad).
 template <int LAYOUT, bool VEC, bool W, class F>
 __device__ __forceinline__ void walk(const uint32_t* __restrict__ col, const uint32_t* __restrict__ wt,

@@ -40,6 +40,17 @@ struct PrHotConfig {
     uint32_t max_ids = 0;     // hot destinations the table holds
 };
 PrHotConfig relax_pr_hot_config(int layout, bool vec);
+// PageRank push with an in-degree-ordered accumulator (pr.cu)
+struct PrCidPlan {
+    void (*fn)(RelaxArgs, const uint32_t*, uint32_t) = nullptr;
+    unsigned grid = 0, tiles = 0;
+    size_t smem = 0;
+};
+bool pr_cid_enabled();
+tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s);
+PrCidPlan pr_cid_plan(tigr_vgraph* vg);
+tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,
+                         double* dsum_next, cudaStream_t s);
 uint32_t pr_hot_max();        // capacity of the workspace's hot-id list (>= any config's max_ids)
 tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uint32_t max_ids, uint32_t* cnt_tmp,
                           uint32_t* hist_tmp, uint32_t* hot_ids, uint32_t* n_hot, cudaStream_t s);

@@ -228,8 +228,14 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     Workspace& ws = vg->ws;
     const uint32_t n = vg->g->n;
     RelaxArgs a = make_args(vg);
-    // preferred: persistent kernel with the hottest destinations privatised in shared memory
-    const PrHotConfig hc = o.collect_stats ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
+    // preferred: in-degree-ordered accumulator (pr.cu); else the hashed hot-destination kernel
+    const bool use_cid = !o.collect_stats && vg->vec && pr_cid_enabled();
+    PrCidPlan cp;
+    if (use_cid) {
+        TIGR_TRY(pr_cid_prepare(vg, s));
+        cp = pr_cid_plan(vg);
+    }
+    const PrHotConfig hc = (o.collect_stats || use_cid) ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
     const RelaxHotFn hot = hc.fn;
     uint32_t* hot_cnt = ws.hot.as<uint32_t>();
     uint32_t* hot_hist = hot_cnt + n;
@@ -272,7 +278,11 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     }
     for (uint32_t t = 0; t < o.pr_iters; ++t) {
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t], s));
-        if (hot && hot_tiles) {
+        if (use_cid && cp.tiles) {
+            cp.fn<<<cp.grid, kRelaxThreads, cp.smem, s>>>(a, ws.col_pr.as<uint32_t>(), cp.tiles);
+            TIGR_CKL("pr relax (cid)");
+            ++launches;
+        } else if (hot && hot_tiles) {
             hot<<<hot_grid, kRelaxThreads, hc.smem, s>>>(a, hot_ids, hot_n, hot_tiles);
             TIGR_CKL("pr relax (hot)");
             ++launches;
@@ -287,6 +297,10 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         double* dcur = &a.ctl->dsum[t & 1];
         double* dnext = &a.ctl->dsum[(t + 1) & 1];
         if (o.pr_dangling) TIGR_CK(cudaMemsetAsync(dnext, 0, sizeof(double), s));
+        if (use_cid) {
+            TIGR_TRY(pr_cid_apply(vg, base, o.pr_damping, o.pr_dangling, dcur, dnext, s));
+            continue;
+        }
         k_pr_apply<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), base, o.pr_damping, o.pr_dangling,
                                                   ws.x.as<double>(), ws.contrib.as<double>(), ws.acc.as<double>(),
                                                   dcur, dnext);

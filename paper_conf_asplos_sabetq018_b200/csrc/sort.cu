@@ -347,6 +347,13 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
 
 }  // namespace
 
+// Stable sort of (key, value) u32 pairs by key (keys < key_limit); results owned by the TmpBufs.
+tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t count, uint32_t key_limit,
+                           cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out) {
+    keys_out.s = vals_out.s = s;
+    return sort_arcs<false>(keys, vals, nullptr, count, count, key_limit, s, keys_out, vals_out);
+}
+
 // Stable device CSR build from an arc list (device pointers).  Caller validated ids < n.
 tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
                              int symmetrize, cudaStream_t s, tigr_graph* g) {

@@ -45,6 +45,10 @@ struct Workspace {
     DevBuf contrib;  // double[n] PR x/deg
     DevBuf acc;      // double[n] PR accumulator
     DevBuf hot;      // uint32: PR hot-destination selection {count[n], hist[33], n_hot, ids[max]}
+    DevBuf cid;      // uint32[n]: PR accumulator id (in-degree order; pr.cu)
+    DevBuf col_pr;   // uint32[4 * nchunks]: arc targets as accumulator ids (PR only)
+    uint32_t n_in = 0;       // nodes with in-arcs (= accumulator entries ever written)
+    bool cid_ready = false;
     DevBuf ctl;      // Ctl
     Ctl* ctl_host = nullptr;  // pinned mirror for the host loop
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
