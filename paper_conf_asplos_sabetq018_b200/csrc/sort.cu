@@ -19,6 +19,9 @@ namespace tigr {
 namespace {
 
 constexpr int kST = 256;                 // threads per sort tile
+#ifndef TIGR_SORT_MINB
+#define TIGR_SORT_MINB 3
+#endif
 constexpr int kSI = 16;                  // items per thread
 constexpr int kSW = kST / 32;            // warps per tile
 constexpr int kTileItems = kST * kSI;    // 4096
@@ -77,8 +80,16 @@ __global__ void k_digit_base(const unsigned long long* __restrict__ hist, int pa
     }
 }
 
+__device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
+    const uint32_t d = (uint32_t)__cvta_generic_to_shared(smem_dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(d), "l"(gsrc) : "memory");
+}
+
+// One pass of the stable LSD radix sort over a tile of 4096 arcs.  Values are staged into
+// shared memory with cp.async as soon as the tile is known (no registers held across the
+// ranking / look-back); keys stay in registers; digits are recomputed from the keys.
 template <bool W, bool FIRST>
-__global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ kin,
+__global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t* __restrict__ kin,
                                                   const typename ValT<W>::T* __restrict__ vin,
                                                   const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst,
                                                   const uint32_t* __restrict__ w, uint64_t m, uint64_t M, int shift,
@@ -87,8 +98,9 @@ __global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ k
                                                   uint32_t* __restrict__ kout, typename ValT<W>::T* __restrict__ vout) {
     typedef typename ValT<W>::T VT;
     extern __shared__ __align__(16) unsigned char smem[];
-    VT* s_val = reinterpret_cast<VT*>(smem);
-    uint32_t* s_key = reinterpret_cast<uint32_t*>(smem + sizeof(VT) * kTileItems);
+    VT* s_vin = reinterpret_cast<VT*>(smem);                                   // tile values, input order
+    VT* s_val = reinterpret_cast<VT*>(smem + sizeof(VT) * kTileItems);         // values, digit order
+    uint32_t* s_key = reinterpret_cast<uint32_t*>(smem + 2 * sizeof(VT) * kTileItems);
     __shared__ uint32_t s_wcnt[kSW][kMaxRadix + 1];
     __shared__ uint32_t s_dstart[kMaxRadix + 1];
     __shared__ uint64_t s_gofs[kMaxRadix];
@@ -103,41 +115,58 @@ __global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ k
     const uint64_t base = (uint64_t)tile * kTileItems;
     const int radix = 1 << bits;
     const uint32_t mask = (uint32_t)radix - 1;
+    const uint32_t cnt = (M - base < (uint64_t)kTileItems) ? (uint32_t)(M - base) : (uint32_t)kTileItems;
 
+    // values -> shared memory (asynchronous, coalesced), keys -> registers
     uint32_t key[kSI];
-    VT val[kSI];
-    uint32_t dig[kSI];
-    uint16_t rank[kSI];
 #pragma unroll
     for (int r = 0; r < kSI; ++r) {
-        const uint64_t idx = base + (uint64_t)wp * (kSI * 32) + r * 32 + lane;
+        const uint32_t li = wp * (kSI * 32) + r * 32 + lane;
+        const uint64_t idx = base + li;
         key[r] = 0;
-        val[r] = 0;
-        if (idx < M) {
-            if constexpr (FIRST) coo_item<W>(src, dst, w, m, idx, key[r], val[r]);
-            else { key[r] = kin[idx]; val[r] = vin[idx]; }
-            dig[r] = (key[r] >> shift) & mask;
-        } else {
-            dig[r] = (uint32_t)radix;  // dummy bin
+        if (li < cnt) {
+            if constexpr (FIRST) {
+                const bool rev = idx >= m;
+                const uint64_t f = rev ? idx - m : idx;
+                key[r] = rev ? dst[f] : src[f];
+                uint32_t* sv = reinterpret_cast<uint32_t*>(&s_vin[li]);
+                cp_async4(sv, rev ? src + f : dst + f);
+                if constexpr (W) cp_async4(sv + 1, w + f);
+            } else {
+                key[r] = kin[idx];
+                if constexpr (W) {
+                    const uint32_t* gv = reinterpret_cast<const uint32_t*>(vin + idx);
+                    uint32_t* sv = reinterpret_cast<uint32_t*>(&s_vin[li]);
+                    cp_async4(sv, gv);
+                    cp_async4(sv + 1, gv + 1);
+                } else {
+                    cp_async4(&s_vin[li], vin + idx);
+                }
+            }
         }
     }
+    asm volatile("cp.async.commit_group;" ::: "memory");
     // stable ranking within the warp's 512 items (item order = round-major, then lane): the
     // lowest lane of each digit group reserves popc(peers) slots with a shared atomic; the
     // warp issues the rounds' atomics in order, so reservations follow item order; the
     // results are broadcast after all rounds are issued (no per-round round trip).
     const uint32_t lt = (1u << lane) - 1;
     uint32_t peers[kSI];
+    uint32_t rank[kSI / 2];  // two 16-bit ranks per register
 #pragma unroll
     for (int r = 0; r < kSI; ++r) {
-        peers[r] = __match_any_sync(0xffffffffu, dig[r]);
+        const uint32_t li = wp * (kSI * 32) + r * 32 + lane;
+        const uint32_t d = li < cnt ? (key[r] >> shift) & mask : (uint32_t)radix;
+        peers[r] = __match_any_sync(0xffffffffu, d);
         uint32_t got = 0;
-        if ((peers[r] & lt) == 0) got = atomicAdd(&s_wcnt[wp][dig[r]], (uint32_t)__popc(peers[r]));
-        rank[r] = (uint16_t)got;
+        if ((peers[r] & lt) == 0) got = atomicAdd(&s_wcnt[wp][d], (uint32_t)__popc(peers[r]));
+        if (r & 1) rank[r >> 1] |= got << 16; else rank[r >> 1] = got;
     }
 #pragma unroll
     for (int r = 0; r < kSI; ++r) {
-        const uint32_t base = __shfl_sync(0xffffffffu, (uint32_t)rank[r], __ffs(peers[r]) - 1);
-        rank[r] = (uint16_t)(base + __popc(peers[r] & lt));
+        const uint32_t mine = (rank[r >> 1] >> ((r & 1) * 16)) & 0xFFFFu;
+        const uint32_t b = __shfl_sync(0xffffffffu, mine, __ffs(peers[r]) - 1) + __popc(peers[r] & lt);
+        rank[r >> 1] = (r & 1) ? ((rank[r >> 1] & 0xFFFFu) | (b << 16)) : ((rank[r >> 1] & 0xFFFF0000u) | b);
     }
     __syncthreads();
     // per digit: exclusive prefix over warps, tile count, publish the aggregate
@@ -184,18 +213,20 @@ __global__ void __launch_bounds__(kST) k_onesweep(const uint32_t* __restrict__ k
         }
         s_gofs[t] = digit_base[t] + excl;
     }
+    asm volatile("cp.async.wait_all;" ::: "memory");
     __syncthreads();
     // reorder the tile by digit in shared memory
 #pragma unroll
     for (int r = 0; r < kSI; ++r) {
-        if (dig[r] < (uint32_t)radix) {
-            const uint32_t lp = s_dstart[dig[r]] + s_wcnt[wp][dig[r]] + rank[r];
+        const uint32_t li = wp * (kSI * 32) + r * 32 + lane;
+        if (li < cnt) {
+            const uint32_t d = (key[r] >> shift) & mask;
+            const uint32_t lp = s_dstart[d] + s_wcnt[wp][d] + ((rank[r >> 1] >> ((r & 1) * 16)) & 0xFFFFu);
             s_key[lp] = key[r];
-            s_val[lp] = val[r];
+            s_val[lp] = s_vin[li];
         }
     }
     __syncthreads();
-    const uint64_t cnt = (M - base < (uint64_t)kTileItems) ? M - base : (uint64_t)kTileItems;
 #pragma unroll
     for (int r = 0; r < kSI; ++r) {
         const uint32_t i = r * kST + t;
@@ -281,7 +312,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     k_digit_base<<<1, kMaxRadix, 0, s>>>(hist.as<unsigned long long>(), passes, dbase.as<uint64_t>());
     TIGR_CKL("digit base");
     trace(s, "sort: digit histograms");
-    const size_t smem = (sizeof(VT) + sizeof(uint32_t)) * kTileItems;
+    const size_t smem = (2 * sizeof(VT) + sizeof(uint32_t)) * kTileItems;
     int cur = 0;
     for (int p = 0; p < passes && M; ++p) {
         auto kern = (p == 0) ? &k_onesweep<W, true> : &k_onesweep<W, false>;
