@@ -35,11 +35,16 @@ constexpr int kCidSlots = 8192;   // shared-memory accumulator entries (64 KB of
 __global__ void k_indeg_flag(const uint4* __restrict__ c4, uint64_t nchunks, uint8_t* __restrict__ flag) {
     for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
          k += (uint64_t)gridDim.x * blockDim.x) {
+        // test before setting: hot targets would otherwise serialise millions of stores on one
+        // L2 sector; a (possibly stale) read of 1 skips the store, a stale 0 only repeats it
         const uint4 c = ldg_chunk(c4 + k);
-        if (c.x != kPad) flag[c.x] = 1;
-        if (c.y != kPad) flag[c.y] = 1;
-        if (c.z != kPad) flag[c.z] = 1;
-        if (c.w != kPad) flag[c.w] = 1;
+        const uint32_t t4[4] = {c.x, c.y, c.z, c.w};
+        uint8_t f[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) f[q] = t4[q] != kPad ? flag[t4[q]] : 1;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if (!f[q]) flag[t4[q]] = 1;
     }
 }
 
@@ -213,6 +218,7 @@ tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
     TIGR_CK(cudaMemsetAsync(flag.p, 0, n, s));
     TIGR_CK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * n, s));
     TIGR_CK(cudaMemsetAsync(nin.p, 0, sizeof(uint32_t), s));
+    trace(s, "pr cid: alloc");
     const uint4* c4 = g->col.as<uint4>();
     if (g->nchunks) {
         k_indeg_flag<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, flag.as<uint8_t>());
@@ -220,6 +226,7 @@ tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
         k_hot_sample<<<grid_cap(g->nchunks / 16 + 1, 16), kBlock, 0, s>>>(c4, g->nchunks, cnt.as<uint32_t>());
         TIGR_CKL("pr sample");
     }
+    trace(s, "pr cid: flags+sample");
     k_pr_key<<<grid_for(n), kBlock, 0, s>>>(flag.as<uint8_t>(), cnt.as<uint32_t>(), n, key.as<uint32_t>(),
                                              ids.as<uint32_t>(), nin.as<uint32_t>());
     TIGR_CKL("pr key");
@@ -227,11 +234,13 @@ tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
     TIGR_TRY(sort_pairs_u32(key.as<uint32_t>(), ids.as<uint32_t>(), n, 34, s, skeys, order));
     k_cid_scatter<<<grid_for(n), kBlock, 0, s>>>(order.as<uint32_t>(), n, ws.cid.as<uint32_t>());
     TIGR_CKL("pr cid");
+    trace(s, "pr cid: key+sort+scatter");
     if (g->nchunks) {
         k_build_col_pr<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, ws.cid.as<uint32_t>(),
                                                                     ws.col_pr.as<uint4>());
         TIGR_CKL("pr col_pr");
     }
+    trace(s, "pr cid: col_pr");
     uint32_t h = 0;
     TIGR_CK(cudaMemcpyAsync(&h, nin.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
     TIGR_CK(cudaStreamSynchronize(s));

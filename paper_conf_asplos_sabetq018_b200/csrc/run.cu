@@ -25,7 +25,6 @@ Workspace::~Workspace() {
     for (auto& e : ev)
         if (e) cudaEventDestroy(e);
     for (auto& e : tev) cudaEventDestroy(e);
-    if (ctl_host) cudaFreeHost(ctl_host);
 }
 
 namespace {
@@ -35,7 +34,11 @@ tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
     const size_t n = vg->g->n ? vg->g->n : 1;
     if (!ws.ctl.p) {
         TIGR_TRY(ws.ctl.alloc(sizeof(Ctl), s));
-        TIGR_CK(cudaMallocHost(&ws.ctl_host, sizeof(Ctl)));
+        // pinned control-block mirror: one per host thread for the process lifetime (a
+        // cudaMallocHost per vgraph would synchronise the device on every graph rebuild)
+        static thread_local Ctl* t_ctl = nullptr;
+        if (!t_ctl) TIGR_CK(cudaMallocHost(&t_ctl, sizeof(Ctl)));
+        ws.ctl_host = t_ctl;
         for (auto& e : ws.ev) TIGR_CK(cudaEventCreate(&e));
     }
     if (pr) {
@@ -267,6 +270,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     k_pr_init<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), ws.x.as<double>(), ws.contrib.as<double>(),
                                              ws.acc.as<double>(), a.ctl);
     TIGR_CKL("pr init");
+    trace(s, "pr: prepare+init");
     double ms_relax = 0.0, ms_ex = 0.0;
     uint32_t launches = 0;
     if (o.time_kernels) {  // 3 events per iteration: relax start / relax end / exchange end
@@ -307,6 +311,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         TIGR_CKL("pr apply");
     }
     TIGR_CK(cudaEventRecord(t1, s));
+    trace(s, "pr: 20 iterations");
     TIGR_CK(cudaMemcpyAsync(ws.ctl_host, a.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     TIGR_CK(cudaStreamSynchronize(s));
     if (o.time_kernels) {

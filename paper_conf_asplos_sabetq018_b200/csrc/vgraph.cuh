@@ -50,7 +50,7 @@ struct Workspace {
     uint32_t n_in = 0;       // nodes with in-arcs (= accumulator entries ever written)
     bool cid_ready = false;
     DevBuf ctl;      // Ctl
-    Ctl* ctl_host = nullptr;  // pinned mirror for the host loop
+    Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (thread-local, not owned)
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> tev;  // per-relax-launch timing events (time_kernels)
     std::map<GraphKey, CachedGraph> graphs;
