@@ -20,17 +20,6 @@ tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const 
 
 namespace {
 
-__global__ void k_maxid(const uint32_t* __restrict__ a, const uint32_t* __restrict__ b, uint64_t m,
-                        uint32_t* out) {
-    uint32_t mx = 0;
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < m;
-         i += (uint64_t)gridDim.x * blockDim.x)
-        mx = max(mx, max(a[i], b[i]));
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
-    if ((threadIdx.x & 31) == 0 && mx) atomicMax(out, mx);
-}
-
 __global__ void k_pad(const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cptr, uint32_t n,
                       uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
@@ -123,18 +112,6 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
                                   const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out) {
     const uint64_t arcs = symmetrize ? 2 * m : m;
     if (arcs >= (1ull << 32) * 3) return fail(TIGR_ERANGE, "graph: too many arcs");
-    if (m) {
-        TmpBuf mx;
-        TIGR_TRY(mx.alloc(sizeof(uint32_t), s));
-        TIGR_CK(cudaMemsetAsync(mx.p, 0, sizeof(uint32_t), s));
-        k_maxid<<<capped_grid(m), kBlock, 0, s>>>(src, dst, m, mx.as<uint32_t>());
-        TIGR_CKL("maxid");
-        uint32_t hmax = 0;
-        TIGR_CK(cudaMemcpyAsync(&hmax, mx.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
-        TIGR_CK(cudaStreamSynchronize(s));
-        if (hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
-        trace(s, "coo: validate ids");
-    }
     tigr_graph* g = new tigr_graph();
     g->n = n;
     g->m = arcs;

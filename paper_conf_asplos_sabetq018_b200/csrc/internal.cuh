@@ -102,6 +102,10 @@ struct tigr_graph {
     tigr::DevBuf cptr;       // uint32[n+1], first chunk of each node's segment
     tigr::DevBuf col;        // uint32[4 * nchunks], padded segments, pads = 0xFFFFFFFF
     tigr::DevBuf wt;         // uint32[4 * nchunks] or empty
+    // in-degree sketch from the arc-list scan (PageRank accumulator order, pr.cu)
+    tigr::DevBuf in_flag;    // uint8[n]: node has an in-arc
+    tigr::DevBuf in_sample;  // uint32[n]: in-arcs among every 16th arc
+    bool has_in_sketch = false;
 };
 
 struct tigr_comm {

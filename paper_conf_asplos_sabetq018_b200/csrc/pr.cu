@@ -209,25 +209,30 @@ tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
     const uint32_t n = g->n;
     TIGR_TRY(ws.cid.alloc(sizeof(uint32_t) * (n ? n : 1), s));
     TIGR_TRY(ws.col_pr.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
-    TmpBuf flag, cnt, key, ids, nin;
-    TIGR_TRY(flag.alloc(n ? n : 1, s));
-    TIGR_TRY(cnt.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TmpBuf flag_t, cnt_t, key, ids, nin;
     TIGR_TRY(key.alloc(sizeof(uint32_t) * (n ? n : 1), s));
     TIGR_TRY(ids.alloc(sizeof(uint32_t) * (n ? n : 1), s));
     TIGR_TRY(nin.alloc(sizeof(uint32_t), s));
-    TIGR_CK(cudaMemsetAsync(flag.p, 0, n, s));
-    TIGR_CK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * n, s));
     TIGR_CK(cudaMemsetAsync(nin.p, 0, sizeof(uint32_t), s));
-    trace(s, "pr cid: alloc");
     const uint4* c4 = g->col.as<uint4>();
-    if (g->nchunks) {
-        k_indeg_flag<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, flag.as<uint8_t>());
-        TIGR_CKL("pr indeg flag");
-        k_hot_sample<<<grid_cap(g->nchunks / 16 + 1, 16), kBlock, 0, s>>>(c4, g->nchunks, cnt.as<uint32_t>());
-        TIGR_CKL("pr sample");
+    const uint8_t* flag = g->in_flag.as<uint8_t>();
+    const uint32_t* cnt = g->in_sample.as<uint32_t>();
+    if (!g->has_in_sketch) {  // graph built from a CSR: sketch the in-degrees from the arc array
+        TIGR_TRY(flag_t.alloc(n ? n : 1, s));
+        TIGR_TRY(cnt_t.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+        TIGR_CK(cudaMemsetAsync(flag_t.p, 0, n, s));
+        TIGR_CK(cudaMemsetAsync(cnt_t.p, 0, sizeof(uint32_t) * n, s));
+        if (g->nchunks) {
+            k_indeg_flag<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, flag_t.as<uint8_t>());
+            TIGR_CKL("pr indeg flag");
+            k_hot_sample<<<grid_cap(g->nchunks / 16 + 1, 16), kBlock, 0, s>>>(c4, g->nchunks, cnt_t.as<uint32_t>());
+            TIGR_CKL("pr sample");
+        }
+        flag = flag_t.as<uint8_t>();
+        cnt = cnt_t.as<uint32_t>();
     }
-    trace(s, "pr cid: flags+sample");
-    k_pr_key<<<grid_for(n), kBlock, 0, s>>>(flag.as<uint8_t>(), cnt.as<uint32_t>(), n, key.as<uint32_t>(),
+    trace(s, "pr cid: sketch");
+    k_pr_key<<<grid_for(n), kBlock, 0, s>>>(flag, cnt, n, key.as<uint32_t>(),
                                              ids.as<uint32_t>(), nin.as<uint32_t>());
     TIGR_CKL("pr key");
     TmpBuf skeys, order;

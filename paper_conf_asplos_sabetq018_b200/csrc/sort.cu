@@ -45,18 +45,36 @@ __device__ __forceinline__ void coo_item(const uint32_t* __restrict__ src, const
     else v = t;
 }
 
-// digit histograms of every pass in one read of the keys
-template <bool FIRST>
-__global__ void k_digit_hist(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
-                             uint64_t M, int passes, int bits, unsigned long long* __restrict__ hist) {
+// One read of the arc list before sorting: the digit histograms of every pass, the largest id
+// (validation: checked on the host before any id is used as an index), and optionally the
+// in-degree sketch the PageRank accumulator order uses (pr.cu): a has-in-arcs flag per node
+// (tested before set, so hub targets do not serialise stores) and an in-degree count sampled
+// on every 16th arc.  Arc e of the (optionally symmetrised) list: key = source, t = target.
+__global__ void k_coo_scan(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
+                           uint64_t M, int passes, int bits, unsigned long long* __restrict__ hist,
+                           uint32_t* __restrict__ maxid, uint32_t n, uint8_t* __restrict__ in_flag,
+                           uint32_t* __restrict__ in_sample) {
     __shared__ uint32_t h[4][kMaxRadix];
     for (int i = threadIdx.x; i < 4 * kMaxRadix; i += blockDim.x) (&h[0][0])[i] = 0;
     __syncthreads();
     const uint32_t mask = (1u << bits) - 1;
+    uint32_t mx = 0;
     for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < M; e += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t k = e < m ? src[e] : dst[e - m];
-        for (int p = 0; p < passes; ++p) atomicAdd(&h[p][(k >> (p * bits)) & mask], 1u);
+        const bool rev = e >= m;
+        const uint64_t f = rev ? e - m : e;
+        const uint32_t s = src[f], d = dst[f];
+        const uint32_t k = rev ? d : s, t = rev ? s : d;
+        mx = max(mx, max(s, d));
+        if (k < n)
+            for (int p = 0; p < passes; ++p) atomicAdd(&h[p][(k >> (p * bits)) & mask], 1u);
+        if (in_flag && t < n) {
+            if (!in_flag[t]) in_flag[t] = 1;
+            if ((e & 15) == 0) atomicAdd(in_sample + t, 1u);
+        }
     }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    if ((threadIdx.x & 31) == 0 && mx) atomicMax(maxid, mx);
     __syncthreads();
     for (int i = threadIdx.x; i < passes * kMaxRadix; i += blockDim.x) {
         const uint32_t c = (&h[0][0])[i];
@@ -281,7 +299,8 @@ unsigned sort_grid(uint64_t items) {
 
 template <bool W>
 tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* w, uint64_t m, uint64_t M,
-                      uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out) {
+                      uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out, bool validate,
+                      uint8_t* in_flag = nullptr, uint32_t* in_sample = nullptr) {
     typedef typename ValT<W>::T VT;
     int key_bits = 0;
     while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
@@ -289,7 +308,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     const int bits = key_bits == 0 ? 1 : (key_bits + passes - 1) / passes;
     const uint64_t tiles = (M + kTileItems - 1) / kTileItems;
 
-    TmpBuf kb[2], vb[2], hist, dbase, status, counters;
+    TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid;
     trace(s, "sort: enter");
     for (int i = 0; i < 2; ++i) {
         TIGR_TRY(kb[i].alloc(sizeof(uint32_t) * (M ? M : 1), s));
@@ -303,11 +322,19 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     TIGR_CK(cudaMemsetAsync(hist.p, 0, sizeof(unsigned long long) * 4 * kMaxRadix, s));
     TIGR_CK(cudaMemsetAsync(status.p, 0, sizeof(uint64_t) * kMaxRadix * (tiles ? tiles : 1), s));
     TIGR_CK(cudaMemsetAsync(counters.p, 0, sizeof(uint32_t) * 4, s));
+    TIGR_TRY(maxid.alloc(sizeof(uint32_t), s));
+    TIGR_CK(cudaMemsetAsync(maxid.p, 0, sizeof(uint32_t), s));
     trace(s, "sort: alloc+memset");
     if (M) {
-        k_digit_hist<true><<<sort_grid(M), kBlock, 0, s>>>(src, dst, m, M, passes, bits,
-                                                            hist.as<unsigned long long>());
-        TIGR_CKL("digit hist");
+        k_coo_scan<<<sort_grid(M), kBlock, 0, s>>>(src, dst, m, M, passes, bits, hist.as<unsigned long long>(),
+                                                    maxid.as<uint32_t>(), n, in_flag, in_sample);
+        TIGR_CKL("coo scan");
+    }
+    if (M && validate) {
+        uint32_t hmax = 0;
+        TIGR_CK(cudaMemcpyAsync(&hmax, maxid.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        TIGR_CK(cudaStreamSynchronize(s));
+        if (hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
     }
     k_digit_base<<<1, kMaxRadix, 0, s>>>(hist.as<unsigned long long>(), passes, dbase.as<uint64_t>());
     TIGR_CKL("digit base");
@@ -340,7 +367,13 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     const uint64_t M = symmetrize ? 2 * m : m;
     TmpBuf keys, vals;
     keys.s = vals.s = s;
-    TIGR_TRY(sort_arcs<W>(src, dst, w, m, M, n, s, keys, vals));
+    TIGR_TRY(g->in_flag.alloc(n ? n : 1, s));
+    TIGR_TRY(g->in_sample.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_CK(cudaMemsetAsync(g->in_flag.p, 0, n, s));
+    TIGR_CK(cudaMemsetAsync(g->in_sample.p, 0, sizeof(uint32_t) * n, s));
+    TIGR_TRY(sort_arcs<W>(src, dst, w, m, M, n, s, keys, vals, true, g->in_flag.as<uint8_t>(),
+                          g->in_sample.as<uint32_t>()));
+    g->has_in_sketch = true;
     // degrees from runs
     TmpBuf st, en;
     TIGR_TRY(st.alloc(sizeof(uint32_t) * n, s));
@@ -382,7 +415,7 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
 tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t count, uint32_t key_limit,
                            cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out) {
     keys_out.s = vals_out.s = s;
-    return sort_arcs<false>(keys, vals, nullptr, count, count, key_limit, s, keys_out, vals_out);
+    return sort_arcs<false>(keys, vals, nullptr, count, count, key_limit, s, keys_out, vals_out, false);
 }
 
 // Stable device CSR build from an arc list (device pointers).  Caller validated ids < n.
