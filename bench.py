@@ -272,7 +272,7 @@ def main():
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": config_obj(args, rec),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": traffic, "kernel": "k_relax_pr (PageRank push relax)",
+                     "traffic": traffic, "kernel": "k_relax_pr_cid (PageRank push relax, pr.cu)",
                      "algorithmic_bytes_per_launch": bytes_launch, "avg_launch_ms": relax_avg_ms,
                      "peak_source": peak_src},
         "breakdown_ms": {"csr_build": statistics.mean(phase[0]), "virtualize": statistics.mean(phase[1]),
