@@ -30,7 +30,6 @@ __global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uin
 
 namespace {
 
-constexpr int kCidSlots = 8192;   // shared-memory accumulator entries (64 KB of f64)
 
 __global__ void k_indeg_flag(const uint4* __restrict__ c4, uint64_t nchunks, uint8_t* __restrict__ flag) {
     for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
@@ -82,25 +81,25 @@ __global__ void k_build_col_pr(const uint4* __restrict__ c4, uint64_t nchunks, c
     }
 }
 
-template <int LAYOUT, int B>
-__global__ void __launch_bounds__(kRelaxThreads, 2) k_relax_pr_cid(RelaxArgs a, const uint32_t* __restrict__ col_pr,
+template <int LAYOUT, int B, int T, int SLOTS, int MINB>
+__global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uint32_t* __restrict__ col_pr,
                                                                    uint32_t tiles) {
-    extern __shared__ __align__(16) double s_acc[];  // kCidSlots entries (dynamic: 64 KB)
+    extern __shared__ __align__(16) double s_acc[];  // SLOTS entries (dynamic: 64 KB)
     const int t = threadIdx.x;
-    for (int i = t; i < kCidSlots; i += kRelaxThreads) s_acc[i] = 0.0;
+    for (int i = t; i < SLOTS; i += T) s_acc[i] = 0.0;
     __syncthreads();
     const uint64_t pol = policy_evict_last();
     const uint4* c4 = reinterpret_cast<const uint4*>(col_pr);
     auto push = [&](uint32_t c, double x) {
-        if (c < (uint32_t)kCidSlots) atomicAdd(&s_acc[c], x);
+        if (c < (uint32_t)SLOTS) atomicAdd(&s_acc[c], x);
         else red_add_f64(a.acc + c, x, pol);
     };
     for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-        const uint64_t base = (uint64_t)a.lo + (uint64_t)tile * (B * kRelaxThreads) + t;
+        const uint64_t base = (uint64_t)a.lo + (uint64_t)tile * (B * T) + t;
         uint32_t v[B];
 #pragma unroll
         for (int r = 0; r < B; ++r) {
-            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+            const uint64_t i = base + (uint64_t)r * T;
             v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
         }
         uint4 info[B];
@@ -115,7 +114,7 @@ __global__ void __launch_bounds__(kRelaxThreads, 2) k_relax_pr_cid(RelaxArgs a, 
         uint32_t kn[B], kend[B], step[B];
 #pragma unroll
         for (int r = 0; r < B; ++r) {
-            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
+            const uint64_t i = base + (uint64_t)r * T;
             const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
             uint32_t k;
             if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
@@ -150,7 +149,7 @@ __global__ void __launch_bounds__(kRelaxThreads, 2) k_relax_pr_cid(RelaxArgs a, 
         }
     }
     __syncthreads();
-    for (int i = t; i < kCidSlots; i += kRelaxThreads)
+    for (int i = t; i < SLOTS; i += T)
         if (s_acc[i] != 0.0) red_add_f64(a.acc + i, s_acc[i], pol);
 }
 
@@ -254,18 +253,35 @@ tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
     return TIGR_OK;
 }
 
+template <int B, int T, int SLOTS, int MINB>
+static void fill_plan(PrCidPlan& p, int layout) {
+    p.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, B, T, SLOTS, MINB>
+                                         : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, B, T, SLOTS, MINB>;
+    p.threads = T;
+    p.per_thread = B;
+    p.smem = sizeof(double) * SLOTS;
+}
+
+// Kernel shape: one 768-thread block per SM (24 warps), 24576 hot slots (192 KB of shared
+// memory: one table per SM instead of two 8192-slot copies), 4 virtual nodes per thread.
+// Measured at cfg4 (relax ms/launch): 256x2 blocks, 8192 slots 1.53; 512x1, 24576 1.15;
+// 768x1, 24576 1.12; 768x1, 28672 1.21; 1024x1 (spills) 1.16.  TIGR_PR_CFG selects the
+// alternatives for experiments.
 PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
     PrCidPlan p;
-    const int B = 4;
-    p.fn = vg->layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, B>
-                                             : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, B>;
-    p.smem = sizeof(double) * kCidSlots;
+    const char* e = getenv("TIGR_PR_CFG");
+    switch (e ? atoi(e) : 5) {
+        case 0: fill_plan<4, 256, 8192, 2>(p, vg->layout); break;
+        case 1: fill_plan<4, 512, 24576, 1>(p, vg->layout); break;
+        case 6: fill_plan<4, 768, 28672, 1>(p, vg->layout); break;
+        default: fill_plan<4, 768, 24576, 1>(p, vg->layout); break;
+    }
     cudaFuncSetAttribute(p.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
     int per_sm = 0, dev = 0, sms = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, p.fn, kRelaxThreads, p.smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, p.fn, p.threads, p.smem);
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const uint64_t per_tile = (uint64_t)kRelaxThreads * B;
+    const uint64_t per_tile = (uint64_t)p.threads * p.per_thread;
     p.tiles = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_tile - 1) / per_tile);
     p.grid = (unsigned)std::min<uint64_t>(p.tiles, (uint64_t)sms * (per_sm > 0 ? per_sm : 1));
     return p;

@@ -44,6 +44,7 @@ PrHotConfig relax_pr_hot_config(int layout, bool vec);
 struct PrCidPlan {
     void (*fn)(RelaxArgs, const uint32_t*, uint32_t) = nullptr;
     unsigned grid = 0, tiles = 0;
+    int threads = 256, per_thread = 4;
     size_t smem = 0;
 };
 bool pr_cid_enabled();

@@ -283,7 +283,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     for (uint32_t t = 0; t < o.pr_iters; ++t) {
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t], s));
         if (use_cid && cp.tiles) {
-            cp.fn<<<cp.grid, kRelaxThreads, cp.smem, s>>>(a, ws.col_pr.as<uint32_t>(), cp.tiles);
+            cp.fn<<<cp.grid, cp.threads, cp.smem, s>>>(a, ws.col_pr.as<uint32_t>(), cp.tiles);
             TIGR_CKL("pr relax (cid)");
             ++launches;
         } else if (hot && hot_tiles) {
