@@ -296,7 +296,8 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
             ++launches;
         }
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t + 1], s));
-        if (comm) TIGR_TRY(comm_allreduce(o.comm, ws.acc.p, n, TIGR_PR, s));
+        // in accumulator-id order only the first n_in entries are ever written (pr.cu)
+        if (comm) TIGR_TRY(comm_allreduce(o.comm, ws.acc.p, use_cid ? ws.n_in : n, TIGR_PR, s));
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t + 2], s));
         double* dcur = &a.ctl->dsum[t & 1];
         double* dnext = &a.ctl->dsum[(t + 1) & 1];
