@@ -209,7 +209,8 @@ def main():
         ev[2].record(s)
         _, st = tigr.tigr_run(vg, "pr", 0, opts=opts, out=out_t, return_stats=True)
         ev[3].record(s)
-        nv = vg.info()["nv"]
+        vi = vg.info()
+        nv = vi["hi"] - vi["lo"]  # this rank's virtual nodes (all of them at N = 1)
         vg.free()
         g.free()
         return ev, st, nv

@@ -406,18 +406,44 @@ void partition_ranges(uint32_t n, const int64_t* rp, const uint32_t* vp, int nra
     }
 }
 
+// the same rule on the device: one thread per cut, binary search over row_ptr (no D2H of the
+// node arrays; only the 2 range bounds come back)
+__global__ void k_partition(const int64_t* __restrict__ rp, const uint32_t* __restrict__ vp, uint32_t n,
+                            int nranks, int rank, uint32_t* out) {
+    const int c = threadIdx.x;  // 0: cut(rank), 1: cut(rank + 1)
+    if (c > 1) return;
+    const int r = rank + c;
+    uint32_t cut;
+    if (r <= 0) cut = 0;
+    else if (r >= nranks) cut = n;
+    else {
+        const uint64_t m = (uint64_t)rp[n];
+        const int64_t target = (int64_t)((unsigned __int128)m * (unsigned)r / (unsigned)nranks);
+        uint32_t lo = 0, hi = n;  // first index in [0, n) with rp[idx] >= target (lower_bound)
+        while (lo < hi) {
+            const uint32_t mid = lo + (hi - lo) / 2;
+            if (rp[mid] < target) lo = mid + 1; else hi = mid;
+        }
+        cut = lo;
+    }
+    out[c] = vp[cut];
+}
+
 tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank) {
     if (nranks < 1 || rank < 0 || rank >= nranks) return fail(TIGR_EINVAL, "partition: bad rank/nranks");
     const tigr_graph* g = vg->g;
     if (nranks == 1 || g->n == 0) { vg->lo = 0; vg->hi = (uint32_t)vg->nv; return TIGR_OK; }
-    std::vector<int64_t> rp((size_t)g->n + 1);
-    std::vector<uint32_t> vp((size_t)g->n + 1);
-    TIGR_CK(cudaMemcpy(rp.data(), g->row_ptr.p, sizeof(int64_t) * rp.size(), cudaMemcpyDeviceToHost));
-    TIGR_CK(cudaMemcpy(vp.data(), vg->vnode_ptr.p, sizeof(uint32_t) * vp.size(), cudaMemcpyDeviceToHost));
-    std::vector<uint32_t> lo(nranks), hi(nranks);
-    partition_ranges(g->n, rp.data(), vp.data(), nranks, lo.data(), hi.data());
-    vg->lo = lo[rank];
-    vg->hi = hi[rank];
+    cudaStream_t s = vg->vnode_ptr.s;
+    TmpBuf out;
+    TIGR_TRY(out.alloc(2 * sizeof(uint32_t), s));
+    k_partition<<<1, 32, 0, s>>>(g->row_ptr.as<int64_t>(), vg->vnode_ptr.as<uint32_t>(), g->n, nranks, rank,
+                                 out.as<uint32_t>());
+    TIGR_CKL("partition");
+    uint32_t h[2] = {0, 0};
+    TIGR_CK(cudaMemcpyAsync(h, out.p, sizeof(h), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    vg->lo = h[0];
+    vg->hi = h[1];
     return TIGR_OK;
 }
 

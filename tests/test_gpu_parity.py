@@ -304,6 +304,9 @@ def test_partition_ranges(tigr):
             assert i["lo"] in set(vp.tolist()) and i["hi"] in set(vp.tolist())  # family-aligned
         assert bounds[0][0] == 0 and bounds[-1][1] == nv
         assert all(bounds[r][1] == bounds[r + 1][0] for r in range(P - 1))
+        rp, _, _ = tigr.tigr_graph_export_csr(g)
+        lo, hi = tigr.tigr_partition_ranges(rp, vp, P)  # host rule == device rule
+        assert [tuple(x) for x in zip(lo.tolist(), hi.tolist())] == bounds
     tigr.tigr_vgraph_partition(vg, 1, 0)
     assert vg.info()["hi"] == nv
 
