@@ -139,7 +139,14 @@ tigr_status tigr_graph_rmat(uint32_t n, uint64_t m, double a, double b, double c
 
 /* Sizes and flags of a graph (any pointer may be NULL). */
 tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* weighted,
-                            int* symmetric, uint64_t* device_bytes);
+                            int* symmetric, int* transposed, uint64_t* device_bytes);
+
+/* In-CSR (transpose) of g on the device: every arc u->v of g becomes v->u, grouped by v and
+ * stable in g's arc order; weights follow their arcs.  The result remembers g's out-degrees,
+ * so TIGR_PR run on a virtual split of it is PULL-based PageRank (
+ * Thm. 3: pull needs an associative combine + atomics across a family).
+ * Errors: ENOMEM, ECUDA. */
+tigr_status tigr_graph_transpose(const tigr_graph* g, void* stream, tigr_graph** out);
 
 /* Copy the CSR out (row_ptr[n+1], col[m], w[m] if weighted and w != NULL), arcs of a
  * source contiguous in the graph's internal order. */

@@ -67,7 +67,8 @@ _SIGS = {
     "tigr_rmat_coo": (_I, [_U32, _U64, _D, _D, _D, _U64, _U64, _U32, _U32, _P, _P, _P, _P]),
     "tigr_graph_rmat": (_I, [_U32, _U64, _D, _D, _D, _U64, _U64, _U32, _U32, _I, _I, _P, ctypes.POINTER(_P)]),
     "tigr_graph_info": (_I, [_P, ctypes.POINTER(_U32), ctypes.POINTER(_U64), ctypes.POINTER(_I),
-                             ctypes.POINTER(_I), ctypes.POINTER(_U64)]),
+                             ctypes.POINTER(_I), ctypes.POINTER(_I), ctypes.POINTER(_U64)]),
+    "tigr_graph_transpose": (_I, [_P, _P, ctypes.POINTER(_P)]),
     "tigr_graph_export_csr": (_I, [_P, _P, _P, _P, _I, _P]),
     "tigr_graph_free": (None, [_P]),
     "tigr_virtualize": (_I, [_P, _U32, _I, _P, ctypes.POINTER(_P)]),
@@ -137,10 +138,10 @@ class Graph:
         return self._ptr
 
     def info(self):
-        n, m, wt, sym, b = _U32(), _U64(), _I(), _I(), _U64()
-        _check(_lib.tigr_graph_info(self._ptr, n, m, wt, sym, b))
+        n, m, wt, sym, tr, b = _U32(), _U64(), _I(), _I(), _I(), _U64()
+        _check(_lib.tigr_graph_info(self._ptr, n, m, wt, sym, tr, b))
         return {"n": n.value, "m": m.value, "weighted": bool(wt.value), "symmetric": bool(sym.value),
-                "device_bytes": b.value}
+                "transposed": bool(tr.value), "device_bytes": b.value}
 
     def free(self):
         if self._ptr:
@@ -250,6 +251,13 @@ def tigr_graph_rmat(n, m, a, b, c, seed, wseed=0, wmin=1, wmax=64, weighted=True
     out = _P()
     _check(_lib.tigr_graph_rmat(n, m, a, b, c, seed, wseed, wmin, wmax, int(weighted), int(symmetrize),
                                 _stream_ptr(stream), ctypes.byref(out)))
+    return Graph(out.value)
+
+
+def tigr_graph_transpose(g: Graph, stream=None) -> Graph:
+    """In-CSR of g (arcs reversed; carries g's out-degrees: TIGR_PR on it is pull-based)."""
+    out = _P()
+    _check(_lib.tigr_graph_transpose(g.ptr, _stream_ptr(stream), ctypes.byref(out)))
     return Graph(out.value)
 
 

@@ -160,6 +160,7 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
 tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col, const uint32_t* w,
                                   int symmetric_hint, cudaStream_t s, tigr_graph** out);
 tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w, cudaStream_t s);
+tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out);
 tigr_status graph_rmat_device(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed, uint64_t wseed,
                               uint32_t wmin, uint32_t wmax, int weighted, int symmetrize, cudaStream_t s,
                               tigr_graph** out);
@@ -274,12 +275,13 @@ tigr_status tigr_graph_rmat(uint32_t n, uint64_t m, double a, double b, double c
 }
 
 tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* weighted, int* symmetric,
-                            uint64_t* device_bytes) {
+                            int* transposed, uint64_t* device_bytes) {
     if (!g) return fail(TIGR_EINVAL, "graph_info: NULL graph");
     if (n) *n = g->n;
     if (m) *m = g->m;
     if (weighted) *weighted = g->weighted;
     if (symmetric) *symmetric = g->symmetric;
+    if (transposed) *transposed = g->transposed;
     if (device_bytes) *device_bytes = g->row_ptr.bytes + g->deg.bytes + g->cptr.bytes + g->col.bytes + g->wt.bytes;
     return TIGR_OK;
 }
@@ -306,6 +308,15 @@ tigr_status tigr_graph_export_csr(const tigr_graph* g, int64_t* row_ptr, uint32_
 }
 
 void tigr_graph_free(tigr_graph* g) { delete g; }
+
+tigr_status tigr_graph_transpose(const tigr_graph* g, void* stream, tigr_graph** out) {
+    if (!g || !out) return fail(TIGR_EINVAL, "graph_transpose: NULL argument");
+    *out = nullptr;
+    cudaStream_t s = (cudaStream_t)stream;
+    TIGR_TRY(graph_transpose_device(g, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
 
 tigr_status tigr_virtualize(const tigr_graph* g, uint32_t K, tigr_layout layout, void* stream, tigr_vgraph** out) {
     if (!g || !out) return fail(TIGR_EINVAL, "virtualize: NULL argument");

@@ -81,6 +81,39 @@ __global__ void k_padded_to_csr(const int64_t* __restrict__ rp, uint32_t n, uint
     }
 }
 
+// canonical arc list (src, dst, w) of a device CSR: thread per node for short segments, a
+// whole warp per long one (ballot loop), so every write is coalesced
+__global__ void k_expand_arcs(const int64_t* __restrict__ rp, const uint32_t* __restrict__ cptr, uint32_t n,
+                              const uint32_t* __restrict__ col, const uint32_t* __restrict__ wt,
+                              uint32_t* __restrict__ src, uint32_t* __restrict__ dst, uint32_t* __restrict__ w) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    uint64_t beg = 0, cb = 0;
+    uint32_t d = 0;
+    if (v < n) { beg = (uint64_t)rp[v]; d = (uint32_t)(rp[v + 1] - rp[v]); cb = (uint64_t)cptr[v] * kChunk; }
+    const bool big = d > 32;
+    if (!big)
+        for (uint32_t p = 0; p < d; ++p) {
+            src[beg + p] = v;
+            dst[beg + p] = col[cb + p];
+            if (w) w[beg + p] = wt[cb + p];
+        }
+    uint32_t mask = __ballot_sync(0xffffffffu, big);
+    while (mask) {
+        const int l = __ffs(mask) - 1;
+        mask &= mask - 1;
+        const uint64_t b = __shfl_sync(0xffffffffu, beg, l);
+        const uint64_t c = __shfl_sync(0xffffffffu, cb, l);
+        const uint32_t dd = __shfl_sync(0xffffffffu, d, l);
+        const uint32_t vv = __shfl_sync(0xffffffffu, v, l);
+        for (uint32_t p = lane; p < dd; p += 32) {
+            src[b + p] = vv;
+            dst[b + p] = col[c + p];
+            if (w) w[b + p] = wt[c + p];
+        }
+    }
+}
+
 unsigned capped_grid(uint64_t items) {
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
@@ -179,6 +212,33 @@ tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* 
             g->wt.as<uint32_t>(), col, g->weighted ? w : nullptr);
         TIGR_CKL("export csr");
     }
+    return TIGR_OK;
+}
+
+// in-CSR of g: arcs reversed, grouped by target, stable in g's (canonical) arc order; carries
+// g's out-degrees (src_deg) for pull-based PageRank
+tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out) {
+    const uint64_t m = g->m;
+    TmpBuf src, dst, w;
+    TIGR_TRY(src.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    TIGR_TRY(dst.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    if (g->weighted) TIGR_TRY(w.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    k_expand_arcs<<<grid_for(g->n), kBlock, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), g->n,
+                                                    g->col.as<uint32_t>(), g->wt.as<uint32_t>(), src.as<uint32_t>(),
+                                                    dst.as<uint32_t>(), g->weighted ? w.as<uint32_t>() : nullptr);
+    TIGR_CKL("expand arcs");
+    tigr_graph* t = nullptr;
+    TIGR_TRY(graph_from_coo_device(g->n, m, dst.as<uint32_t>(), src.as<uint32_t>(),
+                                   g->weighted ? w.as<uint32_t>() : nullptr, 0, s, &t));
+    t->symmetric = g->symmetric;
+    t->transposed = !g->transposed;
+    tigr_status st = t->src_deg.alloc(sizeof(uint32_t) * (g->n ? g->n : 1), s);
+    if (st == TIGR_OK && g->n) {
+        cudaError_t e = cudaMemcpyAsync(t->src_deg.p, g->deg.p, sizeof(uint32_t) * g->n, cudaMemcpyDeviceToDevice, s);
+        if (e != cudaSuccess) st = cuda_fail(e, "transpose src_deg", __FILE__, __LINE__);
+    }
+    if (st != TIGR_OK) { delete t; return st; }
+    *out = t;
     return TIGR_OK;
 }
 

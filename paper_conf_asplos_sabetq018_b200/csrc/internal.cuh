@@ -106,6 +106,10 @@ struct tigr_graph {
     tigr::DevBuf in_flag;    // uint8[n]: node has an in-arc
     tigr::DevBuf in_sample;  // uint32[n]: in-arcs among every 16th arc
     bool has_in_sketch = false;
+    // transposed graphs (tigr_graph_transpose): arcs reversed; src_deg = out-degrees of the
+    // original graph (PageRank pull divides by them)
+    bool transposed = false;
+    tigr::DevBuf src_deg;    // uint32[n] (transposed graphs only)
 };
 
 struct tigr_comm {

@@ -301,3 +301,100 @@ tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangl
 }
 
 }  // namespace tigr
+
+// ==========================================================================================
+// Pull-based PageRank: the relax runs on a virtual split of the
+// TRANSPOSED graph (tigr_graph_transpose).  Virtual node i of node v owns <= K in-arcs u->v
+// and gathers partial = sum contrib[u]; Thm. 3 (L1047-1073): pull is correct on a virtual split
+// iff the combine is associative and the family's partials meet with atomics.  Lanes of one
+// family are consecutive virtual nodes, so a warp first reduces its family segments with a
+// key-equality segmented scan (shfl_up); the segment's last lane then stores (the segment is
+// the whole family) or adds atomically (the family spans warps).  No arc-level atomics at all.
+// ==========================================================================================
+namespace tigr {
+namespace {
+
+template <int LAYOUT, int B>
+__global__ void __launch_bounds__(256) k_relax_pr_pull(RelaxArgs a) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * 256) + threadIdx.x;
+    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
+    uint32_t v[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint64_t i = base + (uint64_t)r * 256;
+        v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
+    }
+    uint4 info[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) info[r] = v[r] != kPad ? __ldg(a.vinfo + v[r]) : make_uint4(0, 0, 0, 1);
+    uint4 c0[B], c1[B];
+    uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint64_t i = base + (uint64_t)r * 256;
+        const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
+        uint32_t k;
+        if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
+        else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
+        else {
+            const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
+            k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
+            kend[r] = (per >= q - k) ? q : k + per;
+        }
+        const uint4* cb = c4 + info[r].x;
+        c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
+        c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
+        kn[r] = k + 2 * step[r];
+    }
+    double part[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+        double g[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) g[q] = nb[q] != kPad ? __ldg(a.contrib + nb[q]) : 0.0;
+        double s = 0.0;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) s += g[q];
+        const uint4* cb = c4 + info[r].x;
+        for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
+            const uint4 c = ldg_chunk(cb + k);
+            s += (c.x != kPad ? __ldg(a.contrib + c.x) : 0.0) + (c.y != kPad ? __ldg(a.contrib + c.y) : 0.0) +
+                 (c.z != kPad ? __ldg(a.contrib + c.z) : 0.0) + (c.w != kPad ? __ldg(a.contrib + c.w) : 0.0);
+        }
+        part[r] = s;
+    }
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
+        // segmented (by node) inclusive sum across the warp's consecutive virtual nodes
+        const uint32_t key = v[r];
+        double val = part[r];
+        uint32_t len = 1;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const double ov = __shfl_up_sync(0xffffffffu, val, o);
+            const uint32_t ok = __shfl_up_sync(0xffffffffu, key, o);
+            const uint32_t ol = __shfl_up_sync(0xffffffffu, len, o);
+            if (lane >= o && ok == key) { val += ov; len += ol; }
+        }
+        const uint32_t next = __shfl_down_sync(0xffffffffu, key, 1);
+        const bool last = (lane == 31) || (next != key);
+        if (key != kPad && last) {
+            const uint64_t i_last = base + (uint64_t)r * 256;
+            const bool whole = (i_last + 1 - len == info[r].z) && (len == info[r].w);
+            if (whole) a.acc[key] = val;
+            else atomicAdd(a.acc + key, val);
+        }
+    }
+}
+
+}  // namespace
+
+RelaxFn relax_pr_pull_kernel(int layout, int* per_thread) {
+    *per_thread = 4;
+    return layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_pull<TIGR_LAYOUT_STRIDED, 4>
+                                         : &k_relax_pr_pull<TIGR_LAYOUT_CONSECUTIVE, 4>;
+}
+
+}  // namespace tigr

@@ -48,6 +48,7 @@ struct PrCidPlan {
     size_t smem = 0;
 };
 bool pr_cid_enabled();
+RelaxFn relax_pr_pull_kernel(int layout, int* per_thread);   // pull PageRank (pr.cu, NEXT-1)
 tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s);
 PrCidPlan pr_cid_plan(tigr_vgraph* vg);
 tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,

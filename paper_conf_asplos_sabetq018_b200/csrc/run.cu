@@ -232,13 +232,18 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     const uint32_t n = vg->g->n;
     RelaxArgs a = make_args(vg);
     // preferred: in-degree-ordered accumulator (pr.cu); else the hashed hot-destination kernel
-    const bool use_cid = !o.collect_stats && vg->vec && pr_cid_enabled();
+    // a transposed graph runs pull-based PageRank (pr.cu, NEXT-1); divide by the original
+    // graph's out-degrees, which the transpose carries
+    const bool pull = vg->g->transposed;
+    const uint32_t* out_deg = pull ? vg->g->src_deg.as<uint32_t>() : vg->g->deg.as<uint32_t>();
+    const bool use_cid = !pull && !o.collect_stats && vg->vec && pr_cid_enabled();
     PrCidPlan cp;
     if (use_cid) {
         TIGR_TRY(pr_cid_prepare(vg, s));
         cp = pr_cid_plan(vg);
     }
-    const PrHotConfig hc = (o.collect_stats || use_cid) ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
+    const PrHotConfig hc =
+        (pull || o.collect_stats || use_cid) ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
     const RelaxHotFn hot = hc.fn;
     uint32_t* hot_cnt = ws.hot.as<uint32_t>();
     uint32_t* hot_hist = hot_cnt + n;
@@ -257,17 +262,26 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         TIGR_TRY(pr_hot_select(vg->g->col.as<uint32_t>(), vg->g->nchunks, n, hc.max_ids, hot_cnt, hot_hist, hot_ids,
                                hot_n, s));
     }
-    RelaxFn relax = relax_pr_mlp_kernel(vg->layout, vg->vec, o.collect_stats != 0);
+    RelaxFn relax = nullptr;
     uint64_t per_block = kRelaxThreads;
-    if (relax) per_block *= pr_vnodes_per_thread(vg->layout, vg->vec, o.collect_stats != 0);
-    else relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
+    if (pull) {
+        if (!vg->vec || o.collect_stats)
+            return fail(TIGR_EUNSUPPORTED, "pull PageRank needs 4 | K and collect_stats = 0");
+        int per = 1;
+        relax = relax_pr_pull_kernel(vg->layout, &per);
+        per_block *= per;
+    } else {
+        relax = relax_pr_mlp_kernel(vg->layout, vg->vec, o.collect_stats != 0);
+        if (relax) per_block *= pr_vnodes_per_thread(vg->layout, vg->vec, o.collect_stats != 0);
+        else relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
+    }
     const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
     const bool comm = o.comm != nullptr;
     const double base = (1.0 - o.pr_damping) / (double)n;
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
     TIGR_CK(cudaEventRecord(t0, s));
     TIGR_CK(cudaMemsetAsync(a.ctl, 0, sizeof(Ctl), s));
-    k_pr_init<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), ws.x.as<double>(), ws.contrib.as<double>(),
+    k_pr_init<<<grid_for(n), kBlock, 0, s>>>(n, out_deg, ws.x.as<double>(), ws.contrib.as<double>(),
                                              ws.acc.as<double>(), a.ctl);
     TIGR_CKL("pr init");
     trace(s, "pr: prepare+init");
@@ -306,7 +320,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
             TIGR_TRY(pr_cid_apply(vg, base, o.pr_damping, o.pr_dangling, dcur, dnext, s));
             continue;
         }
-        k_pr_apply<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), base, o.pr_damping, o.pr_dangling,
+        k_pr_apply<<<grid_for(n), kBlock, 0, s>>>(n, out_deg, base, o.pr_damping, o.pr_dangling,
                                                   ws.x.as<double>(), ws.contrib.as<double>(), ws.acc.as<double>(),
                                                   dcur, dnext);
         TIGR_CKL("pr apply");

@@ -329,3 +329,56 @@ def test_exchange_path_single_rank_nccl(tigr):
     assert np.array_equal(tigr.tigr_run(vgs, "cc", comm=comm), want["cc"])
     assert np.abs(tigr.tigr_run(vg, "pr", comm=comm) - want["pr"]).max() <= 1e-6
     comm.free()
+
+
+# ------------------------------------------------------------------------------------ NEXT-1: pull PR
+def _owner(rp):
+    return np.repeat(np.arange(len(rp) - 1, dtype=np.uint32), np.diff(rp))
+
+
+def test_transpose_matches_oracle(tigr):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    gt = tigr.tigr_graph_transpose(g)
+    assert gt.info()["transposed"] and gt.info()["m"] == rec.m
+    o = oracle.csr_build(rec.n, src, dst, w)
+    # the transpose keeps the forward CSR's arc order (stable): reverse the oracle's CSR arcs
+    ot = oracle.csr_build(rec.n, o.col, _owner(o.row_ptr), o.wt)
+    rp, col, wt = tigr.tigr_graph_export_csr(gt)
+    assert np.array_equal(rp, ot.row_ptr) and np.array_equal(col, ot.col) and np.array_equal(wt, ot.wt)
+    vgt = tigr.tigr_virtualize(gt, 8)
+    assert np.array_equal(tigr.tigr_run(vgt, "bfs", 3), oracle.bfs(ot, 3))   # BFS on the reversed graph
+
+
+@pytest.mark.parametrize("K", [1, 4, 8, 32, 0xFFFFFFFF])
+@pytest.mark.parametrize("layout", ["consecutive", "strided"])
+def test_pull_pagerank_cfg1(tigr, K, layout):
+    """PageRank pulled over a virtual split of the in-CSR equals the
+    push / power-iteration result (Thm. 3)."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, _ = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, None)
+    gt = tigr.tigr_graph_transpose(g)
+    if K % 4 and K != 0xFFFFFFFF:
+        with pytest.raises(tigr.TigrError):
+            tigr.tigr_run(tigr.tigr_virtualize(gt, K, layout), "pr")
+        return
+    got = tigr.tigr_run(tigr.tigr_virtualize(gt, K, layout), "pr")
+    want = oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20)
+    assert np.abs(got - want).max() <= 1e-6
+    assert np.abs(got - want).max() <= 1e-15  # float64, tiny graph: only association differs
+    for dang in (1,):
+        got = tigr.tigr_run(tigr.tigr_virtualize(gt, K, layout), "pr", pr_dangling=dang)
+        want = oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20, 0.85, dang)
+        assert np.abs(got - want).max() <= 1e-6
+
+
+def test_pull_pagerank_edge_cases(tigr):
+    for name, (n, src, dst, w) in _edge_cases().items():
+        src, dst = (np.asarray(x, dtype=np.uint32) for x in (src, dst))
+        g = tigr.tigr_graph_from_coo(n, src, dst, None)
+        gt = tigr.tigr_graph_transpose(g)
+        got = tigr.tigr_run(tigr.tigr_virtualize(gt, 8), "pr")
+        want = oracle.pagerank(oracle.csr_build(n, src, dst), 20)
+        assert np.abs(got - want).max() <= 1e-12, name

@@ -107,3 +107,15 @@ def test_cfg5_twitter_shaped_full(tigr):
     assert np.array_equal(got_sssp, oracle.sssp(o, rec.source))
     del o
     assert np.array_equal(got_cc, oracle.cc(rec.n, src, dst))
+
+
+def test_cfg4_pull_pagerank_full(tigr, cfg4):
+    """NEXT-1 at the bench's size: pull PageRank on the in-CSR of R-MAT scale 24, K=8 strided."""
+    rec, src, dst, _ = cfg4
+    g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False)
+    gt = tigr.tigr_graph_transpose(g)
+    del g
+    got = tigr.tigr_run(tigr.tigr_virtualize(gt, 8, "strided"), "pr")
+    want = oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20)
+    assert np.abs(got - want).max() <= 1e-6
+    assert np.abs(rec.n * got - rec.n * want).max() <= 1e-6
