@@ -354,6 +354,28 @@ def per_algo(tigr, torch, rec, args, s, deg):
                      "edges_processed": st["edges_processed"]}
     vg.free()
     g.free()
+    # NEXT-1: pull PageRank on the in-CSR (same graph, 20 iterations), relax timed per launch
+    g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, stream=s)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    gt = tigr.tigr_graph_transpose(g, stream=s)
+    e1.record(s)
+    torch.cuda.synchronize()
+    g.free()
+    vgt = tigr.tigr_virtualize(gt, args.K, args.layout, stream=s)
+    out64 = torch.empty(n, dtype=torch.float64, device="cuda")
+    runs = []
+    for _ in range(3):
+        _, st = tigr.tigr_run(vgt, "pr", 0, out=out64, stream=s, time_kernels=1, return_stats=True)
+        runs.append(st)
+    best = min(runs, key=lambda d: d["ms_total"])
+    relax_ms = best["ms_relax"] / max(best["relax_launches"], 1)
+    res["pr_pull"] = {"ms_20it": best["ms_total"], "relax_ms_per_launch": relax_ms,
+                      "gteps_20it": 20 * m / (best["ms_total"] * 1e-3) / 1e9,
+                      "gteps_relax": m / (relax_ms * 1e-3) / 1e9, "transpose_ms": e0.elapsed_time(e1),
+                      "note": "SURVEY NEXT-1: in-CSR via tigr_graph_transpose, warp-segmented family sums"}
+    vgt.free()
+    gt.free()
     return res
 
 

@@ -72,3 +72,33 @@ def test_opts_default_and_version():
     assert o.pr_iters == 20 and abs(o.pr_damping - 0.85) < 1e-15 and o.use_graph == 1
     assert "sm_100a" in tigr.tigr_version()
     assert ctypes.sizeof(tigr.tigr_run_opts) == 56
+
+
+def _build_c_example():
+    import paper_conf_asplos_sabetq018_b200 as tigr
+    os.makedirs(os.path.join(ROOT, "build"), exist_ok=True)
+    exe = os.path.join(ROOT, "build", "c_abi_bfs")
+    libdir = os.path.dirname(tigr.LIB_PATH)
+    subprocess.run(["gcc", "-std=c11", "-Wall", "-Werror", "-I", os.path.join(ROOT, "include"),
+                    os.path.join(ROOT, "examples", "c_abi_bfs.c"), "-L", libdir, "-ltigr",
+                    f"-Wl,-rpath,{libdir}", "-o", exe], check=True)
+    return exe
+
+
+def test_c_program_against_header_host_only():
+    """A plain C program compiled against include/tigr.h links libtigr.so and runs the
+    host-only entry points; compute calls report TIGR_ECUDA without a GPU."""
+    import torch
+    exe = _build_c_example()
+    if torch.cuda.is_available():
+        pytest.skip("GPU present: covered by the GPU variant")
+    r = subprocess.run([exe], capture_output=True, text=True)
+    assert r.returncode == 0, r.stdout + r.stderr
+
+
+@pytest.mark.gpu
+def test_c_program_against_header_gpu():
+    exe = _build_c_example()
+    r = subprocess.run([exe, "--gpu"], capture_output=True, text=True)
+    assert r.returncode == 0, r.stdout + r.stderr
+    assert "GPU checks ok" in r.stdout
