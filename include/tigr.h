@@ -148,6 +148,16 @@ tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* 
  * Errors: ENOMEM, ECUDA. */
 tigr_status tigr_graph_transpose(const tigr_graph* g, void* stream, tigr_graph** out);
 
+/* PHYSICAL uniform-degree-tree transformation (UDT, §3.2 Alg. 1): every
+ * node v of out-degree d > K keeps <= K arcs and hands the rest to t = ceil((d-K)/(K-1)) new
+ * split nodes of out-degree exactly K, numbered n, n+1, ... in order of v and creation (the
+ * queue order of Alg. 1).  Arcs to original neighbours keep their weight (unit_weight if g is
+ * unweighted); arcs to split nodes get dumb_weight: 0 for SSSP/BFS, 0xFFFFFFFF for SSWP
+ * (Cor. 2-3, L695-734).  The result is a weighted graph with n + T nodes; results of the
+ * original nodes are its first n values (Thm. 1).  Errors: EINVAL (K < 2), ERANGE. */
+tigr_status tigr_graph_udt(const tigr_graph* g, uint32_t K, uint32_t dumb_weight, uint32_t unit_weight,
+                           void* stream, tigr_graph** out);
+
 /* Copy the CSR out (row_ptr[n+1], col[m], w[m] if weighted and w != NULL), arcs of a
  * source contiguous in the graph's internal order. */
 tigr_status tigr_graph_export_csr(const tigr_graph* g, int64_t* row_ptr, uint32_t* col, uint32_t* w,

@@ -44,6 +44,7 @@ def _lib():
             "or_sswp": (ctypes.c_int, [_U32, _P, _P, _P, _U32, _P]),
             "or_cc": (ctypes.c_int, [_U32, _U64, _P, _P, _P]),
             "or_pagerank": (ctypes.c_int, [_U32, _P, _P, _U32, ctypes.c_double, ctypes.c_int, _P]),
+            "or_udt": (_U64, [_U32, _P, _P, _P, _U64, _U32, _U32, _P, _P, _P, _P]),
             "or_push_virtual": (_I64, [_U32, _P, _P, _P, _P, _P, _U64, ctypes.c_int, _U64,
                                        ctypes.c_int, _U32, ctypes.c_int, ctypes.c_int, _P, _U64, _P]),
         }
@@ -172,6 +173,23 @@ def push_virtual(g: CSR, vg: Virtual, algo: int, source: int = 0, layout: int = 
     if it < 0:
         raise ValueError(f"or_push_virtual failed ({it})")
     return out, int(it), bool(conv.value)
+
+
+def udt(g: CSR, K: int, dumb: int, unit_weight: int = 1):
+    """Alg. 1 (UDT) on the oracle CSR: returns (n', src, dst, w) of the transformed graph.
+    Arcs to original neighbours keep their weight (unit_weight when g is unweighted), arcs
+    to new split nodes get `dumb` (0 for SSSP/BFS, 0xFFFFFFFF for SSWP; Cor. 2-3)."""
+    m = ctypes.c_uint64(0)
+    _lib().or_udt(g.n, _p(g.row_ptr), _p(g.col), _p(g.wt), K, dumb, unit_weight, None, None, None,
+                  ctypes.byref(m))
+    src = np.empty(m.value, np.uint32)
+    dst = np.empty(m.value, np.uint32)
+    w = np.empty(m.value, np.uint32)
+    n2 = _lib().or_udt(g.n, _p(g.row_ptr), _p(g.col), _p(g.wt), K, dumb, unit_weight, _p(src), _p(dst),
+                       _p(w), ctypes.byref(m))
+    if n2 == 0 and g.n:
+        raise ValueError("or_udt failed (K < 2?)")
+    return int(n2), src, dst, w
 
 
 def run(algo: str, n: int, src, dst, w=None, source: int = 0, pr_iters: int = 20,

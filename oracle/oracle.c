@@ -381,3 +381,61 @@ int64_t or_push_virtual(uint32_t n, const int64_t* row_ptr, const uint32_t* col,
     free(prev); free(active); free(next); free(edges);
     return it;
 }
+
+/* ------------------------------------------------------------------------- */
+/* UDT physical transformation (§3.2 Alg. 1; dumb weights §3.3 Cor. 2-3 */
+/* L695-734), run literally with a queue per high-degree node.  Node v with    */
+/* d_v > K: q = v's neighbours (in CSR order), remove them from v; while       */
+/* |q| > K: new node u gets K neighbours popped from the front, u is pushed;   */
+/* finally v gets the <= K remaining entries.  New nodes are numbered n, n+1,  */
+/* ... in creation order over v = 0..n-1.  An arc to an original neighbour      */
+/* keeps its weight; an arc to a new node gets `dumb`.  Output: arc list        */
+/* (src, dst, w) in creation order; returns the new node count n' (or 0 when    */
+/* the output buffers are NULL: then *m_out receives the arc count only).      */
+/* K >= 2 (K = 1 never terminates: each step removes 1 and adds 1).            */
+/* ------------------------------------------------------------------------- */
+uint64_t or_udt(uint32_t n, const int64_t* row_ptr, const uint32_t* col, const uint32_t* wt, uint64_t K,
+                uint32_t dumb, uint32_t unit_weight, uint32_t* src, uint32_t* dst, uint32_t* w, uint64_t* m_out) {
+    if (K < 2) return 0;
+    uint64_t next = n, arcs = 0;
+    uint64_t maxd = 0;
+    for (uint32_t v = 0; v < n; ++v) {
+        uint64_t d = (uint64_t)(row_ptr[v + 1] - row_ptr[v]);
+        if (d > maxd) maxd = d;
+    }
+    /* queue of (node id, weight of the arc that will point to it) */
+    uint64_t cap = maxd + maxd / (K - 1) + 2;
+    uint64_t* qn = (uint64_t*)malloc(sizeof(uint64_t) * cap);
+    uint32_t* qw = (uint32_t*)malloc(sizeof(uint32_t) * cap);
+    if (!qn || !qw) { free(qn); free(qw); return 0; }
+#define OR_EMIT(s_, d_, w_)                              \
+    do {                                                 \
+        if (src) { src[arcs] = (uint32_t)(s_); dst[arcs] = (uint32_t)(d_); w[arcs] = (w_); } \
+        ++arcs;                                          \
+    } while (0)
+    for (uint32_t v = 0; v < n; ++v) {
+        uint64_t d = (uint64_t)(row_ptr[v + 1] - row_ptr[v]);
+        if (d <= K) {                                    /* not a high-degree node: unchanged */
+            for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) OR_EMIT(v, col[e], wt ? wt[e] : unit_weight);
+            continue;
+        }
+        uint64_t head = 0, tail = 0;
+        for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; ++e) {   /* Alg. 1 lines 3-5 */
+            qn[tail] = col[e];
+            qw[tail] = wt ? wt[e] : unit_weight;
+            ++tail;
+        }
+        while (tail - head > K) {                                   /* lines 6-10 */
+            uint64_t u = next++;
+            for (uint64_t i = 0; i < K; ++i, ++head) OR_EMIT(u, qn[head], qw[head]);
+            qn[tail] = u;
+            qw[tail] = dumb;
+            ++tail;
+        }
+        for (; head < tail; ++head) OR_EMIT(v, qn[head], qw[head]);  /* lines 11-13 */
+    }
+#undef OR_EMIT
+    free(qn); free(qw);
+    if (m_out) *m_out = arcs;
+    return next;
+}

@@ -69,6 +69,7 @@ _SIGS = {
     "tigr_graph_info": (_I, [_P, ctypes.POINTER(_U32), ctypes.POINTER(_U64), ctypes.POINTER(_I),
                              ctypes.POINTER(_I), ctypes.POINTER(_I), ctypes.POINTER(_U64)]),
     "tigr_graph_transpose": (_I, [_P, _P, ctypes.POINTER(_P)]),
+    "tigr_graph_udt": (_I, [_P, _U32, _U32, _U32, _P, ctypes.POINTER(_P)]),
     "tigr_graph_export_csr": (_I, [_P, _P, _P, _P, _I, _P]),
     "tigr_graph_free": (None, [_P]),
     "tigr_virtualize": (_I, [_P, _U32, _I, _P, ctypes.POINTER(_P)]),
@@ -258,6 +259,13 @@ def tigr_graph_transpose(g: Graph, stream=None) -> Graph:
     """In-CSR of g (arcs reversed; carries g's out-degrees: TIGR_PR on it is pull-based)."""
     out = _P()
     _check(_lib.tigr_graph_transpose(g.ptr, _stream_ptr(stream), ctypes.byref(out)))
+    return Graph(out.value)
+
+
+def tigr_graph_udt(g: Graph, K: int, dumb_weight: int = 0, unit_weight: int = 1, stream=None) -> Graph:
+    """Physical UDT transformation (Alg. 1): n + T nodes; originals keep ids 0..n-1."""
+    out = _P()
+    _check(_lib.tigr_graph_udt(g.ptr, K, dumb_weight, unit_weight, _stream_ptr(stream), ctypes.byref(out)))
     return Graph(out.value)
 
 

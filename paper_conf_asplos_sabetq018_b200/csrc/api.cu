@@ -161,6 +161,8 @@ tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, con
                                   int symmetric_hint, cudaStream_t s, tigr_graph** out);
 tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w, cudaStream_t s);
 tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out);
+tigr_status graph_udt_device(const tigr_graph* g, uint32_t K, uint32_t dumb, uint32_t unit, cudaStream_t s,
+                             tigr_graph** out);
 tigr_status graph_rmat_device(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed, uint64_t wseed,
                               uint32_t wmin, uint32_t wmax, int weighted, int symmetrize, cudaStream_t s,
                               tigr_graph** out);
@@ -308,6 +310,16 @@ tigr_status tigr_graph_export_csr(const tigr_graph* g, int64_t* row_ptr, uint32_
 }
 
 void tigr_graph_free(tigr_graph* g) { delete g; }
+
+tigr_status tigr_graph_udt(const tigr_graph* g, uint32_t K, uint32_t dumb_weight, uint32_t unit_weight, void* stream,
+                           tigr_graph** out) {
+    if (!g || !out) return fail(TIGR_EINVAL, "graph_udt: NULL argument");
+    *out = nullptr;
+    cudaStream_t s = (cudaStream_t)stream;
+    TIGR_TRY(graph_udt_device(g, K, dumb_weight, unit_weight, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
 
 tigr_status tigr_graph_transpose(const tigr_graph* g, void* stream, tigr_graph** out) {
     if (!g || !out) return fail(TIGR_EINVAL, "graph_transpose: NULL argument");

@@ -114,6 +114,67 @@ __global__ void k_expand_arcs(const int64_t* __restrict__ rp, const uint32_t* __
     }
 }
 
+// ---- UDT (physical uniform-degree-tree transformation, §3.2 Alg. 1) ----
+// Node v of out-degree d > K gets t = ceil((d-K)/(K-1)) new split nodes.  Alg. 1's queue is
+// the sequence S = (v's neighbours in CSR order, then the new nodes N_0..N_{t-1}); N_k pops
+// S[kK, kK+K) and the root v keeps S[tK, d+t).  So every arc's new source follows from its
+// S-position alone: N_{p/K} if p < tK else v -- no queue needed on the device.
+__global__ void k_udt_count(const uint32_t* __restrict__ deg, uint32_t n, uint32_t K, uint32_t* __restrict__ t) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    const uint32_t d = deg[v];
+    t[v] = d > K ? (d - K + (K - 2)) / (K - 1) : 0u;
+}
+
+__global__ void k_udt_arcs(const int64_t* __restrict__ rp, const uint32_t* __restrict__ cptr, uint32_t n,
+                           uint64_t m, const uint32_t* __restrict__ col, const uint32_t* __restrict__ wt,
+                           const uint32_t* __restrict__ tptr, uint32_t K, uint32_t dumb, uint32_t unit,
+                           uint32_t* __restrict__ src, uint32_t* __restrict__ dst, uint32_t* __restrict__ w) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    const int lane = threadIdx.x & 31;
+    uint64_t beg = 0, cb = 0;
+    uint32_t d = 0, tb = 0, t = 0;
+    if (v < n) {
+        beg = (uint64_t)rp[v]; d = (uint32_t)(rp[v + 1] - rp[v]); cb = (uint64_t)cptr[v] * kChunk;
+        tb = tptr[v]; t = tptr[v + 1] - tb;
+    }
+    auto parent = [&](uint32_t vv, uint64_t p, uint32_t tt, uint32_t tbb) -> uint32_t {
+        return p < (uint64_t)tt * K ? n + tbb + (uint32_t)(p / K) : vv;
+    };
+    const uint32_t work = d + t;
+    const bool big = work > 32;
+    if (!big) {
+        for (uint32_t p = 0; p < d; ++p) {
+            src[beg + p] = parent(v, p, t, tb);
+            dst[beg + p] = col[cb + p];
+            w[beg + p] = wt ? wt[cb + p] : unit;
+        }
+        for (uint32_t k = 0; k < t; ++k) {
+            src[m + tb + k] = parent(v, (uint64_t)d + k, t, tb);
+            dst[m + tb + k] = n + tb + k;
+            w[m + tb + k] = dumb;
+        }
+    }
+    uint32_t mask = __ballot_sync(0xffffffffu, big);
+    while (mask) {
+        const int l = __ffs(mask) - 1;
+        mask &= mask - 1;
+        const uint64_t b = __shfl_sync(0xffffffffu, beg, l), c = __shfl_sync(0xffffffffu, cb, l);
+        const uint32_t dd = __shfl_sync(0xffffffffu, d, l), vv = __shfl_sync(0xffffffffu, v, l);
+        const uint32_t tt = __shfl_sync(0xffffffffu, t, l), tbb = __shfl_sync(0xffffffffu, tb, l);
+        for (uint32_t p = lane; p < dd; p += 32) {
+            src[b + p] = parent(vv, p, tt, tbb);
+            dst[b + p] = col[c + p];
+            w[b + p] = wt ? wt[c + p] : unit;
+        }
+        for (uint32_t k = lane; k < tt; k += 32) {
+            src[m + tbb + k] = parent(vv, (uint64_t)dd + k, tt, tbb);
+            dst[m + tbb + k] = n + tbb + k;
+            w[m + tbb + k] = dumb;
+        }
+    }
+}
+
 unsigned capped_grid(uint64_t items) {
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
@@ -240,6 +301,32 @@ tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_gra
     if (st != TIGR_OK) { delete t; return st; }
     *out = t;
     return TIGR_OK;
+}
+
+tigr_status graph_udt_device(const tigr_graph* g, uint32_t K, uint32_t dumb, uint32_t unit, cudaStream_t s,
+                             tigr_graph** out) {
+    if (K < 2) return fail(TIGR_EINVAL, "udt: K must be >= 2 (Alg. 1 does not terminate for K = 1)");
+    const uint32_t n = g->n;
+    TmpBuf t, tptr;
+    TIGR_TRY(t.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(tptr.alloc(sizeof(uint32_t) * ((size_t)n + 1), s));
+    k_udt_count<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), n, K, t.as<uint32_t>());
+    TIGR_CKL("udt count");
+    uint64_t T = 0;
+    TIGR_TRY(exclusive_scan_u32(t.as<uint32_t>(), n, SCAN_U32, 1, tptr.as<uint32_t>(), s, &T));
+    if ((uint64_t)n + T > 0xFFFFFFFEull) return fail(TIGR_ERANGE, "udt: too many split nodes");
+    const uint64_t M = g->m + T;
+    TmpBuf src, dst, w;
+    TIGR_TRY(src.alloc(sizeof(uint32_t) * (M ? M : 1), s));
+    TIGR_TRY(dst.alloc(sizeof(uint32_t) * (M ? M : 1), s));
+    TIGR_TRY(w.alloc(sizeof(uint32_t) * (M ? M : 1), s));
+    k_udt_arcs<<<grid_for(n), kBlock, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), n, g->m,
+                                              g->col.as<uint32_t>(), g->weighted ? g->wt.as<uint32_t>() : nullptr,
+                                              tptr.as<uint32_t>(), K, dumb, unit, src.as<uint32_t>(),
+                                              dst.as<uint32_t>(), w.as<uint32_t>());
+    TIGR_CKL("udt arcs");
+    return graph_from_coo_device((uint32_t)(n + T), M, src.as<uint32_t>(), dst.as<uint32_t>(), w.as<uint32_t>(), 0, s,
+                                 out);
 }
 
 tigr_status graph_rmat_device(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed,

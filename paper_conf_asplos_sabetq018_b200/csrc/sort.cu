@@ -11,6 +11,7 @@
 // hottest vertex owns 0.14% of all arcs at scale 24) costs nothing.  Degrees come from the
 // run boundaries of the sorted keys; a final kernel places each arc into the 16-byte-aligned,
 // padded segment of its source.
+#include <cstdlib>
 #include <utility>
 
 #include "internal.cuh"
@@ -22,9 +23,7 @@ constexpr int kST = 256;                 // threads per sort tile
 #ifndef TIGR_SORT_MINB
 #define TIGR_SORT_MINB 3
 #endif
-constexpr int kSI = 16;                  // items per thread
 constexpr int kSW = kST / 32;            // warps per tile
-constexpr int kTileItems = kST * kSI;    // 4096
 constexpr int kMaxRadix = 256;
 constexpr uint64_t kFlagAgg = 1ull << 46, kFlagInc = 2ull << 46, kValMask = (1ull << 46) - 1;
 
@@ -106,8 +105,8 @@ __device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
 // One pass of the stable LSD radix sort over a tile of 4096 arcs.  Values are staged into
 // shared memory with cp.async as soon as the tile is known (no registers held across the
 // ranking / look-back); keys stay in registers; digits are recomputed from the keys.
-template <bool W, bool FIRST>
-__global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t* __restrict__ kin,
+template <bool W, bool FIRST, int SI>
+__global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_onesweep(const uint32_t* __restrict__ kin,
                                                   const typename ValT<W>::T* __restrict__ vin,
                                                   const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst,
                                                   const uint32_t* __restrict__ w, uint64_t m, uint64_t M, int shift,
@@ -117,8 +116,8 @@ __global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t
     typedef typename ValT<W>::T VT;
     extern __shared__ __align__(16) unsigned char smem[];
     VT* s_vin = reinterpret_cast<VT*>(smem);                                   // tile values, input order
-    VT* s_val = reinterpret_cast<VT*>(smem + sizeof(VT) * kTileItems);         // values, digit order
-    uint32_t* s_key = reinterpret_cast<uint32_t*>(smem + 2 * sizeof(VT) * kTileItems);
+    VT* s_val = reinterpret_cast<VT*>(smem + sizeof(VT) * (kST * SI));         // values, digit order
+    uint32_t* s_key = reinterpret_cast<uint32_t*>(smem + 2 * sizeof(VT) * (kST * SI));
     __shared__ uint32_t s_wcnt[kSW][kMaxRadix + 1];
     __shared__ uint32_t s_dstart[kMaxRadix + 1];
     __shared__ uint64_t s_gofs[kMaxRadix];
@@ -130,16 +129,16 @@ __global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t
     for (int i = t; i < kSW * (kMaxRadix + 1); i += kST) (&s_wcnt[0][0])[i] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t base = (uint64_t)tile * kTileItems;
+    const uint64_t base = (uint64_t)tile * (kST * SI);
     const int radix = 1 << bits;
     const uint32_t mask = (uint32_t)radix - 1;
-    const uint32_t cnt = (M - base < (uint64_t)kTileItems) ? (uint32_t)(M - base) : (uint32_t)kTileItems;
+    const uint32_t cnt = (M - base < (uint64_t)(kST * SI)) ? (uint32_t)(M - base) : (uint32_t)(kST * SI);
 
     // values -> shared memory (asynchronous, coalesced), keys -> registers
-    uint32_t key[kSI];
+    uint32_t key[SI];
 #pragma unroll
-    for (int r = 0; r < kSI; ++r) {
-        const uint32_t li = wp * (kSI * 32) + r * 32 + lane;
+    for (int r = 0; r < SI; ++r) {
+        const uint32_t li = wp * (SI * 32) + r * 32 + lane;
         const uint64_t idx = base + li;
         key[r] = 0;
         if (li < cnt) {
@@ -169,11 +168,11 @@ __global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t
     // warp issues the rounds' atomics in order, so reservations follow item order; the
     // results are broadcast after all rounds are issued (no per-round round trip).
     const uint32_t lt = (1u << lane) - 1;
-    uint32_t peers[kSI];
-    uint32_t rank[kSI / 2];  // two 16-bit ranks per register
+    uint32_t peers[SI];
+    uint32_t rank[SI / 2];  // two 16-bit ranks per register
 #pragma unroll
-    for (int r = 0; r < kSI; ++r) {
-        const uint32_t li = wp * (kSI * 32) + r * 32 + lane;
+    for (int r = 0; r < SI; ++r) {
+        const uint32_t li = wp * (SI * 32) + r * 32 + lane;
         const uint32_t d = li < cnt ? (key[r] >> shift) & mask : (uint32_t)radix;
         peers[r] = __match_any_sync(0xffffffffu, d);
         uint32_t got = 0;
@@ -181,7 +180,7 @@ __global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t
         if (r & 1) rank[r >> 1] |= got << 16; else rank[r >> 1] = got;
     }
 #pragma unroll
-    for (int r = 0; r < kSI; ++r) {
+    for (int r = 0; r < SI; ++r) {
         const uint32_t mine = (rank[r >> 1] >> ((r & 1) * 16)) & 0xFFFFu;
         const uint32_t b = __shfl_sync(0xffffffffu, mine, __ffs(peers[r]) - 1) + __popc(peers[r] & lt);
         rank[r >> 1] = (r & 1) ? ((rank[r >> 1] & 0xFFFFu) | (b << 16)) : ((rank[r >> 1] & 0xFFFF0000u) | b);
@@ -235,8 +234,8 @@ __global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t
     __syncthreads();
     // reorder the tile by digit in shared memory
 #pragma unroll
-    for (int r = 0; r < kSI; ++r) {
-        const uint32_t li = wp * (kSI * 32) + r * 32 + lane;
+    for (int r = 0; r < SI; ++r) {
+        const uint32_t li = wp * (SI * 32) + r * 32 + lane;
         if (li < cnt) {
             const uint32_t d = (key[r] >> shift) & mask;
             const uint32_t lp = s_dstart[d] + s_wcnt[wp][d] + ((rank[r >> 1] >> ((r & 1) * 16)) & 0xFFFFu);
@@ -246,7 +245,7 @@ __global__ void __launch_bounds__(kST, TIGR_SORT_MINB) k_onesweep(const uint32_t
     }
     __syncthreads();
 #pragma unroll
-    for (int r = 0; r < kSI; ++r) {
+    for (int r = 0; r < SI; ++r) {
         const uint32_t i = r * kST + t;
         if (i < cnt) {
             const uint32_t k = s_key[i];
@@ -306,7 +305,10 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
     const int passes = key_bits == 0 ? 1 : (key_bits + 7) / 8;
     const int bits = key_bits == 0 ? 1 : (key_bits + passes - 1) / passes;
-    const uint64_t tiles = (M + kTileItems - 1) / kTileItems;
+    const char* si_env = getenv("TIGR_SORT_SI");
+    const int SI = si_env ? atoi(si_env) : 16;
+    const uint64_t tile_items = (uint64_t)kST * SI;
+    const uint64_t tiles = (M + tile_items - 1) / tile_items;
 
     TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid;
     trace(s, "sort: enter");
@@ -339,10 +341,17 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     k_digit_base<<<1, kMaxRadix, 0, s>>>(hist.as<unsigned long long>(), passes, dbase.as<uint64_t>());
     TIGR_CKL("digit base");
     trace(s, "sort: digit histograms");
-    const size_t smem = (2 * sizeof(VT) + sizeof(uint32_t)) * kTileItems;
+    const size_t smem = (2 * sizeof(VT) + sizeof(uint32_t)) * tile_items;
     int cur = 0;
     for (int p = 0; p < passes && M; ++p) {
-        auto kern = (p == 0) ? &k_onesweep<W, true> : &k_onesweep<W, false>;
+        void (*kern)(const uint32_t*, const VT*, const uint32_t*, const uint32_t*, const uint32_t*, uint64_t,
+                     uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*, uint64_t, uint32_t*, VT*);
+        switch (SI) {
+            case 12: kern = p == 0 ? &k_onesweep<W, true, 12> : &k_onesweep<W, false, 12>; break;
+            case 20: kern = p == 0 ? &k_onesweep<W, true, 20> : &k_onesweep<W, false, 20>; break;
+            case 24: kern = p == 0 ? &k_onesweep<W, true, 24> : &k_onesweep<W, false, 24>; break;
+            default: kern = p == 0 ? &k_onesweep<W, true, 16> : &k_onesweep<W, false, 16>; break;
+        }
         TIGR_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         const int out = (p == 0) ? 0 : 1 - cur;
         kern<<<(unsigned)tiles, kST, smem, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), src, dst, w, m, M, p * bits,

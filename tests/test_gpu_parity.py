@@ -382,3 +382,32 @@ def test_pull_pagerank_edge_cases(tigr):
         got = tigr.tigr_run(tigr.tigr_virtualize(gt, 8), "pr")
         want = oracle.pagerank(oracle.csr_build(n, src, dst), 20)
         assert np.abs(got - want).max() <= 1e-12, name
+
+
+# ------------------------------------------------------------------------------------ NEXT-4: UDT
+@pytest.mark.parametrize("K", [2, 3, 8])
+def test_udt_matches_oracle(tigr, K):
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    n2, us, ud, uw = oracle.udt(o, K, 0)
+    gu = tigr.tigr_graph_udt(g, K, 0)
+    assert gu.info()["n"] == n2 and gu.info()["m"] == len(us)
+    ou = oracle.csr_build(n2, us, ud, uw)
+    rp, col, wt = tigr.tigr_graph_export_csr(gu)
+    assert np.array_equal(rp, ou.row_ptr) and np.array_equal(col, ou.col) and np.array_equal(wt, ou.wt)
+    # Cor. 2: SSSP over the UDT graph (any virtual split of it) keeps the original distances
+    for vk in (8, 0xFFFFFFFF):
+        vgu = tigr.tigr_virtualize(gu, vk)
+        assert np.array_equal(tigr.tigr_run(vgu, "sssp", 0)[:rec.n], oracle.sssp(o, 0))
+    # Cor. 3: SSWP with dumb weight = +inf
+    gw = tigr.tigr_graph_udt(g, K, 0xFFFFFFFF)
+    assert np.array_equal(tigr.tigr_run(tigr.tigr_virtualize(gw, 8), "sswp", 0)[:rec.n], oracle.sswp(o, 0))
+    # BFS = SSSP with unit weights on an unweighted graph's UDT
+    g1 = tigr.tigr_graph_from_coo(rec.n, src, dst, None)
+    gb = tigr.tigr_graph_udt(g1, K, 0, 1)
+    assert np.array_equal(tigr.tigr_run(tigr.tigr_virtualize(gb, 8), "sssp", 0)[:rec.n],
+                          oracle.bfs(oracle.csr_build(rec.n, src, dst), 0))
+    with pytest.raises(tigr.TigrError):
+        tigr.tigr_graph_udt(g, 1, 0)

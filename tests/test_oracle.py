@@ -299,3 +299,43 @@ def test_fixed_point_invariants_cfg2():
     lab = oracle.cc(n, src, dst)
     assert (lab[src] == lab[dst]).all() and (lab <= np.arange(n)).all()
     assert (lab[lab] == lab).all()
+
+
+# --------------------------------------------------------------------------------------------
+# UDT (Alg. 1) -- pinned by Thm. 1 / Cor. 1-3 against the textbook results on the original
+# --------------------------------------------------------------------------------------------
+
+@pytest.mark.parametrize("K", [2, 3, 8])
+def test_udt_preserves_results(K):
+    n = 300
+    src, dst, w = graphgen.rmat(n, 5000, 0.57, 0.19, 0.19, seed=61, wseed=62)
+    g = oracle.csr_build(n, src, dst, w)
+    deg = g.degrees()
+    # SSSP with dumb weight 0 (Cor. 2): distances of original nodes unchanged
+    n2, us, ud, uw = oracle.udt(g, K, 0)
+    gu = oracle.csr_build(n2, us, ud, uw)
+    assert np.array_equal(oracle.sssp(gu, 0)[:n], oracle.sssp(g, 0))
+    # structure: every node has out-degree <= K; new nodes exactly K (L567-569); arcs = m + #new
+    du = gu.degrees()
+    assert du.max() <= K and (du[n:] == K).all() and gu.m == g.m + (n2 - n)
+    # #new nodes per high-degree node d: ceil((d-K)/(K-1)) (queue shrinks by K-1 per new node)
+    hi_deg = deg[deg > K]
+    assert n2 - n == int(sum(-(-(d - K) // (K - 1)) for d in hi_deg))
+    # BFS = SSSP with unit weights on original arcs and dumb 0 (L718-720)
+    g1 = oracle.csr_build(n, src, dst)
+    n2, us, ud, uw = oracle.udt(g1, K, 0, unit_weight=1)
+    assert np.array_equal(oracle.sssp(oracle.csr_build(n2, us, ud, uw), 0)[:n], oracle.bfs(g1, 0))
+    # SSWP with dumb weight +inf (Cor. 3)
+    n2, us, ud, uw = oracle.udt(g, K, 0xFFFFFFFF)
+    assert np.array_equal(oracle.sswp(oracle.csr_build(n2, us, ud, uw), 0)[:n], oracle.sswp(g, 0))
+    # connectivity (Cor. 1): weak components restricted to original nodes unchanged
+    assert np.array_equal(oracle.cc(n2, us, ud)[:n], oracle.cc(n, src, dst))
+
+
+def test_udt_example_degree_five():
+    """Fig. 6-(b) (L566): a node of degree five with K = 2 -> 3 new nodes, root keeps 2."""
+    g = oracle.csr_build(6, [0] * 5, [1, 2, 3, 4, 5], [1, 1, 1, 1, 1])
+    n2, us, ud, uw = oracle.udt(g, 2, 0)
+    assert n2 == 6 + 3
+    gu = oracle.csr_build(n2, us, ud, uw)
+    assert list(gu.degrees()) == [2, 0, 0, 0, 0, 0, 2, 2, 2]

@@ -59,6 +59,32 @@ def main():
                                   "edges_processed": st2["edges_processed"],
                                   "active_vnodes": st2["active_vnodes"]}), flush=True)
             vg.free()
+        # Tigr-UDT (physical transformation, Alg. 1 + dumb weights, Cor. 2-3): no virtual split
+        if algo in ("sssp", "sswp", "bfs"):
+            for Ku in (8, 32):
+                if algo == "bfs":
+                    g1 = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed,
+                                              weighted=False, stream=s)
+                    gu = tigr.tigr_graph_udt(g1, Ku, 0, 1, stream=s)
+                    g1.free()
+                    run_algo = "sssp"  # BFS = SSSP with unit weights and dumb weight 0
+                else:
+                    gu = tigr.tigr_graph_udt(g, Ku, 0 if algo == "sssp" else 0xFFFFFFFF, stream=s)
+                    run_algo = algo
+                vgu = tigr.tigr_virtualize(gu, INF_K, "strided", stream=s)
+                for mname, front, sched in (("worklist async", 1, 0), ("worklist BSP", 1, 1)):
+                    times = []
+                    for _ in range(args.reps):
+                        _, st = tigr.tigr_run(vgu, run_algo, rec.source, stream=s, return_stats=True,
+                                              frontier=front, schedule=sched)
+                        times.append(st["ms_total"])
+                    ms = statistics.median(times)
+                    print(json.dumps({"cfg": args.cfg, "algo": algo, "variant": f"Tigr-UDT K={Ku}", "mode": mname,
+                                      "K": Ku, "layout": "physical", "nodes": gu.info()["n"], "ms": ms,
+                                      "speedup_vs_baseline": base_ms[mname] / ms,
+                                      "iterations": st["iterations"]}), flush=True)
+                vgu.free()
+                gu.free()
 
 
 if __name__ == "__main__":
