@@ -192,14 +192,22 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
             info[r] = __ldg(a.vinfo + v[r]);
         }
     }
-    uint4 c0[B], c1[B], w0[B], w1[B];
-    uint32_t kn[B], kend[B], step[B];
+    bool any = false;
 #pragma unroll
     for (int r = 0; r < B; ++r) {
         if (FRONT == TIGR_FRONTIER_NONE) {
             if ((A == TIGR_BFS || A == TIGR_SSSP) && x[r] == kInf) act[r] = false;
             if (A == TIGR_SSWP && x[r] == 0) act[r] = false;
         }
+        any |= act[r];
+    }
+    // a warp whose 4x32 virtual nodes are all inactive leaves now: sparse iterations cost one
+    // coalesced vn_phys read and one stamp gather per virtual node, not the whole relax body
+    if (!__any_sync(0xffffffffu, any)) return;
+    uint4 c0[B], c1[B], w0[B], w1[B];
+    uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+    for (int r = 0; r < B; ++r) {
         const uint64_t i = base + (uint64_t)r * kRelaxThreads;
         const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
         uint32_t k;
