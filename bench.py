@@ -59,15 +59,47 @@ def parse():
 
 
 # ------------------------------------------------------------------------------------------ clocks
+def gpu_uuid(torch, dev):
+    try:
+        u = str(torch.cuda.get_device_properties(dev).uuid)
+        return u if u.startswith("GPU-") else "GPU-" + u
+    except Exception:
+        return None
+
+
 class ClockSampler:
+    """SM clock + throttle reasons sampled DURING the timed region: an NVML thread polling every
+    10 ms (no process start-up lag, so even a short timed region gets samples); nvidia-smi
+    -lms 100 when NVML is unavailable."""
     Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
          "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
-    def __init__(self, index):
-        self.index, self.rows, self.proc = index, [], None
+    def __init__(self, index, uuid=None):
+        self.index, self.uuid, self.rows, self.proc, self.nvml = index, uuid, [], None, None
+        self.stop_flag = threading.Event()
 
     def start(self):
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            try:
+                h = nv.nvmlDeviceGetHandleByUUID(self.uuid) if self.uuid else None
+            except nv.NVMLError:
+                h = None
+            self.h = h if h is not None else nv.nvmlDeviceGetHandleByIndex(self.index)
+            self.nvml = nv
+            self.max_sm = nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM)
+            self.bits = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                         nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+            self._sample_nvml()
+            self.rows.clear()
+            self.thread = threading.Thread(target=self._poll_nvml, daemon=True)
+            self.thread.start()
+            return
+        except Exception:
+            self.nvml = None
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
@@ -77,6 +109,20 @@ class ClockSampler:
         except OSError:
             self.proc = None
 
+    def _sample_nvml(self):
+        nv = self.nvml
+        sm = nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM)
+        r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        self.rows.append([str(sm), str(self.max_sm), ""] + ["Active" if r & b else "Not Active" for b in self.bits])
+
+    def _poll_nvml(self):
+        while not self.stop_flag.is_set():
+            try:
+                self._sample_nvml()
+            except Exception:
+                return
+            self.stop_flag.wait(0.01)
+
     def _read(self):
         for line in self.proc.stdout:
             parts = [p.strip() for p in line.split(",")]
@@ -84,18 +130,22 @@ class ClockSampler:
                 self.rows.append(parts)
 
     def stop(self):
+        src = "nvml 10 ms" if self.nvml else "nvidia-smi 100 ms"
+        if self.nvml:
+            self.stop_flag.set()
+            self.thread.join(timeout=2)
         if self.proc:
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)
             except subprocess.TimeoutExpired:
                 self.proc.kill()
-        sms = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
-        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower() == "active"})
+        rows = list(self.rows)
+        sms = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in rows if r[1].replace(".", "").isdigit()]
+        reasons = sorted({self.NAMES[i] for r in rows for i in range(4) if r[3 + i].lower() == "active"})
         return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(rows), "sampler": src}
 
 
 # ------------------------------------------------------------------------------------------ reference arm
@@ -154,7 +204,8 @@ def config_obj(args, rec):
     return {"workload": f"{args.config}: R-MAT n={rec.n:,} m={rec.m:,} (a,b,c)=({rec.a},{rec.b},{rec.c}) "
                         f"PageRank 20 iterations, K={args.K}, {args.layout} layout",
             "algorithm": "pagerank", "K": args.K, "layout": args.layout, "n": rec.n, "m": rec.m,
-            "parallelism": "vnode-range data parallel + NCCL all-reduce" if args.gpus > 1 else "single GPU",
+            "parallelism": ("source-range partitioned CSR build per rank (arc-balanced cuts) + NCCL all-reduce "
+                            "of the PageRank accumulator each iteration") if args.gpus > 1 else "single GPU",
             "l2": "flushed between steps (512 MiB write outside the timed events); arc list 2.1 GB > L2"}
 
 
@@ -201,16 +252,19 @@ def main():
         """a1 CSR build -> a2-a5 virtualize -> a6-a10 PageRank; returns per-phase events."""
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
         ev[0].record(s)
-        g = tigr.tigr_graph_from_coo(n, src_t, dst_t, None, stream=s)
+        if comm is None:
+            g = tigr.tigr_graph_from_coo(n, src_t, dst_t, None, stream=s)
+        else:  # e: each rank sorts only the arcs of its source range (arc-balanced cuts)
+            cuts = tigr.tigr_coo_source_cuts(n, src_t, dst_t, world, stream=s)
+            g = tigr.tigr_graph_from_coo_part(n, src_t, dst_t, None, src_lo=int(cuts[rank]),
+                                              src_hi=int(cuts[rank + 1]), stream=s)
         ev[1].record(s)
         vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
-        if comm is not None:
-            tigr.tigr_vgraph_partition(vg, world, rank)
         ev[2].record(s)
         _, st = tigr.tigr_run(vg, "pr", 0, opts=opts, out=out_t, return_stats=True)
         ev[3].record(s)
         vi = vg.info()
-        nv = vi["hi"] - vi["lo"]  # this rank's virtual nodes (all of them at N = 1)
+        nv = (vi["hi"] - vi["lo"], g.info()["m"])  # this rank's virtual nodes and arcs
         vg.free()
         g.free()
         return ev, st, nv
@@ -222,7 +276,7 @@ def main():
 
     deg_t = torch.bincount(src, minlength=n)
     n_out = int(torch.count_nonzero(deg_t).item())
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(local, gpu_uuid(torch, local))
     clocks.start()
     l0 = tigr.tigr_launch_count()
     step_ms, phase, relax_ms, relax_launches, nv = [], [[], [], []], 0.0, 0, 0
@@ -253,8 +307,8 @@ def main():
 
     # roofline of the dominant kernel (PR relax), live CUDA-event durations from the timed region
     relax_avg_ms = relax_ms / max(relax_launches, 1)
-    my_nv = nv
-    bytes_launch = relax_bytes_pr(m // world if world > 1 else m, my_nv, n_out // world if world > 1 else n_out)
+    my_nv, my_m = nv
+    bytes_launch = relax_bytes_pr(my_m, my_nv, n_out // world if world > 1 else n_out)
     peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(peaks_path):
         peak = json.load(open(peaks_path))["hbm_gbs"]

@@ -118,6 +118,23 @@ tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, con
                                 const uint32_t* w, int is_device_ptr, int symmetrize, void* stream,
                                 tigr_graph** out);
 
+/* Multi-GPU partitioned build: like tigr_graph_from_coo but keeps only the arcs
+ * whose source lies in [src_lo, src_hi).  The graph still spans all n nodes (others have no
+ * arcs), so a virtual split of it covers exactly this rank's virtual nodes and tigr_run with a
+ * communicator merges the replicated values with the other ranks.  Every rank must use the
+ * same full arc list (the PageRank accumulator order is derived from all arcs' targets).
+ * tigr_graph_info's m is the kept arc count.  PageRank with pr_dangling = 1 is not supported
+ * on partitioned graphs (dangling detection needs every rank's out-degrees). */
+tigr_status tigr_graph_from_coo_part(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                     const uint32_t* w, int is_device_ptr, int symmetrize, uint32_t src_lo,
+                                     uint32_t src_hi, void* stream, tigr_graph** out);
+
+/* Source-node cuts for nranks partitions with ~equal arc counts: cuts[0] = 0 <= cuts[1] <= ...
+ * <= cuts[nranks] = n (host array of nranks+1 entries); rank r builds [cuts[r], cuts[r+1]).
+ * Granularity n/16384 nodes; deterministic for the same arc list. */
+tigr_status tigr_coo_source_cuts(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                 int is_device_ptr, int symmetrize, int nranks, void* stream, uint32_t* cuts);
+
 /* Build from a CSR (row_ptr[n+1] int64, col[m], optional w[m]).  symmetric_hint=1 declares
  * the caller's graph symmetric (required for TIGR_CC).  Errors: EINVAL on a non-monotone
  * row_ptr, row_ptr[0] != 0, row_ptr[n] != m, or col >= n. */

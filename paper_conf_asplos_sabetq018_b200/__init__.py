@@ -64,6 +64,8 @@ _SIGS = {
     "tigr_run_opts_default": (None, [ctypes.POINTER(tigr_run_opts)]),
     "tigr_graph_from_coo": (_I, [_U32, _U64, _P, _P, _P, _I, _I, _P, ctypes.POINTER(_P)]),
     "tigr_graph_from_csr": (_I, [_U32, _U64, _P, _P, _P, _I, _I, _P, ctypes.POINTER(_P)]),
+    "tigr_graph_from_coo_part": (_I, [_U32, _U64, _P, _P, _P, _I, _I, _U32, _U32, _P, ctypes.POINTER(_P)]),
+    "tigr_coo_source_cuts": (_I, [_U32, _U64, _P, _P, _I, _I, _I, _P, _P]),
     "tigr_rmat_coo": (_I, [_U32, _U64, _D, _D, _D, _U64, _U64, _U32, _U32, _P, _P, _P, _P]),
     "tigr_graph_rmat": (_I, [_U32, _U64, _D, _D, _D, _U64, _U64, _U32, _U32, _I, _I, _P, ctypes.POINTER(_P)]),
     "tigr_graph_info": (_I, [_P, ctypes.POINTER(_U32), ctypes.POINTER(_U64), ctypes.POINTER(_I),
@@ -224,6 +226,29 @@ def tigr_graph_from_coo(n, src, dst, w=None, symmetrize=False, stream=None) -> G
     out = _P()
     _check(_lib.tigr_graph_from_coo(n, m, ps, pd, pw, ds, int(symmetrize), _stream_ptr(stream), ctypes.byref(out)))
     return Graph(out.value)
+
+
+def tigr_graph_from_coo_part(n, src, dst, w=None, symmetrize=False, src_lo=0, src_hi=0xFFFFFFFF,
+                             stream=None) -> Graph:
+    """Partitioned build: keep only arcs with source in [src_lo, src_hi) (multi-GPU ranks)."""
+    m = _len(src)
+    ps, ds, ks = _arr(src)
+    pd, dd, kd = _arr(dst)
+    pw, dw, kw = _arr(w)
+    out = _P()
+    _check(_lib.tigr_graph_from_coo_part(n, m, ps, pd, pw, ds, int(symmetrize), src_lo, src_hi,
+                                         _stream_ptr(stream), ctypes.byref(out)))
+    return Graph(out.value)
+
+
+def tigr_coo_source_cuts(n, src, dst, nranks, symmetrize=False, stream=None):
+    """Source-node cuts (nranks+1 entries) balancing arc counts across ranks."""
+    ps, ds, ks = _arr(src)
+    pd, dd, kd = _arr(dst)
+    cuts = np.empty(nranks + 1, dtype=np.uint32)
+    _check(_lib.tigr_coo_source_cuts(n, _len(src), ps, pd, ds, int(symmetrize), nranks, _stream_ptr(stream),
+                                     cuts.ctypes.data))
+    return cuts
 
 
 def tigr_graph_from_csr(n, row_ptr, col, w=None, symmetric_hint=False, stream=None) -> Graph:

@@ -157,6 +157,11 @@ tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double
                        cudaStream_t s);
 tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
                                   const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out);
+tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                       const uint32_t* w, int symmetrize, uint32_t src_lo, uint32_t src_hi,
+                                       cudaStream_t s, tigr_graph** out);
+tigr_status coo_source_cuts(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, int symmetrize,
+                            int nranks, cudaStream_t s, uint32_t* cuts);
 tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col, const uint32_t* w,
                                   int symmetric_hint, cudaStream_t s, tigr_graph** out);
 tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w, cudaStream_t s);
@@ -235,6 +240,40 @@ tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, con
     TIGR_CK(cudaStreamSynchronize(s));
     trace(s, "coo: done");
     return TIGR_OK;
+}
+
+tigr_status tigr_graph_from_coo_part(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                     const uint32_t* w, int is_device_ptr, int symmetrize, uint32_t src_lo,
+                                     uint32_t src_hi, void* stream, tigr_graph** out) {
+    if (!out) return fail(TIGR_EINVAL, "graph_from_coo_part: out is NULL");
+    *out = nullptr;
+    if (n == 0) return fail(TIGR_EINVAL, "graph_from_coo_part: n == 0");
+    if (n > 0xFFFFFFFEu) return fail(TIGR_ERANGE, "graph_from_coo_part: n > 0xFFFFFFFE");
+    if (m && (!src || !dst)) return fail(TIGR_EINVAL, "graph_from_coo_part: src/dst NULL");
+    if (src_lo > src_hi) return fail(TIGR_EINVAL, "graph_from_coo_part: src_lo > src_hi");
+    TIGR_TRY(need_device());
+    cudaStream_t s = (cudaStream_t)stream;
+    TmpBuf ts, td, tw;
+    const uint32_t *ds = nullptr, *dd = nullptr, *dw = nullptr;
+    TIGR_TRY(stage(src, m, is_device_ptr, s, ts, &ds));
+    TIGR_TRY(stage(dst, m, is_device_ptr, s, td, &dd));
+    TIGR_TRY(stage(w, m, is_device_ptr, s, tw, &dw));
+    TIGR_TRY(graph_from_coo_part_device(n, m, ds, dd, dw, symmetrize, src_lo, src_hi, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_coo_source_cuts(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, int is_device_ptr,
+                                 int symmetrize, int nranks, void* stream, uint32_t* cuts) {
+    if (!cuts || nranks < 1 || n == 0) return fail(TIGR_EINVAL, "coo_source_cuts: bad argument");
+    if (m && (!src || !dst)) return fail(TIGR_EINVAL, "coo_source_cuts: src/dst NULL");
+    TIGR_TRY(need_device());
+    cudaStream_t s = (cudaStream_t)stream;
+    TmpBuf ts, td;
+    const uint32_t *ds = nullptr, *dd = nullptr;
+    TIGR_TRY(stage(src, m, is_device_ptr, s, ts, &ds));
+    TIGR_TRY(stage(dst, m, is_device_ptr, s, td, &dd));
+    return coo_source_cuts(n, m, ds, dd, symmetrize, nranks, s, cuts);
 }
 
 tigr_status tigr_graph_from_csr(uint32_t n, uint64_t m, const int64_t* row_ptr, const uint32_t* col, const uint32_t* w,

@@ -16,7 +16,7 @@ tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double
                        uint64_t seed, uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src,
                        uint32_t* dst, uint32_t* w, cudaStream_t s);
 tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
-                             int symmetrize, cudaStream_t s, tigr_graph* g);
+                             int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi);
 
 namespace {
 
@@ -202,8 +202,11 @@ tigr_status layout_from_degrees(tigr_graph* g, cudaStream_t s) {
 
 }  // namespace
 
-tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
-                                  const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out) {
+// src_lo/src_hi: keep only the arcs whose source lies in [src_lo, src_hi) (multi-GPU partitioned
+// builds); the in-degree sketch and the id validation still cover every arc
+tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                       const uint32_t* w, int symmetrize, uint32_t src_lo, uint32_t src_hi,
+                                       cudaStream_t s, tigr_graph** out) {
     const uint64_t arcs = symmetrize ? 2 * m : m;
     if (arcs >= (1ull << 32) * 3) return fail(TIGR_ERANGE, "graph: too many arcs");
     tigr_graph* g = new tigr_graph();
@@ -211,7 +214,9 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
     g->m = arcs;
     g->weighted = w != nullptr;
     g->symmetric = symmetrize != 0;
-    tigr_status st = csr_build_sorted(n, m, src, dst, w, symmetrize, s, g);
+    tigr_status st = csr_build_sorted(n, m, src, dst, w, symmetrize, s, g, src_lo, src_hi);
+    g->part_lo = src_lo;
+    g->part_hi = src_hi < n ? src_hi : n;
     if (st == TIGR_OK) {
         k_pad<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), g->cptr.as<uint32_t>(), n, g->col.as<uint32_t>(),
                                               g->wt.as<uint32_t>());
@@ -222,6 +227,11 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
     if (st != TIGR_OK) { delete g; return st; }
     *out = g;
     return TIGR_OK;
+}
+
+tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
+                                  const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out) {
+    return graph_from_coo_part_device(n, m, src, dst, w, symmetrize, 0, 0xFFFFFFFFu, s, out);
 }
 
 tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col,
@@ -293,6 +303,8 @@ tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_gra
                                    g->weighted ? w.as<uint32_t>() : nullptr, 0, s, &t));
     t->symmetric = g->symmetric;
     t->transposed = !g->transposed;
+    t->part_lo = g->part_lo;
+    t->part_hi = g->part_hi;
     tigr_status st = t->src_deg.alloc(sizeof(uint32_t) * (g->n ? g->n : 1), s);
     if (st == TIGR_OK && g->n) {
         cudaError_t e = cudaMemcpyAsync(t->src_deg.p, g->deg.p, sizeof(uint32_t) * g->n, cudaMemcpyDeviceToDevice, s);

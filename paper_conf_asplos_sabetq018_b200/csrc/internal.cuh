@@ -109,6 +109,8 @@ struct tigr_graph {
     // transposed graphs (tigr_graph_transpose): arcs reversed; src_deg = out-degrees of the
     // original graph (PageRank pull divides by them)
     bool transposed = false;
+    // partitioned builds (tigr_graph_from_coo_part): only sources in [part_lo, part_hi) have arcs
+    uint32_t part_lo = 0, part_hi = 0xFFFFFFFFu;
     tigr::DevBuf src_deg;    // uint32[n] (transposed graphs only)
 };
 

@@ -235,6 +235,8 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     // a transposed graph runs pull-based PageRank (pr.cu, NEXT-1); divide by the original
     // graph's out-degrees, which the transpose carries
     const bool pull = vg->g->transposed;
+    if (o.pr_dangling && (vg->g->part_lo != 0 || vg->g->part_hi < n))
+        return fail(TIGR_EUNSUPPORTED, "pr_dangling = 1 needs every out-degree: not on a partitioned graph");
     const uint32_t* out_deg = pull ? vg->g->src_deg.as<uint32_t>() : vg->g->deg.as<uint32_t>();
     const bool use_cid = !pull && !o.collect_stats && vg->vec && pr_cid_enabled();
     PrCidPlan cp;

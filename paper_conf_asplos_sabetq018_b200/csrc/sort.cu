@@ -11,8 +11,10 @@
 // hottest vertex owns 0.14% of all arcs at scale 24) costs nothing.  Degrees come from the
 // run boundaries of the sorted keys; a final kernel places each arc into the 16-byte-aligned,
 // padded segment of its source.
+#include <algorithm>
 #include <cstdlib>
 #include <utility>
+#include <vector>
 
 #include "internal.cuh"
 
@@ -52,28 +54,35 @@ __device__ __forceinline__ void coo_item(const uint32_t* __restrict__ src, const
 __global__ void k_coo_scan(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
                            uint64_t M, int passes, int bits, unsigned long long* __restrict__ hist,
                            uint32_t* __restrict__ maxid, uint32_t n, uint8_t* __restrict__ in_flag,
-                           uint32_t* __restrict__ in_sample) {
+                           uint32_t* __restrict__ in_sample, uint32_t klo, uint32_t khi,
+                           unsigned long long* __restrict__ n_local) {
     __shared__ uint32_t h[4][kMaxRadix];
     for (int i = threadIdx.x; i < 4 * kMaxRadix; i += blockDim.x) (&h[0][0])[i] = 0;
     __syncthreads();
     const uint32_t mask = (1u << bits) - 1;
-    uint32_t mx = 0;
+    uint32_t mx = 0, local = 0;
     for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < M; e += (uint64_t)gridDim.x * blockDim.x) {
         const bool rev = e >= m;
         const uint64_t f = rev ? e - m : e;
         const uint32_t s = src[f], d = dst[f];
         const uint32_t k = rev ? d : s, t = rev ? s : d;
         mx = max(mx, max(s, d));
-        if (k < n)
+        if (k < n && k >= klo && k < khi) {  // this build's source range (partitioned graphs)
+            ++local;
             for (int p = 0; p < passes; ++p) atomicAdd(&h[p][(k >> (p * bits)) & mask], 1u);
+        }
         if (in_flag && t < n) {
             if (!in_flag[t]) in_flag[t] = 1;
             if ((e & 15) == 0) atomicAdd(in_sample + t, 1u);
         }
     }
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    for (int o = 16; o > 0; o >>= 1) {
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        local += __shfl_xor_sync(0xffffffffu, local, o);
+    }
     if ((threadIdx.x & 31) == 0 && mx) atomicMax(maxid, mx);
+    if ((threadIdx.x & 31) == 0 && local) atomicAdd(n_local, (unsigned long long)local);
     __syncthreads();
     for (int i = threadIdx.x; i < passes * kMaxRadix; i += blockDim.x) {
         const uint32_t c = (&h[0][0])[i];
@@ -105,14 +114,15 @@ __device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
 // One pass of the stable LSD radix sort over a tile of 4096 arcs.  Values are staged into
 // shared memory with cp.async as soon as the tile is known (no registers held across the
 // ranking / look-back); keys stay in registers; digits are recomputed from the keys.
-template <bool W, bool FIRST, int SI>
+template <bool W, bool FIRST, int SI, bool FILT>
 __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_onesweep(const uint32_t* __restrict__ kin,
                                                   const typename ValT<W>::T* __restrict__ vin,
                                                   const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst,
                                                   const uint32_t* __restrict__ w, uint64_t m, uint64_t M, int shift,
                                                   int bits, const uint64_t* __restrict__ digit_base,
                                                   uint64_t* status, uint32_t* tile_counter, uint64_t epoch,
-                                                  uint32_t* __restrict__ kout, typename ValT<W>::T* __restrict__ vout) {
+                                                  uint32_t* __restrict__ kout, typename ValT<W>::T* __restrict__ vout,
+                                                  uint32_t klo, uint32_t khi) {
     typedef typename ValT<W>::T VT;
     extern __shared__ __align__(16) unsigned char smem[];
     VT* s_vin = reinterpret_cast<VT*>(smem);                                   // tile values, input order
@@ -134,8 +144,14 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
     const uint32_t mask = (uint32_t)radix - 1;
     const uint32_t cnt = (M - base < (uint64_t)(kST * SI)) ? (uint32_t)(M - base) : (uint32_t)(kST * SI);
 
-    // values -> shared memory (asynchronous, coalesced), keys -> registers
+    // values -> shared memory (asynchronous, coalesced), keys -> registers; in the first pass
+    // arcs whose source lies outside [klo, khi) are dropped (partitioned builds)
     uint32_t key[SI];
+    uint32_t valid = 0;  // FILT: bit r = item r of this thread passed the filter
+    auto keep = [&](int r) -> bool {
+        if constexpr (FILT) return (valid >> r) & 1u;
+        else return (uint32_t)(wp * (SI * 32) + r * 32 + lane) < cnt;
+    };
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
         const uint32_t li = wp * (SI * 32) + r * 32 + lane;
@@ -146,9 +162,12 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
                 const bool rev = idx >= m;
                 const uint64_t f = rev ? idx - m : idx;
                 key[r] = rev ? dst[f] : src[f];
-                uint32_t* sv = reinterpret_cast<uint32_t*>(&s_vin[li]);
-                cp_async4(sv, rev ? src + f : dst + f);
-                if constexpr (W) cp_async4(sv + 1, w + f);
+                if (!FILT || (key[r] >= klo && key[r] < khi)) {
+                    if constexpr (FILT) valid |= 1u << r;
+                    uint32_t* sv = reinterpret_cast<uint32_t*>(&s_vin[li]);
+                    cp_async4(sv, rev ? src + f : dst + f);
+                    if constexpr (W) cp_async4(sv + 1, w + f);
+                }
             } else {
                 key[r] = kin[idx];
                 if constexpr (W) {
@@ -172,8 +191,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
     uint32_t rank[SI / 2];  // two 16-bit ranks per register
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
-        const uint32_t li = wp * (SI * 32) + r * 32 + lane;
-        const uint32_t d = li < cnt ? (key[r] >> shift) & mask : (uint32_t)radix;
+        const uint32_t d = keep(r) ? (key[r] >> shift) & mask : (uint32_t)radix;
         peers[r] = __match_any_sync(0xffffffffu, d);
         uint32_t got = 0;
         if ((peers[r] & lt) == 0) got = atomicAdd(&s_wcnt[wp][d], (uint32_t)__popc(peers[r]));
@@ -213,6 +231,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         uint32_t wofs = 0;
         for (int wi = 0; wi < wp; ++wi) wofs += s_wsum[wi];
         s_dstart[t] = wofs + v - tile_cnt;
+        if (FILT && t == kST - 1) s_dstart[kMaxRadix] = wofs + v;  // the tile's kept items
     }
     // decoupled look-back for this digit
     if (t < radix) {
@@ -236,7 +255,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
         const uint32_t li = wp * (SI * 32) + r * 32 + lane;
-        if (li < cnt) {
+        if (keep(r)) {
             const uint32_t d = (key[r] >> shift) & mask;
             const uint32_t lp = s_dstart[d] + s_wcnt[wp][d] + ((rank[r >> 1] >> ((r & 1) * 16)) & 0xFFFFu);
             s_key[lp] = key[r];
@@ -244,10 +263,11 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         }
     }
     __syncthreads();
+    const uint32_t nvalid = FILT ? s_dstart[kMaxRadix] : cnt;
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
         const uint32_t i = r * kST + t;
-        if (i < cnt) {
+        if (i < nvalid) {
             const uint32_t k = s_key[i];
             const uint32_t d = (k >> shift) & mask;
             const uint64_t pos = s_gofs[d] + (i - s_dstart[d]);
@@ -299,7 +319,8 @@ unsigned sort_grid(uint64_t items) {
 template <bool W>
 tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* w, uint64_t m, uint64_t M,
                       uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out, bool validate,
-                      uint8_t* in_flag = nullptr, uint32_t* in_sample = nullptr) {
+                      uint8_t* in_flag = nullptr, uint32_t* in_sample = nullptr, uint32_t klo = 0,
+                      uint32_t khi = 0xFFFFFFFFu, uint64_t* M_out = nullptr) {
     typedef typename ValT<W>::T VT;
     int key_bits = 0;
     while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
@@ -310,7 +331,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     const uint64_t tile_items = (uint64_t)kST * SI;
     const uint64_t tiles = (M + tile_items - 1) / tile_items;
 
-    TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid;
+    TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid, nloc;
     trace(s, "sort: enter");
     for (int i = 0; i < 2; ++i) {
         TIGR_TRY(kb[i].alloc(sizeof(uint32_t) * (M ? M : 1), s));
@@ -326,18 +347,27 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     TIGR_CK(cudaMemsetAsync(counters.p, 0, sizeof(uint32_t) * 4, s));
     TIGR_TRY(maxid.alloc(sizeof(uint32_t), s));
     TIGR_CK(cudaMemsetAsync(maxid.p, 0, sizeof(uint32_t), s));
+    TIGR_TRY(nloc.alloc(sizeof(unsigned long long), s));
+    TIGR_CK(cudaMemsetAsync(nloc.p, 0, sizeof(unsigned long long), s));
+    const bool filtered = klo != 0 || khi < n;
     trace(s, "sort: alloc+memset");
     if (M) {
         k_coo_scan<<<sort_grid(M), kBlock, 0, s>>>(src, dst, m, M, passes, bits, hist.as<unsigned long long>(),
-                                                    maxid.as<uint32_t>(), n, in_flag, in_sample);
+                                                    maxid.as<uint32_t>(), n, in_flag, in_sample, klo, khi,
+                                                    nloc.as<unsigned long long>());
         TIGR_CKL("coo scan");
     }
-    if (M && validate) {
+    uint64_t Mloc = M;  // items that survive the source-range filter
+    if (M && (validate || filtered)) {
         uint32_t hmax = 0;
+        unsigned long long hl = 0;
         TIGR_CK(cudaMemcpyAsync(&hmax, maxid.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+        TIGR_CK(cudaMemcpyAsync(&hl, nloc.p, sizeof(unsigned long long), cudaMemcpyDeviceToHost, s));
         TIGR_CK(cudaStreamSynchronize(s));
-        if (hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
+        if (validate && hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
+        Mloc = hl;
     }
+    if (M_out) *M_out = Mloc;
     k_digit_base<<<1, kMaxRadix, 0, s>>>(hist.as<unsigned long long>(), passes, dbase.as<uint64_t>());
     TIGR_CKL("digit base");
     trace(s, "sort: digit histograms");
@@ -345,19 +375,25 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     int cur = 0;
     for (int p = 0; p < passes && M; ++p) {
         void (*kern)(const uint32_t*, const VT*, const uint32_t*, const uint32_t*, const uint32_t*, uint64_t,
-                     uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*, uint64_t, uint32_t*, VT*);
+                     uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*, uint64_t, uint32_t*, VT*, uint32_t,
+                     uint32_t);
         switch (SI) {
-            case 12: kern = p == 0 ? &k_onesweep<W, true, 12> : &k_onesweep<W, false, 12>; break;
-            case 20: kern = p == 0 ? &k_onesweep<W, true, 20> : &k_onesweep<W, false, 20>; break;
-            case 24: kern = p == 0 ? &k_onesweep<W, true, 24> : &k_onesweep<W, false, 24>; break;
-            default: kern = p == 0 ? &k_onesweep<W, true, 16> : &k_onesweep<W, false, 16>; break;
+            case 12: kern = p == 0 ? &k_onesweep<W, true, 12, false> : &k_onesweep<W, false, 12, false>; break;
+            case 20: kern = p == 0 ? &k_onesweep<W, true, 20, false> : &k_onesweep<W, false, 20, false>; break;
+            case 24: kern = p == 0 ? &k_onesweep<W, true, 24, false> : &k_onesweep<W, false, 24, false>; break;
+            default: kern = p == 0 ? &k_onesweep<W, true, 16, false> : &k_onesweep<W, false, 16, false>; break;
         }
+        // partitioned builds: the first pass drops the arcs outside [klo, khi)
+        if (p == 0 && filtered) kern = &k_onesweep<W, true, 16, true>;
         TIGR_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         const int out = (p == 0) ? 0 : 1 - cur;
-        kern<<<(unsigned)tiles, kST, smem, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), src, dst, w, m, M, p * bits,
-                                                bits, dbase.as<uint64_t>() + p * kMaxRadix, status.as<uint64_t>(),
-                                                counters.as<uint32_t>() + p, (uint64_t)(p + 1), kb[out].as<uint32_t>(),
-                                                vb[out].as<VT>());
+        const uint64_t Mp = (p == 0) ? M : Mloc;  // the first pass reads (and filters) the full list
+        const uint64_t tp = (Mp + tile_items - 1) / tile_items;
+        if (tp == 0) break;
+        kern<<<(unsigned)tp, kST, smem, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), src, dst, w, m, Mp, p * bits,
+                                             bits, dbase.as<uint64_t>() + p * kMaxRadix, status.as<uint64_t>(),
+                                             counters.as<uint32_t>() + p, (uint64_t)(p + 1), kb[out].as<uint32_t>(),
+                                             vb[out].as<VT>(), klo, khi);
         TIGR_CKL("onesweep");
         trace(s, "sort: onesweep pass");
         cur = out;
@@ -371,18 +407,20 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
 
 template <bool W>
 tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
-                         int symmetrize, cudaStream_t s, tigr_graph* g) {
+                         int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi) {
     typedef typename ValT<W>::T VT;
-    const uint64_t M = symmetrize ? 2 * m : m;
+    const uint64_t Mall = symmetrize ? 2 * m : m;
+    uint64_t M = Mall;
     TmpBuf keys, vals;
     keys.s = vals.s = s;
     TIGR_TRY(g->in_flag.alloc(n ? n : 1, s));
     TIGR_TRY(g->in_sample.alloc(sizeof(uint32_t) * (n ? n : 1), s));
     TIGR_CK(cudaMemsetAsync(g->in_flag.p, 0, n, s));
     TIGR_CK(cudaMemsetAsync(g->in_sample.p, 0, sizeof(uint32_t) * n, s));
-    TIGR_TRY(sort_arcs<W>(src, dst, w, m, M, n, s, keys, vals, true, g->in_flag.as<uint8_t>(),
-                          g->in_sample.as<uint32_t>()));
+    TIGR_TRY(sort_arcs<W>(src, dst, w, m, Mall, n, s, keys, vals, true, g->in_flag.as<uint8_t>(),
+                          g->in_sample.as<uint32_t>(), klo, khi, &M));
     g->has_in_sketch = true;
+    g->m = M;  // arcs of this build's source range (all arcs unless partitioned)
     // degrees from runs
     TmpBuf st, en;
     TIGR_TRY(st.alloc(sizeof(uint32_t) * n, s));
@@ -418,7 +456,60 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     return TIGR_OK;
 }
 
+constexpr int kCutBuckets = 16384;
+
+// histogram of the arc sources over kCutBuckets contiguous vertex ranges (per-block shared copy)
+__global__ void k_src_hist(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m, uint64_t M,
+                           int shift, unsigned long long* __restrict__ hist) {
+    extern __shared__ uint32_t sh[];
+    for (int i = threadIdx.x; i < kCutBuckets; i += blockDim.x) sh[i] = 0;
+    __syncthreads();
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < M; e += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t k = e < m ? src[e] : dst[e - m];
+        atomicAdd(&sh[min((uint32_t)(k >> shift), (uint32_t)kCutBuckets - 1)], 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < kCutBuckets; i += blockDim.x)
+        if (sh[i]) atomicAdd(&hist[i], (unsigned long long)sh[i]);
+}
+
 }  // namespace
+
+// Source-vertex cuts for nranks partitions with ~equal arc counts, at a granularity of
+// n / 16384 vertices (deterministic: every rank computes the same cuts from the same arcs).
+tigr_status coo_source_cuts(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, int symmetrize,
+                            int nranks, cudaStream_t s, uint32_t* cuts) {
+    const uint64_t M = symmetrize ? 2 * m : m;
+    int key_bits = 0;
+    while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
+    const int shift = key_bits > 14 ? key_bits - 14 : 0;
+    TmpBuf hist;
+    TIGR_TRY(hist.alloc(sizeof(unsigned long long) * kCutBuckets, s));
+    TIGR_CK(cudaMemsetAsync(hist.p, 0, sizeof(unsigned long long) * kCutBuckets, s));
+    if (M) {
+        TIGR_CK(cudaFuncSetAttribute(k_src_hist, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)(sizeof(uint32_t) * kCutBuckets)));
+        k_src_hist<<<sort_grid(M), kBlock, sizeof(uint32_t) * kCutBuckets, s>>>(src, dst, m, M, shift,
+                                                                               hist.as<unsigned long long>());
+        TIGR_CKL("source histogram");
+    }
+    std::vector<unsigned long long> h(kCutBuckets);
+    TIGR_CK(cudaMemcpyAsync(h.data(), hist.p, sizeof(unsigned long long) * kCutBuckets, cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    cuts[0] = 0;
+    cuts[nranks] = n;
+    unsigned long long acc = 0;
+    int b = 0;
+    for (int r = 1; r < nranks; ++r) {
+        const unsigned long long target = (unsigned long long)((unsigned __int128)M * (unsigned)r / (unsigned)nranks);
+        while (b < kCutBuckets && acc + h[b] <= target) acc += h[b++];
+        // bucket b straddles the target: cut at the nearer of its two boundaries
+        uint64_t v = (uint64_t)b << shift;
+        if (b < kCutBuckets && target - acc > acc + h[b] - target) v = (uint64_t)(b + 1) << shift;
+        cuts[r] = (uint32_t)std::min<uint64_t>(std::max<uint64_t>(v, cuts[r - 1]), n);
+    }
+    return TIGR_OK;
+}
 
 // Stable sort of (key, value) u32 pairs by key (keys < key_limit); results owned by the TmpBufs.
 tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t count, uint32_t key_limit,
@@ -429,9 +520,9 @@ tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t 
 
 // Stable device CSR build from an arc list (device pointers).  Caller validated ids < n.
 tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
-                             int symmetrize, cudaStream_t s, tigr_graph* g) {
-    if (w) return build_sorted<true>(n, m, src, dst, w, symmetrize, s, g);
-    return build_sorted<false>(n, m, src, dst, w, symmetrize, s, g);
+                             int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi) {
+    if (w) return build_sorted<true>(n, m, src, dst, w, symmetrize, s, g, klo, khi);
+    return build_sorted<false>(n, m, src, dst, w, symmetrize, s, g, klo, khi);
 }
 
 }  // namespace tigr

@@ -411,3 +411,64 @@ def test_udt_matches_oracle(tigr, K):
                           oracle.bfs(oracle.csr_build(rec.n, src, dst), 0))
     with pytest.raises(tigr.TigrError):
         tigr.tigr_graph_udt(g, 1, 0)
+
+
+# ------------------------------------------------------------------------------------ e: partitioned builds
+@pytest.mark.parametrize("sym", [False, True])
+def test_partitioned_build_union(tigr, sym):
+    """Rank r's source-filtered build holds exactly the rows [cuts[r], cuts[r+1]) of the full
+    CSR (same stable order); the cuts balance arcs to within one histogram bucket."""
+    rec = graphgen.recipe("cfg2")
+    n = rec.n
+    src, dst, w = graphgen.rmat(n, rec.m // 4, rec.a, rec.b, rec.c, rec.seed, rec.wseed)
+    S, D, W = oracle.symmetrize(src, dst, w) if sym else (src, dst, w)
+    o = oracle.csr_build(n, S, D, W)
+    deg = np.diff(o.row_ptr)
+    M = len(S)
+    for P in (1, 2, 3, 8):
+        cuts = tigr.tigr_coo_source_cuts(n, src, dst, P, symmetrize=sym)
+        assert cuts[0] == 0 and cuts[-1] == n and np.all(np.diff(cuts.astype(np.int64)) >= 0)
+        width = max(1, n // 16384)
+        assert all(c % width == 0 for c in cuts[:-1])
+        bucket_max = int(np.add.reduceat(deg, np.arange(0, n, width)).max())
+        for r in range(1, P):
+            assert abs(int(o.row_ptr[cuts[r]]) - r * M // P) <= bucket_max
+    cuts = tigr.tigr_coo_source_cuts(n, src, dst, 3, symmetrize=sym)
+    total = 0
+    for r in range(3):
+        lo, hi = int(cuts[r]), int(cuts[r + 1])
+        gp = tigr.tigr_graph_from_coo_part(n, src, dst, w, symmetrize=sym, src_lo=lo, src_hi=hi)
+        rp, col, wt = tigr.tigr_graph_export_csr(gp)
+        pd = np.diff(rp)
+        assert np.array_equal(pd[lo:hi], deg[lo:hi]) and not pd[:lo].any() and not pd[hi:].any()
+        a, b = int(o.row_ptr[lo]), int(o.row_ptr[hi])
+        assert np.array_equal(col, o.col[a:b]) and np.array_equal(wt, o.wt[a:b])
+        assert gp.info()["m"] == b - a
+        total += b - a
+    assert total == M
+    # empty and full ranges
+    ge = tigr.tigr_graph_from_coo_part(n, src, dst, w, src_lo=5, src_hi=5)
+    assert ge.info()["m"] == 0
+    gf = tigr.tigr_graph_from_coo_part(n, src, dst, w, src_lo=0, src_hi=n)
+    assert np.array_equal(tigr.tigr_graph_export_csr(gf)[1], oracle.csr_build(n, src, dst, w).col)
+
+
+def test_partitioned_graph_runs(tigr):
+    """A partition is a graph of its own: without a communicator every algorithm reaches the
+    oracle's result on the filtered arc list; PageRank's dangling mass is refused there."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    cuts = tigr.tigr_coo_source_cuts(rec.n, src, dst, 2)
+    for r in range(2):
+        lo, hi = int(cuts[r]), int(cuts[r + 1])
+        keep = (src >= lo) & (src < hi)
+        o = oracle.csr_build(rec.n, src[keep], dst[keep], w[keep])
+        gp = tigr.tigr_graph_from_coo_part(rec.n, src, dst, w, src_lo=lo, src_hi=hi)
+        for K, layout in ((8, "strided"), (3, "consecutive")):
+            vg = tigr.tigr_virtualize(gp, K, layout)
+            assert np.array_equal(tigr.tigr_run(vg, "bfs", 0), oracle.bfs(o, 0))
+            assert np.array_equal(tigr.tigr_run(vg, "sssp", 0), oracle.sssp(o, 0))
+            assert np.array_equal(tigr.tigr_run(vg, "sswp", 0), oracle.sswp(o, 0))
+            assert np.abs(tigr.tigr_run(vg, "pr") - oracle.pagerank(o, 20)).max() <= 1e-6
+            with pytest.raises(tigr.TigrError):
+                tigr.tigr_run(vg, "pr", pr_dangling=1)
