@@ -67,9 +67,16 @@ typedef enum {
 
 /* Worklist policy (§5; Table 8). */
 typedef enum {
-    TIGR_FRONTIER_AUTO = 0,    /* = DENSE in this version */
-    TIGR_FRONTIER_DENSE = 1,   /* per-node active flags; inactive vnodes exit early */
-    TIGR_FRONTIER_NONE = 2     /* every vnode every iteration (Table 8 "without worklist") */
+    TIGR_FRONTIER_AUTO = 0,    /* per iteration, on the device: QUEUE while the active nodes own
+                                  fewer than 1/2 of the virtual nodes, else DENSE
+                                  (16-byte-chunk layouts, i.e. 4 | K; otherwise DENSE) */
+    TIGR_FRONTIER_DENSE = 1,   /* per-node active flags; every stored virtual node tests its node's
+                                  flag, inactive ones exit early */
+    TIGR_FRONTIER_NONE = 2,    /* every vnode every iteration (Table 8 "without worklist") */
+    TIGR_FRONTIER_QUEUE = 3    /* queue of active nodes, virtual nodes derived on the fly from the
+                                  queue and the degree bound ("dynamic mapping reasoning", §4.1
+                                  L962-972): the stored virtual node array is never read.
+                                  Needs 4 | K (else EUNSUPPORTED). */
 } tigr_frontier;
 
 typedef struct tigr_graph tigr_graph;   /* device CSR; owns its buffers */
@@ -102,6 +109,8 @@ typedef struct {
     double ms_total;          /* device time of the whole run (init -> values on device) */
     double ms_relax;          /* device time of the relax launches (time_kernels) */
     double ms_exchange;       /* device time of the multi-GPU exchanges (time_kernels) */
+    uint32_t queue_iterations;/* iterations whose relax ran from the active-node queue (FRONTIER_AUTO/QUEUE) */
+    uint32_t reserved;
 } tigr_stats;
 
 /* Fill *opts with the defaults above. */

@@ -29,7 +29,7 @@ TIGR_OK, TIGR_EINVAL, TIGR_ENOMEM, TIGR_ECUDA, TIGR_ENCCL, TIGR_ERANGE, TIGR_ENO
     0, -1, -2, -3, -4, -5, -6, -7
 TIGR_BFS, TIGR_SSSP, TIGR_CC, TIGR_SSWP, TIGR_PR = 0, 1, 2, 3, 4
 TIGR_LAYOUT_CONSECUTIVE, TIGR_LAYOUT_STRIDED = 0, 1
-TIGR_FRONTIER_AUTO, TIGR_FRONTIER_DENSE, TIGR_FRONTIER_NONE = 0, 1, 2
+TIGR_FRONTIER_AUTO, TIGR_FRONTIER_DENSE, TIGR_FRONTIER_NONE, TIGR_FRONTIER_QUEUE = 0, 1, 2, 3
 ALGOS = {"bfs": TIGR_BFS, "sssp": TIGR_SSSP, "cc": TIGR_CC, "sswp": TIGR_SSWP, "pr": TIGR_PR}
 LAYOUTS = {"consecutive": TIGR_LAYOUT_CONSECUTIVE, "strided": TIGR_LAYOUT_STRIDED}
 INF = 0xFFFFFFFF
@@ -53,7 +53,7 @@ class tigr_stats(ctypes.Structure):
     _fields_ = [("iterations", ctypes.c_uint32), ("relax_launches", ctypes.c_uint32),
                 ("edges_processed", ctypes.c_uint64), ("updates", ctypes.c_uint64),
                 ("active_vnodes", ctypes.c_uint64), ("ms_total", ctypes.c_double), ("ms_relax", ctypes.c_double),
-                ("ms_exchange", ctypes.c_double)]
+                ("ms_exchange", ctypes.c_double), ("queue_iterations", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -1,0 +1,353 @@
+// frontier.cu -- queue-driven frontier relax with dynamic virtual-node mapping
+// (§8(f) NEXT-3 "dynamic mapping reasoning").
+//
+// The paper's worklist (§5) keeps the nodes whose value changed; its "dynamic
+// mapping reasoning" (§4.1) derives a node's virtual nodes from the degree bound at
+// run time instead of storing the virtual node array ("before processing node v2, a
+// reasoning runtime finds its degree is 6, which is greater than K, hence splits it into two
+// virtual nodes (ceil(6/3))").  Here both meet:
+//
+//   k_compact  after each iteration, the nodes stamped active for the next iteration that own
+//              virtual nodes in this rank's range are appended to a queue {node, offset}, where
+//              offset is the exclusive prefix of the family sizes m_v = ceil(d_v/K) in queue
+//              order (one 64-bit atomic per 2048-node tile packs entry and vnode counts, so
+//              offsets increase with the entry index).
+//   k_relax_fq the next relax covers the queue's virtual nodes t in [0, total): a warp takes 32
+//              consecutive t per round, finds the queue entry of its first t with a 32-ary
+//              search over the offsets (ballot per step), and maps every lane to its entry with
+//              one OR-reduction of entry-start bits (entries own >= 1 vnode, so 32 entries
+//              always cover 32 vnodes).  Lane t then is virtual node j = t - offset of node v,
+//              and walks the same <= K arcs, in the same strided (Fig. 12) or consecutive
+//              (Fig. 10) order, as virtual node vnode_ptr[v] + j of the stored array would.
+//              No vn_phys read at all: the mapping is reasoned from the queue and the node
+//              record.
+//   When the queue holds many virtual nodes (>= 1/div of this rank's), the same kernel
+//   instead sweeps the stored virtual node array with the stamp test (the dense frontier of
+//   relax.cu): per-iteration cost then tracks the active work in sparse iterations and the
+//   streaming rate in dense ones.  The choice is made on the device from the queue size, so
+//   the whole loop stays one CUDA graph launch.
+//
+// The relax itself is Alg. 2/3 unchanged: x = value[v]; for each arc alt = f(x, w); if
+// better(alt, value[nbr]) then atomic{Min,Max} and stamp nbr for the next iteration.
+#include <algorithm>
+
+#include "devutil.cuh"
+#include "internal.cuh"
+#include "relax.cuh"
+#include "vgraph.cuh"
+
+namespace tigr {
+
+namespace {
+
+constexpr int kFqThreads = 256;
+constexpr int kCompactPer = 8;  // nodes per thread in k_compact
+constexpr uint32_t kFull = 0xffffffffu;
+
+// largest k in [0, qn) with qo[k] <= t (qo increasing, qo[0] == 0 <= t): 32-ary search, one
+// ballot per step
+__device__ __forceinline__ uint32_t warp_search(const uint32_t* __restrict__ qo, uint32_t qn, uint32_t t, int lane) {
+    uint32_t lo = 0, hi = qn;
+    while (hi - lo > 32) {
+        const uint32_t step = (hi - lo + 31) / 32;
+        const uint32_t idx = lo + (uint32_t)lane * step;
+        const bool p = idx < hi && __ldg(qo + idx) <= t;
+        const uint32_t b = __ballot_sync(kFull, p);
+        const uint32_t L = 31u - __clz(b);  // lane 0 always holds (qo[lo] <= t)
+        lo += L * step;
+        hi = min(hi, lo + step);
+    }
+    const uint32_t idx = lo + (uint32_t)lane;
+    const uint32_t b = __ballot_sync(kFull, idx < hi && __ldg(qo + idx) <= t);
+    return lo + (31u - __clz(b));
+}
+
+// map lanes of round start tr (vnodes tr + lane) to queue entries, starting from a window
+// whose first entry starts at or before tr.  Returns the lane's (node, vnode index j) and the
+// entry index the next round may start from.
+__device__ __forceinline__ void map_round(const uint32_t* __restrict__ qv, const uint32_t* __restrict__ qo,
+                                          uint32_t qn, uint32_t& k, uint32_t tr, int lane, uint32_t& v,
+                                          uint32_t& j) {
+    uint32_t idx = k + (uint32_t)lane;
+    uint32_t off = idx < qn ? __ldg(qo + idx) : kInf;
+    // entries starting at or before tr form a prefix of the window; its last one owns tr.
+    // Rebase the window there, so that its 32 entries (>= 1 vnode each) cover tr .. tr + 31.
+    const uint32_t le = __ballot_sync(kFull, off <= tr);
+    const int first = 31 - __clz(le);  // le != 0: the window's first entry starts at or before tr
+    if (first > 0) {                   // warp-uniform
+        k += (uint32_t)first;
+        idx = k + (uint32_t)lane;
+        off = idx < qn ? __ldg(qo + idx) : kInf;
+    }
+    const uint32_t node = idx < qn ? __ldg(qv + idx) : kPad;
+    uint32_t bit = 0;
+    if (lane == 0) bit = 1u;
+    else if (off < tr + 32u) bit = 1u << (off - tr);  // off > tr here
+    const uint32_t starts = __reduce_or_sync(kFull, bit);
+    const uint32_t upto = lane == 31 ? kFull : ((2u << lane) - 1u);
+    const int e = __popc(starts & upto) - 1;  // window lane of this lane's entry
+    v = __shfl_sync(kFull, node, e);
+    const uint32_t eo = __shfl_sync(kFull, off, e);
+    j = (tr + (uint32_t)lane) - eo;
+    k += (uint32_t)__shfl_sync(kFull, e, 31);
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------------------------------
+// relax: queue mode (dynamic mapping) or dense mode (stored array + stamps), chosen per launch
+// ------------------------------------------------------------------------------------------
+template <int A, int LAYOUT, bool BSP, int B, bool STATS>
+__global__ void __launch_bounds__(kFqThreads) k_relax_fq(RelaxArgs a, FqArgs f) {
+    constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    const int lane = threadIdx.x & 31;
+    const uint32_t it = a.ctl->it;
+    const unsigned long long qp = a.ctl->qpack[it & 1u];
+    const uint32_t qn = (uint32_t)(qp >> 32), qt = (uint32_t)qp;
+    const uint64_t span = (uint64_t)(a.hi - a.lo);
+    const bool queue = f.mode == 1 || (f.mode == 0 && (uint64_t)qt * f.dense_div < span);
+    const uint32_t* qv = f.qv + (uint64_t)(it & 1u) * a.n;
+    const uint32_t* qo = f.qo + (uint64_t)(it & 1u) * a.n;
+    const uint32_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;
+    uint32_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
+    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
+    const uint4* w4 = reinterpret_cast<const uint4*>(a.wt);
+    if (blockIdx.x == 0 && threadIdx.x == 0 && queue) atomicAdd(&a.ctl->queue_iters, 1u);
+    const uint64_t total = queue ? (uint64_t)qt : span;
+    constexpr uint32_t kTile = 32u * B;
+    const uint64_t tiles = (total + kTile - 1) / kTile;
+    const uint64_t warp0 = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    bool touched = false;
+    uint32_t n_edges = 0, n_upd = 0, n_vn = 0;
+
+    for (uint64_t tile = warp0; tile < tiles; tile += nwarps) {
+        const uint64_t t0 = tile * kTile;
+        uint32_t v[B], j[B];
+        bool act[B];
+        if (queue) {
+            uint32_t k = warp_search(qo, qn, (uint32_t)t0, lane);
+#pragma unroll
+            for (int r = 0; r < B; ++r) {
+                const uint32_t tr = (uint32_t)t0 + 32u * r;
+                if (tr < qt) {  // warp-uniform
+                    map_round(qv, qo, qn, k, tr, lane, v[r], j[r]);
+                    act[r] = tr + (uint32_t)lane < qt;
+                } else {
+                    v[r] = kPad; j[r] = 0; act[r] = false;
+                }
+                if (!act[r]) v[r] = kPad;
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < B; ++r) {
+                const uint64_t i = (uint64_t)a.lo + t0 + 32u * r + lane;
+                v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
+                j[r] = (uint32_t)i;  // absolute vnode index; made family-relative below
+            }
+#pragma unroll
+            for (int r = 0; r < B; ++r) act[r] = v[r] != kPad && __ldg(stamp_cur + v[r]) == it;
+        }
+        uint32_t x[B];
+        uint4 info[B];
+        bool any = false;
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            x[r] = 0;
+            info[r] = make_uint4(0, 0, 0, 1);
+            if (act[r]) {
+                x[r] = BSP ? __ldg(a.prev + v[r]) : a.val[v[r]];
+                info[r] = __ldg(a.vinfo + v[r]);
+            }
+            any |= act[r];
+        }
+        if (!__any_sync(kFull, any)) continue;
+        uint4 c0[B], c1[B], w0[B], w1[B];
+        uint32_t kn[B], kend[B], step[B];
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
+            const uint32_t jj = queue ? j[r] : j[r] - info[r].z;  // offset within the family
+            uint32_t k;
+            if (!act[r]) { k = 0; step[r] = 1; kend[r] = 0; }
+            else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = jj; step[r] = info[r].w; kend[r] = q; }
+            else {
+                const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
+                k = jj * per; step[r] = 1;
+                kend[r] = (per >= q - k) ? q : k + per;
+            }
+            const uint4 pad4 = make_uint4(kPad, kPad, kPad, kPad);
+            const bool h0 = k < kend[r], h1 = k + step[r] < kend[r];
+            c0[r] = h0 ? ldg_chunk(c4 + info[r].x + k) : pad4;
+            c1[r] = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : pad4;
+            if (W) {
+                w0[r] = h0 ? ldg_chunk(w4 + info[r].x + k) : make_uint4(0, 0, 0, 0);
+                w1[r] = h1 ? ldg_chunk(w4 + info[r].x + k + step[r]) : make_uint4(0, 0, 0, 0);
+            }
+            kn[r] = k + 2 * step[r];
+            if (STATS && act[r]) ++n_vn;
+        }
+        auto relax8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv) {
+            uint32_t cur[8];
+#pragma unroll
+            for (int q = 0; q < 8; ++q) cur[q] = (nb[q] != kPad) ? a.val[nb[q]] : 0u;
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+                if (nb[q] == kPad) continue;
+                if (STATS) ++n_edges;
+                const uint32_t alt = combine<A>(xv, W ? ww[q] : 0u);
+                if (better<A>(alt, cur[q])) {
+                    if (A == TIGR_SSWP) atomicMax(a.val + nb[q], alt);
+                    else atomicMin(a.val + nb[q], alt);
+                    stamp_next[nb[q]] = it + 1;
+                    touched = true;
+                    if (STATS) ++n_upd;
+                }
+            }
+        };
+#pragma unroll
+        for (int r = 0; r < B; ++r) {
+            const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+            uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
+                     ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
+            relax8(nb, ww, x[r]);
+        }
+#pragma unroll
+        for (int r = 0; r < B; ++r) {  // chunks beyond the first two (K > 8 or no split)
+            for (uint32_t k = kn[r]; k < kend[r]; k += 2 * step[r]) {
+                const bool h1 = k + step[r] < kend[r];
+                const uint4 a0 = ldg_chunk(c4 + info[r].x + k);
+                const uint4 a1 = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
+                uint4 b0 = make_uint4(0, 0, 0, 0), b1 = b0;
+                if (W) { b0 = ldg_chunk(w4 + info[r].x + k); if (h1) b1 = ldg_chunk(w4 + info[r].x + k + step[r]); }
+                const uint32_t nb[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+                const uint32_t ww[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+                relax8(nb, ww, x[r]);
+            }
+        }
+    }
+    if (__any_sync(kFull, touched) && lane == 0) a.ctl->changed = 1;
+    if (STATS) {
+        unsigned long long e = n_edges, u = n_upd, q = n_vn;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            e += __shfl_xor_sync(kFull, e, o);
+            u += __shfl_xor_sync(kFull, u, o);
+            q += __shfl_xor_sync(kFull, q, o);
+        }
+        if (lane == 0) {
+            if (e) atomicAdd(&a.ctl->edges, e);
+            if (u) atomicAdd(&a.ctl->updates, u);
+            if (q) atomicAdd(&a.ctl->vnodes, q);
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// queue build: nodes stamped for iteration it + delta that own virtual nodes in [lo, hi)
+// ------------------------------------------------------------------------------------------
+__global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restrict__ stamp,
+                                                         const uint4* __restrict__ vinfo, uint32_t n, uint32_t lo,
+                                                         uint32_t hi, Ctl* ctl, uint32_t* __restrict__ qv,
+                                                         uint32_t* __restrict__ qo, int delta) {
+    __shared__ unsigned long long s_warp[kFqThreads / 32];
+    __shared__ unsigned long long s_base;
+    const uint32_t itn = ctl->it + (uint32_t)delta;
+    const uint32_t slot = itn & 1u;
+    const uint32_t* st = stamp + (uint64_t)slot * n;
+    uint32_t* ov = qv + (uint64_t)slot * n;
+    uint32_t* oo = qo + (uint64_t)slot * n;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    constexpr uint32_t kTileNodes = kFqThreads * kCompactPer;
+    for (uint64_t tile0 = (uint64_t)blockIdx.x * kTileNodes; tile0 < n; tile0 += (uint64_t)gridDim.x * kTileNodes) {
+        const uint64_t v0 = tile0 + (uint64_t)threadIdx.x * kCompactPer;
+        uint32_t m[kCompactPer];
+        unsigned long long mine = 0;  // (entries << 32) | vnodes of this thread's nodes
+#pragma unroll
+        for (int q = 0; q < kCompactPer; ++q) {
+            const uint64_t v = v0 + q;
+            m[q] = 0;
+            if (v < n && __ldg(st + v) == itn) {
+                const uint4 info = __ldg(vinfo + v);
+                if (info.w && info.z >= lo && info.z < hi) m[q] = info.w;
+            }
+            if (m[q]) mine += (1ull << 32) | m[q];
+        }
+        // block exclusive scan of the packed counts (no carry: vnodes < 2^32)
+        unsigned long long inc = mine;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long y = __shfl_up_sync(kFull, inc, o);
+            if (lane >= o) inc += y;
+        }
+        if (lane == 31) s_warp[wid] = inc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            unsigned long long run = 0;
+            for (int w = 0; w < kFqThreads / 32; ++w) { const unsigned long long t = s_warp[w]; s_warp[w] = run; run += t; }
+            s_base = run ? atomicAdd(&ctl->qpack[slot], run) : 0ull;
+        }
+        __syncthreads();
+        unsigned long long pos = s_base + s_warp[wid] + (inc - mine);
+        __syncthreads();  // s_warp / s_base reused by the next tile
+#pragma unroll
+        for (int q = 0; q < kCompactPer; ++q) {
+            if (!m[q]) continue;
+            const uint32_t e = (uint32_t)(pos >> 32);
+            ov[e] = (uint32_t)(v0 + q);
+            oo[e] = (uint32_t)pos;
+            pos += (1ull << 32) | m[q];
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------------------
+// dispatch
+// ------------------------------------------------------------------------------------------
+template <int A, int LAYOUT>
+static FqFn pick_fq(bool bsp, bool stats) {
+    if (bsp) return stats ? &k_relax_fq<A, LAYOUT, true, 4, true> : &k_relax_fq<A, LAYOUT, true, 4, false>;
+    return stats ? &k_relax_fq<A, LAYOUT, false, 4, true> : &k_relax_fq<A, LAYOUT, false, 4, false>;
+}
+
+FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats) {
+    const bool st = layout == TIGR_LAYOUT_STRIDED;
+    switch (algo) {
+        case TIGR_BFS: return st ? pick_fq<TIGR_BFS, TIGR_LAYOUT_STRIDED>(bsp, stats)
+                                 : pick_fq<TIGR_BFS, TIGR_LAYOUT_CONSECUTIVE>(bsp, stats);
+        case TIGR_SSSP: return st ? pick_fq<TIGR_SSSP, TIGR_LAYOUT_STRIDED>(bsp, stats)
+                                  : pick_fq<TIGR_SSSP, TIGR_LAYOUT_CONSECUTIVE>(bsp, stats);
+        case TIGR_CC: return st ? pick_fq<TIGR_CC, TIGR_LAYOUT_STRIDED>(bsp, stats)
+                                : pick_fq<TIGR_CC, TIGR_LAYOUT_CONSECUTIVE>(bsp, stats);
+        case TIGR_SSWP: return st ? pick_fq<TIGR_SSWP, TIGR_LAYOUT_STRIDED>(bsp, stats)
+                                  : pick_fq<TIGR_SSWP, TIGR_LAYOUT_CONSECUTIVE>(bsp, stats);
+    }
+    return nullptr;
+}
+
+unsigned relax_fq_grid(FqFn fn) {
+    int per_sm = 0, dev = 0, sms = 148;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kFqThreads, 0);
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    return (unsigned)(sms * (per_sm > 0 ? per_sm : 1));
+}
+
+int relax_fq_threads() { return kFqThreads; }
+
+tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s) {
+    const uint32_t n = vg->g->n;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t tiles = ((uint64_t)n + kFqThreads * kCompactPer - 1) / (kFqThreads * kCompactPer);
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(tiles, (uint64_t)sms * 8));
+    k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<uint32_t>(), vg->vinfo.as<uint4>(), n, vg->lo, vg->hi, ctl,
+                                          const_cast<uint32_t*>(vg->ws.qv.as<uint32_t>()),
+                                          const_cast<uint32_t*>(vg->ws.qo.as<uint32_t>()), delta);
+    TIGR_CK(cudaGetLastError());
+    return TIGR_OK;
+}
+
+}  // namespace tigr

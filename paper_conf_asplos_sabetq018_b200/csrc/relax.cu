@@ -77,22 +77,6 @@ __device__ __forceinline__ void walk(const uint32_t* __restrict__ col, const uin
 // ------------------------------------------------------------------------------------------
 // relax kernel
 // ------------------------------------------------------------------------------------------
-template <int A>
-__device__ __forceinline__ bool better(uint32_t alt, uint32_t cur) {
-    return A == TIGR_SSWP ? alt > cur : alt < cur;
-}
-
-template <int A>
-__device__ __forceinline__ uint32_t combine(uint32_t x, uint32_t w) {
-    if (A == TIGR_BFS) return x + 1;
-    if (A == TIGR_SSSP) {
-        const uint64_t s = (uint64_t)x + w;
-        return s >= kInf ? kInf - 1 : (uint32_t)s;
-    }
-    if (A == TIGR_CC) return x;
-    return x < w ? x : w;  // SSWP
-}
-
 template <int A, int LAYOUT, bool VEC, int FRONT, bool BSP, bool STATS>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
@@ -700,12 +684,14 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
     if (v == 0) {
         ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
+        ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0;
     }
 }
 
 // end of one iteration: decide whether to continue; sets the graph's WHILE condition
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle) {
     const uint32_t changed = ctl->changed;
+    ctl->qpack[ctl->it & 1u] = 0ull;  // queue slot consumed by this iteration (frontier.cu)
     uint32_t cont = changed ? 1u : 0u;
     if (changed && ctl->it >= ctl->max_iters) { cont = 0; ctl->notconv = 1; }
     ctl->changed = 0;

@@ -23,6 +23,20 @@ struct RelaxArgs {
 };
 
 typedef void (*RelaxFn)(RelaxArgs);
+
+// queue-driven frontier relax with dynamic virtual-node mapping (frontier.cu)
+struct FqArgs {
+    const uint32_t* qv;   // uint32[2][n] queue node ids (slot = iteration parity)
+    const uint32_t* qo;   // uint32[2][n] queue-space first virtual node of each entry
+    int mode;             // 0 = per iteration (queue if vnodes * dense_div < span), 1 = queue, 2 = dense
+    uint32_t dense_div;
+};
+typedef void (*FqFn)(RelaxArgs, FqArgs);
+FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);
+unsigned relax_fq_grid(FqFn fn);
+int relax_fq_threads();
+struct Ctl;
+tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s);
 typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
 
 RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats);

@@ -53,6 +53,10 @@ tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
         TIGR_TRY(ws.prev.alloc(sizeof(uint32_t) * n, s));
         TIGR_TRY(ws.stamp.alloc(sizeof(uint32_t) * 2 * n, s));
     }
+    if (!pr && vg->vec && !ws.qv.p) {  // active-node queues (frontier.cu), one per iteration parity
+        TIGR_TRY(ws.qv.alloc(sizeof(uint32_t) * 2 * n, s));
+        TIGR_TRY(ws.qo.alloc(sizeof(uint32_t) * 2 * n, s));
+    }
     return TIGR_OK;
 }
 
@@ -78,6 +82,9 @@ RelaxArgs make_args(tigr_vgraph* vg) {
 
 struct FrontierPlan {
     RelaxFn relax;
+    FqFn fq = nullptr;     // queue / dynamic-mapping relax (frontier.cu); relax unused when set
+    FqArgs fa;
+    const tigr_vgraph* vg = nullptr;
     RelaxArgs args;
     unsigned grid;
     bool bsp, comm;
@@ -93,7 +100,11 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
     if (p.bsp && !p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * p.n, cudaMemcpyDeviceToDevice, s));
     if (ev_a) TIGR_CK(cudaEventRecord(ev_a, s));
-    if (p.grid) {
+    if (p.grid && p.fq) {
+        p.fq<<<p.grid, relax_fq_threads(), 0, s>>>(p.args, p.fa);
+        TIGR_CK(cudaGetLastError());
+        ++k;
+    } else if (p.grid) {
         p.relax<<<p.grid, kRelaxThreads, 0, s>>>(p.args);
         TIGR_CK(cudaGetLastError());
         ++k;
@@ -107,6 +118,10 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
         TIGR_CK(cudaGetLastError());
         ++k;
     }
+    if (p.fq) {  // next iteration's queue from the stamps just written
+        TIGR_TRY(compact_launch(p.vg, p.args.ctl, 1, s));
+        ++k;
+    }
     k_control<<<1, 1, 0, s>>>(p.args.ctl, h, use_handle);
     TIGR_CK(cudaGetLastError());
     ++k;
@@ -118,8 +133,22 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
                          tigr_stats* st) {
     Workspace& ws = vg->ws;
     const uint32_t n = vg->g->n;
-    int front = o.frontier == TIGR_FRONTIER_AUTO ? TIGR_FRONTIER_DENSE : o.frontier;
+    int front = o.frontier;
     FrontierPlan p;
+    p.vg = vg;
+    if ((front == TIGR_FRONTIER_AUTO || front == TIGR_FRONTIER_QUEUE) && vg->vec) {
+        p.fq = relax_fq_kernel(algo, vg->layout, o.schedule == 1, o.collect_stats != 0);
+        p.fa.qv = ws.qv.as<uint32_t>();
+        p.fa.qo = ws.qo.as<uint32_t>();
+        p.fa.mode = front == TIGR_FRONTIER_QUEUE ? 1 : 0;
+        const char* e = getenv("TIGR_FQ_MODE");   // development knob: force 1 = queue, 2 = dense
+        if (e && front == TIGR_FRONTIER_AUTO) p.fa.mode = atoi(e);
+        const char* d = getenv("TIGR_FQ_DIV");
+        p.fa.dense_div = d ? (uint32_t)atoi(d) : 2u;
+    } else if (front == TIGR_FRONTIER_QUEUE) {
+        return fail(TIGR_EUNSUPPORTED, "frontier QUEUE needs the 16-byte-chunk layout (4 | K)");
+    }
+    if (front == TIGR_FRONTIER_AUTO || front == TIGR_FRONTIER_QUEUE) front = TIGR_FRONTIER_DENSE;
     p.bsp = o.schedule == 1;
     p.comm = o.comm != nullptr;  // a 1-rank communicator still runs the exchange path (tests)
     p.c = o.comm;
@@ -135,6 +164,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         per_thread = 1;
     const uint64_t per_block = (uint64_t)kRelaxThreads * per_thread;
     p.grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
+    if (p.fq) p.grid = vg->hi > vg->lo ? relax_fq_grid(p.fq) : 0;  // persistent
     const uint32_t max_iters = o.max_iters ? o.max_iters : (n + 1 > n ? n + 1 : n);
 
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
@@ -143,6 +173,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     TIGR_CKL("init");
     if (p.bsp || p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
+    if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s));  // iteration 1's queue
 
     int kpi = 0;
     uint32_t launches = 0;
@@ -150,8 +181,8 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
     const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
     if (use_graph) {
-        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0), front, p.bsp ? 1 : 0, o.collect_stats ? 1 : 0,
-                     p.comm ? 1 : 0, vg->lo, vg->hi};
+        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0), p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div : front,
+                     p.bsp ? 1 : 0, o.collect_stats ? 1 : 0, p.comm ? 1 : 0, vg->lo, vg->hi};
         auto itg = ws.graphs.find(key);
         if (itg == ws.graphs.end()) {
             CachedGraph cg;
@@ -222,6 +253,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         st->active_vnodes = c.vnodes;
         st->ms_total = ms;
         st->ms_relax = ms_relax;
+        st->queue_iterations = c.queue_iters;
     }
     if (c.notconv) return fail(TIGR_ENOTCONV, "max_iters reached before the fixed point");
     return TIGR_OK;
@@ -361,6 +393,8 @@ tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const t
                        int out_is_device, tigr_stats* st) {
     const tigr_graph* g = vg->g;
     if ((int)algo < TIGR_BFS || (int)algo > TIGR_PR) return fail(TIGR_EINVAL, "run: unknown algorithm");
+    if (o.frontier == TIGR_FRONTIER_QUEUE && algo == TIGR_PR)
+        return fail(TIGR_EUNSUPPORTED, "run: frontier QUEUE applies to BFS/SSSP/CC/SSWP");
     if ((algo == TIGR_BFS || algo == TIGR_SSSP || algo == TIGR_SSWP) && source >= g->n)
         return fail(TIGR_EINVAL, "run: source >= n");
     if ((algo == TIGR_SSSP || algo == TIGR_SSWP) && !g->weighted)
@@ -369,7 +403,7 @@ tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const t
         return fail(TIGR_EINVAL, "run: CC needs a symmetric graph (build with symmetrize=1)");
     if (algo == TIGR_PR && !(o.pr_damping >= 0.0 && o.pr_damping <= 1.0))
         return fail(TIGR_EINVAL, "run: pr_damping outside [0, 1]");
-    if (o.frontier < TIGR_FRONTIER_AUTO || o.frontier > TIGR_FRONTIER_NONE)
+    if (o.frontier < TIGR_FRONTIER_AUTO || o.frontier > TIGR_FRONTIER_QUEUE)
         return fail(TIGR_EINVAL, "run: unknown frontier mode");
     cudaStream_t s = (cudaStream_t)o.stream;
     if (st) *st = tigr_stats{};

@@ -19,6 +19,10 @@ struct Ctl {
     uint32_t pad[3];
     unsigned long long edges, updates, vnodes;
     double dsum[2];        // PR: dangling mass of the iterate (parity of the iteration)
+    // active-node queue of iteration it (frontier.cu): slot it&1 packs (entries << 32) | vnodes
+    unsigned long long qpack[2];
+    uint32_t queue_iters;  // iterations the queue-driven (dynamic-mapping) path ran
+    uint32_t pad2;
 };
 
 struct GraphKey {
@@ -49,6 +53,8 @@ struct Workspace {
     DevBuf col_pr;   // uint32[4 * nchunks]: arc targets as accumulator ids (PR only)
     uint32_t n_in = 0;       // nodes with in-arcs (= accumulator entries ever written)
     bool cid_ready = false;
+    DevBuf qv;       // uint32[2][n]: active-node queue (node ids), one slot per iteration parity
+    DevBuf qo;       // uint32[2][n]: first queue-space virtual node of each entry (exclusive prefix)
     DevBuf ctl;      // Ctl
     Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (thread-local, not owned)
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};

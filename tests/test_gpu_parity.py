@@ -156,7 +156,8 @@ def test_cfg1_all_algorithms(tigr, K, layout):
     _assert_parity(_run_all(tigr, rec.n, src, dst, w, K, layout), _oracle_all(rec.n, src, dst, w))
 
 
-@pytest.mark.parametrize("schedule,frontier,use_graph", [(0, 1, 1), (1, 1, 1), (0, 2, 1), (1, 2, 0), (0, 1, 0)])
+@pytest.mark.parametrize("schedule,frontier,use_graph", [(0, 1, 1), (1, 1, 1), (0, 2, 1), (1, 2, 0), (0, 1, 0),
+                                                          (0, 3, 1), (1, 3, 1), (0, 3, 0), (1, 0, 1), (0, 0, 0)])
 def test_cfg1_schedules(tigr, schedule, frontier, use_graph):
     rec = graphgen.recipe("cfg1")
     src, dst, w = graphgen.generate(rec)
@@ -218,6 +219,63 @@ def test_edge_cases(tigr, name, K):
     n, src, dst, w = _edge_cases()[name]
     src, dst, w = (np.asarray(x, dtype=np.uint32) for x in (src, dst, w))
     _assert_parity(_run_all(tigr, n, src, dst, w, K), _oracle_all(n, src, dst, w))
+
+
+@pytest.mark.parametrize("name", list(_edge_cases()))
+@pytest.mark.parametrize("K", [4, 8, 32])
+@pytest.mark.parametrize("schedule", [0, 1])
+def test_edge_cases_queue(tigr, name, K, schedule):
+    """Frontier QUEUE (dynamic mapping, frontier.cu): the active-node queue and the on-the-fly
+    (node, j) mapping reproduce the oracle on every edge case, incl. a 70 000-arc hub whose
+    8750 virtual nodes span hundreds of warp rounds of one queue entry."""
+    n, src, dst, w = _edge_cases()[name]
+    src, dst, w = (np.asarray(x, dtype=np.uint32) for x in (src, dst, w))
+    got = _run_all(tigr, n, src, dst, w, K, frontier=3, schedule=schedule)
+    _assert_parity(got, _oracle_all(n, src, dst, w))
+
+
+@pytest.mark.parametrize("layout", ["consecutive", "strided"])
+@pytest.mark.parametrize("div", ["1", "2", "1000000"])
+def test_hybrid_frontier_switch(tigr, layout, div, monkeypatch):
+    """FRONTIER_AUTO switches between the queue and the dense sweep per iteration on the device
+    (TIGR_FQ_DIV = D: queue while the queued vnodes are < 1/D of all, so D = 1 is almost always
+    the queue and D = 1e6 almost always the dense sweep): every switch point gives the oracle's
+    values and BSP iteration counts."""
+    monkeypatch.setenv("TIGR_FQ_DIV", div)
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    want = _oracle_all(rec.n, src, dst, w)
+    for K in (4, 8, 32):
+        _assert_parity(_run_all(tigr, rec.n, src, dst, w, K, layout), want)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(g, 8, layout)
+    for algo, code in (("bfs", oracle.BFS), ("sssp", oracle.SSSP), ("sswp", oracle.SSWP)):
+        _, want_it, _ = oracle.push_virtual(o, oracle.Virtual(o, 8), code, 0, schedule=1, worklist=1)
+        vals, st = tigr.tigr_run(vg, algo, 0, schedule=1, return_stats=True)
+        assert np.array_equal(vals, want[algo]) and st["iterations"] == want_it, (algo, st["iterations"], want_it)
+
+
+def test_queue_mode_stats_and_errors(tigr):
+    """QUEUE counts the same processed arcs as the dense sweep (BSP BFS: every arc of every
+    reached node), reports its queue iterations, and needs the 16-byte-chunk layout."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(g, 8)
+    deg = np.bincount(src, minlength=rec.n)
+    lv, st = tigr.tigr_run(vg, "bfs", 0, schedule=1, frontier=3, collect_stats=1, return_stats=True)
+    assert st["edges_processed"] == int(deg[lv != INF].sum())
+    assert st["queue_iterations"] == st["iterations"]
+    _, st1 = tigr.tigr_run(vg, "bfs", 0, schedule=1, frontier=1, collect_stats=1, return_stats=True)
+    assert st1["edges_processed"] == st["edges_processed"] and st1["queue_iterations"] == 0
+    vg3 = tigr.tigr_virtualize(g, 3)  # 4 does not divide K: per-arc units, no queue kernel
+    with pytest.raises(tigr.TigrError) as e:
+        tigr.tigr_run(vg3, "bfs", 0, frontier=3)
+    assert e.value.status == tigr.TIGR_EUNSUPPORTED
+    assert np.array_equal(tigr.tigr_run(vg3, "bfs", 0), lv)  # AUTO falls back to the dense sweep
+    with pytest.raises(tigr.TigrError):
+        tigr.tigr_run(vg, "pr", frontier=3)
 
 
 def test_unit_weights_sssp_equals_bfs(tigr):
