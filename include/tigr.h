@@ -174,6 +174,23 @@ tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* 
  * Errors: ENOMEM, ECUDA. */
 tigr_status tigr_graph_transpose(const tigr_graph* g, void* stream, tigr_graph** out);
 
+/* Node relabelling by decreasing in-degree (ties by increasing id): node c of the result is
+ * node order[c] of g, with its arcs in g's order and targets relabelled.  The paper's
+ * transformations change which thread owns which edges, never the node numbering (§4,
+ * L819-1180); this is a locality transformation of the same graph, beside them: the hottest
+ * destinations get the smallest ids, so the frontier relax can bound their values in shared
+ * memory and their value gathers share cache lines.  The result remembers the
+ * permutation: tigr_run on a virtual split of it takes the source as an ORIGINAL id and
+ * returns values indexed by ORIGINAL ids (CC labels stay the minimum original id).  Its
+ * exported CSR / virtual arrays are in the new numbering.  g may be freed afterwards.
+ * Errors: EUNSUPPORTED (transposed, partitioned or already reordered g), ENOMEM, ECUDA. */
+tigr_status tigr_graph_reorder(const tigr_graph* g, void* stream, tigr_graph** out);
+
+/* Permutation of a reordered graph: cid[v] = new id of original node v, order[c] = original
+ * id of new node c (n entries each; either may be NULL).  EINVAL if g is not reordered. */
+tigr_status tigr_graph_permutation(const tigr_graph* g, uint32_t* cid, uint32_t* order, int is_device_ptr,
+                                   void* stream);
+
 /* PHYSICAL uniform-degree-tree transformation (UDT, §3.2 Alg. 1): every
  * node v of out-degree d > K keeps <= K arcs and hands the rest to t = ceil((d-K)/(K-1)) new
  * split nodes of out-degree exactly K, numbered n, n+1, ... in order of v and creation (the

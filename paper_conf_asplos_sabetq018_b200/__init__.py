@@ -72,6 +72,8 @@ _SIGS = {
                              ctypes.POINTER(_I), ctypes.POINTER(_I), ctypes.POINTER(_U64)]),
     "tigr_graph_transpose": (_I, [_P, _P, ctypes.POINTER(_P)]),
     "tigr_graph_udt": (_I, [_P, _U32, _U32, _U32, _P, ctypes.POINTER(_P)]),
+    "tigr_graph_reorder": (_I, [_P, _P, ctypes.POINTER(_P)]),
+    "tigr_graph_permutation": (_I, [_P, _P, _P, _I, _P]),
     "tigr_graph_export_csr": (_I, [_P, _P, _P, _P, _I, _P]),
     "tigr_graph_free": (None, [_P]),
     "tigr_virtualize": (_I, [_P, _U32, _I, _P, ctypes.POINTER(_P)]),
@@ -285,6 +287,22 @@ def tigr_graph_transpose(g: Graph, stream=None) -> Graph:
     out = _P()
     _check(_lib.tigr_graph_transpose(g.ptr, _stream_ptr(stream), ctypes.byref(out)))
     return Graph(out.value)
+
+
+def tigr_graph_reorder(g: Graph, stream=None) -> Graph:
+    """Same graph, nodes relabelled by decreasing in-degree; runs on it take and return original ids."""
+    out = _P()
+    _check(_lib.tigr_graph_reorder(g.ptr, _stream_ptr(stream), ctypes.byref(out)))
+    return Graph(out.value)
+
+
+def tigr_graph_permutation(g: Graph, stream=None):
+    """Host copies (cid uint32[n]: original -> new id, order uint32[n]: new -> original id)."""
+    n = g.info()["n"]
+    cid = np.empty(max(n, 1), dtype=np.uint32)
+    order = np.empty(max(n, 1), dtype=np.uint32)
+    _check(_lib.tigr_graph_permutation(g.ptr, cid.ctypes.data, order.ctypes.data, 0, _stream_ptr(stream)))
+    return cid[:n], order[:n]
 
 
 def tigr_graph_udt(g: Graph, K: int, dumb_weight: int = 0, unit_weight: int = 1, stream=None) -> Graph:

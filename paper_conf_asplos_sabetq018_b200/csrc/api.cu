@@ -166,6 +166,7 @@ tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, con
                                   int symmetric_hint, cudaStream_t s, tigr_graph** out);
 tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w, cudaStream_t s);
 tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out);
+tigr_status graph_reorder_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out);
 tigr_status graph_udt_device(const tigr_graph* g, uint32_t K, uint32_t dumb, uint32_t unit, cudaStream_t s,
                              tigr_graph** out);
 tigr_status graph_rmat_device(uint32_t n, uint64_t m, double a, double b, double c, uint64_t seed, uint64_t wseed,
@@ -365,6 +366,27 @@ tigr_status tigr_graph_transpose(const tigr_graph* g, void* stream, tigr_graph**
     *out = nullptr;
     cudaStream_t s = (cudaStream_t)stream;
     TIGR_TRY(graph_transpose_device(g, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_graph_reorder(const tigr_graph* g, void* stream, tigr_graph** out) {
+    if (!g || !out) return fail(TIGR_EINVAL, "graph_reorder: NULL argument");
+    *out = nullptr;
+    cudaStream_t s = (cudaStream_t)stream;
+    TIGR_TRY(graph_reorder_device(g, s, out));
+    TIGR_CK(cudaStreamSynchronize(s));
+    return TIGR_OK;
+}
+
+tigr_status tigr_graph_permutation(const tigr_graph* g, uint32_t* cid, uint32_t* order, int is_device_ptr,
+                                   void* stream) {
+    if (!g) return fail(TIGR_EINVAL, "graph_permutation: NULL graph");
+    if (!g->reordered) return fail(TIGR_EINVAL, "graph_permutation: graph is not reordered");
+    cudaStream_t s = (cudaStream_t)stream;
+    const cudaMemcpyKind k = is_device_ptr ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
+    if (cid && g->n) TIGR_CK(cudaMemcpyAsync(cid, g->perm_cid.p, sizeof(uint32_t) * g->n, k, s));
+    if (order && g->n) TIGR_CK(cudaMemcpyAsync(order, g->perm_order.p, sizeof(uint32_t) * g->n, k, s));
     TIGR_CK(cudaStreamSynchronize(s));
     return TIGR_OK;
 }

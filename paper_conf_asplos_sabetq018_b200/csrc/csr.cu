@@ -20,6 +20,8 @@ tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const 
 
 namespace {
 
+constexpr uint32_t kReorderKeyMax = (1u << 24) - 1;  // in-degrees beyond tie (stable: by id)
+
 __global__ void k_pad(const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cptr, uint32_t n,
                       uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
@@ -200,6 +202,42 @@ tigr_status layout_from_degrees(tigr_graph* g, cudaStream_t s) {
     return TIGR_OK;
 }
 
+
+// exact in-degrees: one RED.ADD per arc (pads skipped)
+__global__ void k_indeg_count(const uint4* __restrict__ c4, uint64_t nchunks, uint32_t* __restrict__ cnt) {
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
+         k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 c = c4[k];
+        if (c.x != kPad) atomicAdd(cnt + c.x, 1u);
+        if (c.y != kPad) atomicAdd(cnt + c.y, 1u);
+        if (c.z != kPad) atomicAdd(cnt + c.z, 1u);
+        if (c.w != kPad) atomicAdd(cnt + c.w, 1u);
+    }
+}
+
+// sort key for decreasing in-degree (ties: increasing id, the sort is stable)
+__global__ void k_reorder_key(const uint32_t* __restrict__ cnt, uint32_t n, uint32_t* __restrict__ key,
+                              uint32_t* __restrict__ ids) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    const uint32_t c = cnt[v] < kReorderKeyMax ? cnt[v] : kReorderKeyMax;
+    key[v] = kReorderKeyMax - c;
+    ids[v] = v;
+}
+
+__global__ void k_inverse(const uint32_t* __restrict__ order, uint32_t n, uint32_t* __restrict__ cid) {
+    const uint32_t c = blockIdx.x * blockDim.x + threadIdx.x;
+    if (c < n) cid[order[c]] = c;
+}
+
+__global__ void k_relabel(uint32_t* __restrict__ src, uint32_t* __restrict__ dst, uint64_t m,
+                          const uint32_t* __restrict__ cid) {
+    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x) {
+        src[e] = __ldg(cid + src[e]);
+        dst[e] = __ldg(cid + dst[e]);
+    }
+}
+
 }  // namespace
 
 // src_lo/src_hi: keep only the arcs whose source lies in [src_lo, src_hi) (multi-GPU partitioned
@@ -309,6 +347,64 @@ tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_gra
     if (st == TIGR_OK && g->n) {
         cudaError_t e = cudaMemcpyAsync(t->src_deg.p, g->deg.p, sizeof(uint32_t) * g->n, cudaMemcpyDeviceToDevice, s);
         if (e != cudaSuccess) st = cuda_fail(e, "transpose src_deg", __FILE__, __LINE__);
+    }
+    if (st != TIGR_OK) { delete t; return st; }
+    *out = t;
+    return TIGR_OK;
+}
+
+// Node relabelling by decreasing in-degree (tigr_graph_reorder).  The arcs are expanded,
+// both endpoints mapped through cid, and rebuilt by the stable CSR builder, so node c's
+// segment is node order[c]'s segment in its canonical order with relabelled targets.
+tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t count, uint32_t key_limit,
+                           cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out);
+
+tigr_status graph_reorder_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out) {
+    if (g->transposed || g->reordered || g->part_lo != 0 || g->part_hi < g->n)
+        return fail(TIGR_EUNSUPPORTED, "reorder: needs a full, forward, not yet reordered graph");
+    const uint32_t n = g->n;
+    const uint64_t m = g->m;
+    TmpBuf cnt, key, ids;
+    TIGR_TRY(cnt.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(key.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_TRY(ids.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_CK(cudaMemsetAsync(cnt.p, 0, sizeof(uint32_t) * (n ? n : 1), s));
+    if (g->nchunks) {
+        k_indeg_count<<<capped_grid(g->nchunks), kBlock, 0, s>>>(g->col.as<uint4>(), g->nchunks, cnt.as<uint32_t>());
+        TIGR_CKL("reorder indeg");
+    }
+    k_reorder_key<<<grid_for(n), kBlock, 0, s>>>(cnt.as<uint32_t>(), n, key.as<uint32_t>(), ids.as<uint32_t>());
+    TIGR_CKL("reorder key");
+    TmpBuf skeys, order;
+    TIGR_TRY(sort_pairs_u32(key.as<uint32_t>(), ids.as<uint32_t>(), n, kReorderKeyMax + 1, s, skeys, order));
+    TmpBuf cid;
+    TIGR_TRY(cid.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    k_inverse<<<grid_for(n), kBlock, 0, s>>>(order.as<uint32_t>(), n, cid.as<uint32_t>());
+    TIGR_CKL("reorder inverse");
+    TmpBuf src, dst, w;
+    TIGR_TRY(src.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    TIGR_TRY(dst.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    if (g->weighted) TIGR_TRY(w.alloc(sizeof(uint32_t) * (m ? m : 1), s));
+    k_expand_arcs<<<grid_for(n), kBlock, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), n,
+                                                 g->col.as<uint32_t>(), g->wt.as<uint32_t>(), src.as<uint32_t>(),
+                                                 dst.as<uint32_t>(), g->weighted ? w.as<uint32_t>() : nullptr);
+    TIGR_CKL("reorder expand");
+    if (m) {
+        k_relabel<<<capped_grid(m), kBlock, 0, s>>>(src.as<uint32_t>(), dst.as<uint32_t>(), m, cid.as<uint32_t>());
+        TIGR_CKL("reorder relabel");
+    }
+    tigr_graph* t = nullptr;
+    TIGR_TRY(graph_from_coo_device(n, m, src.as<uint32_t>(), dst.as<uint32_t>(),
+                                   g->weighted ? w.as<uint32_t>() : nullptr, 0, s, &t));
+    t->symmetric = g->symmetric;
+    t->reordered = true;
+    tigr_status st = t->perm_cid.alloc(sizeof(uint32_t) * (n ? n : 1), s);
+    if (st == TIGR_OK) st = t->perm_order.alloc(sizeof(uint32_t) * (n ? n : 1), s);
+    if (st == TIGR_OK && n) {
+        cudaError_t e = cudaMemcpyAsync(t->perm_cid.p, cid.p, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s);
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(t->perm_order.p, order.p, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s);
+        if (e != cudaSuccess) st = cuda_fail(e, "reorder perm", __FILE__, __LINE__);
     }
     if (st != TIGR_OK) { delete t; return st; }
     *out = t;

@@ -97,8 +97,8 @@ __device__ __forceinline__ void map_round(const uint32_t* __restrict__ qv, const
 // ------------------------------------------------------------------------------------------
 // relax: queue mode (dynamic mapping) or dense mode (stored array + stamps), chosen per launch
 // ------------------------------------------------------------------------------------------
-template <int A, int LAYOUT, bool BSP, int B, bool STATS>
-__global__ void __launch_bounds__(kFqThreads) k_relax_fq(RelaxArgs a, FqArgs f) {
+template <int A, int LAYOUT, bool BSP, int B, bool STATS, int MINB, bool PRE>
+__global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     const int lane = threadIdx.x & 31;
     const uint32_t it = a.ctl->it;
@@ -120,7 +120,6 @@ __global__ void __launch_bounds__(kFqThreads) k_relax_fq(RelaxArgs a, FqArgs f) 
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     bool touched = false;
     uint32_t n_edges = 0, n_upd = 0, n_vn = 0;
-
     for (uint64_t tile = warp0; tile < tiles; tile += nwarps) {
         const uint64_t t0 = tile * kTile;
         uint32_t v[B], j[B];
@@ -187,10 +186,12 @@ __global__ void __launch_bounds__(kFqThreads) k_relax_fq(RelaxArgs a, FqArgs f) 
             kn[r] = k + 2 * step[r];
             if (STATS && act[r]) ++n_vn;
         }
-        auto relax8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv) {
-            uint32_t cur[8];
+        auto gather8 = [&](const uint32_t* nb, uint32_t* cur) {
 #pragma unroll
-            for (int q = 0; q < 8; ++q) cur[q] = (nb[q] != kPad) ? a.val[nb[q]] : 0u;
+            for (int q = 0; q < 8; ++q)
+                cur[q] = (nb[q] == kPad) ? 0u : a.val[nb[q]];
+        };
+        auto apply8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv, const uint32_t* cur) {
 #pragma unroll
             for (int q = 0; q < 8; ++q) {
                 if (nb[q] == kPad) continue;
@@ -205,13 +206,35 @@ __global__ void __launch_bounds__(kFqThreads) k_relax_fq(RelaxArgs a, FqArgs f) 
                 }
             }
         };
+        auto relax8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv) {
+            uint32_t cur[8];
+            gather8(nb, cur);
+            apply8(nb, ww, xv, cur);
+        };
+        if (PRE) {  // every target value of the first two chunks of all B vnodes in flight at once
+            uint32_t cur[B][8];
 #pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
-            uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
-                     ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
-            relax8(nb, ww, x[r]);
+            for (int r = 0; r < B; ++r) {
+                const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+                gather8(nb, cur[r]);
+            }
+#pragma unroll
+            for (int r = 0; r < B; ++r) {
+                const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+                uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
+                         ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
+                apply8(nb, ww, x[r], cur[r]);
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < B; ++r) {
+                const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+                uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+                if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
+                         ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
+                relax8(nb, ww, x[r]);
+            }
         }
 #pragma unroll
         for (int r = 0; r < B; ++r) {  // chunks beyond the first two (K > 8 or no split)
@@ -305,10 +328,19 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
 // ------------------------------------------------------------------------------------------
 // dispatch
 // ------------------------------------------------------------------------------------------
+
+// Kernel shape per algorithm (cfg4 sweep, tools/dev/fq_sweep.sh): the relax
+// is bound by L1tex wavefronts of the random target-value gathers and by latency, so
+// occupancy matters more than per-thread depth.  Unweighted (BFS, CC): 4 vnodes per thread,
+// 80 registers, 3 blocks/SM.  Weighted (SSSP, SSWP; one more 16-byte load per chunk): 2 vnodes
+// per thread with all target gathers of both issued before the first atomic, 3 blocks/SM.
 template <int A, int LAYOUT>
 static FqFn pick_fq(bool bsp, bool stats) {
-    if (bsp) return stats ? &k_relax_fq<A, LAYOUT, true, 4, true> : &k_relax_fq<A, LAYOUT, true, 4, false>;
-    return stats ? &k_relax_fq<A, LAYOUT, false, 4, true> : &k_relax_fq<A, LAYOUT, false, 4, false>;
+    constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    constexpr int B = W ? 2 : 4;
+    constexpr bool PRE = W;
+    if (bsp) return stats ? &k_relax_fq<A, LAYOUT, true, B, true, 3, PRE> : &k_relax_fq<A, LAYOUT, true, B, false, 3, PRE>;
+    return stats ? &k_relax_fq<A, LAYOUT, false, B, true, 3, PRE> : &k_relax_fq<A, LAYOUT, false, B, false, 3, PRE>;
 }
 
 FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats) {

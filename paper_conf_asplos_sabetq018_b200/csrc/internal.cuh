@@ -112,6 +112,11 @@ struct tigr_graph {
     // partitioned builds (tigr_graph_from_coo_part): only sources in [part_lo, part_hi) have arcs
     uint32_t part_lo = 0, part_hi = 0xFFFFFFFFu;
     tigr::DevBuf src_deg;    // uint32[n] (transposed graphs only)
+    // reordered graphs (tigr_graph_reorder): node c here is node perm_order[c] of the source
+    // graph, perm_cid is the inverse; sources and results are translated at the ABI
+    bool reordered = false;
+    tigr::DevBuf perm_cid;   // uint32[n]: original id -> id here
+    tigr::DevBuf perm_order; // uint32[n]: id here -> original id
 };
 
 struct tigr_comm {

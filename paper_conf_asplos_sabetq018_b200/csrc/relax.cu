@@ -670,22 +670,41 @@ RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool s
 // init / control / PR apply / multi-GPU diff / assignment dump
 // ------------------------------------------------------------------------------------------
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
-                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters) {
+                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
+                       const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order) {
+    // reordered graphs (tigr_graph_reorder): the source is an original id, CC labels are
+    // original ids (the minimum original id of the component)
+    const uint32_t src = cid ? cid[source] : source;
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
     if (v < n) {
         uint32_t x = kInf;
-        if (algo == TIGR_CC) x = v;
+        if (algo == TIGR_CC) x = order ? order[v] : v;
         else if (algo == TIGR_SSWP) x = 0;
-        if (v == source && algo != TIGR_CC) x = (algo == TIGR_SSWP) ? kInf : 0;
+        if (v == src && algo != TIGR_CC) x = (algo == TIGR_SSWP) ? kInf : 0;
         val[v] = x;
-        stamp[v] = 0u;                                                   // parity 0
-        stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == source) ? 1u : 0u;  // parity 1: it = 1
+        stamp[v] = 0u;                                                // parity 0
+        stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == src) ? 1u : 0u;  // parity 1: it = 1
     }
     if (v == 0) {
         ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
         ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0;
     }
+}
+
+// results of a reordered graph back to original ids: out[v] = val[cid[v]]
+template <class T>
+__global__ void k_unpermute(uint32_t n, const uint32_t* __restrict__ cid, const T* __restrict__ val,
+                            T* __restrict__ out) {
+    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v < n) out[v] = val[cid[v]];
+}
+
+tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* out, bool f64, cudaStream_t s) {
+    if (f64) k_unpermute<double><<<grid_for(n), kBlock, 0, s>>>(n, cid, (const double*)val, (double*)out);
+    else k_unpermute<uint32_t><<<grid_for(n), kBlock, 0, s>>>(n, cid, (const uint32_t*)val, (uint32_t*)out);
+    TIGR_CKL("unpermute");
+    return TIGR_OK;
 }
 
 // end of one iteration: decide whether to continue; sets the graph's WHILE condition

@@ -33,7 +33,7 @@ struct FqArgs {
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
 FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);
-unsigned relax_fq_grid(FqFn fn);
+unsigned relax_fq_grid(FqFn fn);   // persistent grid: SMs x resident blocks
 int relax_fq_threads();
 struct Ctl;
 tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s);
@@ -73,7 +73,10 @@ tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uin
 AssignFn assign_kernel(int layout, bool vec);
 
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
-                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters);
+                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
+                       const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order);
+// out[v] = val[cid[v]] (results of a reordered graph in original ids)
+tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* out, bool f64, cudaStream_t s);
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle);
 __global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
                        uint32_t* __restrict__ stamp, Ctl* ctl);

@@ -169,7 +169,10 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
 
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
     TIGR_CK(cudaEventRecord(t0, s));
-    k_init<<<grid_for(n), kBlock, 0, s>>>(algo, n, source, p.args.val, p.args.stamp, p.args.ctl, max_iters);
+    const tigr_graph* gg = vg->g;
+    k_init<<<grid_for(n), kBlock, 0, s>>>(algo, n, source, p.args.val, p.args.stamp, p.args.ctl, max_iters,
+                                          gg->reordered ? gg->perm_cid.as<uint32_t>() : nullptr,
+                                          gg->reordered ? gg->perm_order.as<uint32_t>() : nullptr);
     TIGR_CKL("init");
     if (p.bsp || p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
@@ -181,7 +184,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
     const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
     if (use_graph) {
-        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0), p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div : front,
+        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0), p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div * 16 : front,
                      p.bsp ? 1 : 0, o.collect_stats ? 1 : 0, p.comm ? 1 : 0, vg->lo, vg->hi};
         auto itg = ws.graphs.find(key);
         if (itg == ws.graphs.end()) {
@@ -414,7 +417,18 @@ tigr_status run_device(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const t
     const void* res = (algo == TIGR_PR) ? vg->ws.x.p : vg->ws.val.p;
     const size_t bytes = (size_t)g->n * (algo == TIGR_PR ? sizeof(double) : sizeof(uint32_t));
     if (out) {
-        TIGR_CK(cudaMemcpyAsync(out, res, bytes, out_is_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
+        TmpBuf tmp;
+        if (g->reordered) {  // values back to original ids
+            void* dst = out;
+            if (!out_is_device) {
+                TIGR_TRY(tmp.alloc(bytes, s));
+                dst = tmp.p;
+            }
+            TIGR_TRY(unpermute(g->n, g->perm_cid.as<uint32_t>(), res, dst, algo == TIGR_PR, s));
+            res = dst;
+        }
+        if (res != out)
+            TIGR_CK(cudaMemcpyAsync(out, res, bytes, out_is_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, s));
         TIGR_CK(cudaStreamSynchronize(s));
     }
     return rs;
