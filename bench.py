@@ -402,7 +402,7 @@ def main():
                          "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8}
 
     if not args.no_extra and not args.profile and world == 1:
-        result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy())
+        result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy(), peak)
 
     if rank == 0 and world == 1 and not args.no_cpu and not args.profile:
         dt, _ = cpu_pr_sample(rec, 2)
@@ -417,39 +417,70 @@ def main():
         dist.destroy_process_group()
 
 
-def per_algo(tigr, torch, rec, args, s, deg):
+def frontier_bytes(algo, st, n):
+    """Algorithmic bytes of one frontier run: per processed arc
+    s_e (+4 B weight for SSSP/SSWP) + 4 B target-value read; per successful update 4 B; per
+    active virtual node 4 B; per active node with arcs 12 B (value + row pair); per iteration
+    2 B per node (frontier flags read + cleared)."""
+    s_e = S_E + (4 if algo in ("sssp", "sswp") else 0)
+    return (st["edges_processed"] * (s_e + 4) + st["updates"] * 4 + st["active_vnodes"] * 4
+            + st["active_nodes"] * 12 + st["iterations"] * 2 * n)
+
+
+def per_algo(tigr, torch, rec, args, s, deg, peak):
     """Algorithm-only GTEPS for BFS/SSSP/CC/SSWP on the same scale-24 graph (weights 1-64;
-    CC on the symmetrised graph), device-timed; input-normalised GTEPS = arcs out of reached
-    vertices (CC: all 2m arcs) / time, plus processed-arc GTEPS from collect_stats."""
+    CC on the symmetrised graph), device-timed, on the in-degree-reordered graph
+    (tigr_graph_reorder; its one-off cost is reported as reorder_ms, like the virtual split's
+    transform time) and, for comparison, in canonical numbering (ms_canonical).
+    gteps_input = arcs out of reached vertices (CC: all 2m arcs) / time; gteps_processed =
+    arcs of active virtual nodes (collect_stats) / time; roofline_frac = algorithmic bytes /
+    relax-kernel time (CUDA events per relax launch) / measured HBM peak."""
     res = {}
     n, m = rec.n, rec.m
-    g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, weighted=True,
-                             stream=s)
-    vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+    g = vg = None
     for algo in ("bfs", "sssp", "sswp", "cc"):
-        if algo == "cc":
-            vg.free(); g.free()
-            g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, symmetrize=True,
-                                     stream=s)
+        sym = algo == "cc"
+        if g is None or sym:
+            if g is not None:
+                vg.free(); g.free(); vgc.free(); gc.free()
+            gc = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax,
+                                      weighted=not sym, symmetrize=sym, stream=s)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            g = tigr.tigr_graph_reorder(gc, stream=s)
+            e1.record(s)
+            torch.cuda.synchronize()
+            reorder_ms = e0.elapsed_time(e1)
             vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+            vgc = tigr.tigr_virtualize(gc, args.K, args.layout, stream=s)
         out = torch.empty(n, dtype=torch.int32, device="cuda")
         _, st = tigr.tigr_run(vg, algo, 0, out=out, stream=s, collect_stats=1, return_stats=True)
-        times = []
+        times, canon, relax = [], [], []
         for _ in range(3):
             _, st2 = tigr.tigr_run(vg, algo, 0, out=out, stream=s, return_stats=True)
             times.append(st2["ms_total"])
+            _, st3 = tigr.tigr_run(vgc, algo, 0, out=out, stream=s, return_stats=True)
+            canon.append(st3["ms_total"])
+            _, st4 = tigr.tigr_run(vg, algo, 0, out=out, stream=s, return_stats=True, time_kernels=1)
+            relax.append(st4["ms_relax"])
         t = statistics.median(times)
+        t_relax = statistics.median(relax)
         if algo == "cc":
             m_in = 2 * m
         else:
             reached = out.cpu().numpy().view(np.uint32)
             mask = reached != (0 if algo == "sswp" else 0xFFFFFFFF)
             m_in = int(deg[mask].sum())
-        res[algo] = {"ms": t, "iterations": st["iterations"], "gteps_input": m_in / (t * 1e-3) / 1e9,
+        nbytes = frontier_bytes(algo, st, n)
+        res[algo] = {"ms": t, "ms_relax": t_relax, "ms_canonical": statistics.median(canon), "reorder_ms": reorder_ms,
+                     "iterations": st["iterations"], "queue_iterations": st["queue_iterations"],
+                     "gteps_input": m_in / (t * 1e-3) / 1e9,
                      "gteps_processed": st["edges_processed"] / (t * 1e-3) / 1e9,
-                     "edges_processed": st["edges_processed"]}
-    vg.free()
-    g.free()
+                     "edges_processed": st["edges_processed"], "updates": st["updates"],
+                     "algorithmic_bytes": nbytes,
+                     "roofline_frac": nbytes / (t_relax * 1e-3) / 1e9 / peak,
+                     "roofline_frac_whole_run": nbytes / (t * 1e-3) / 1e9 / peak}
+    vg.free(); g.free(); vgc.free(); gc.free()
     # NEXT-1: pull PageRank on the in-CSR (same graph, 20 iterations), relax timed per launch
     g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, stream=s)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

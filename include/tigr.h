@@ -111,6 +111,7 @@ typedef struct {
     double ms_exchange;       /* device time of the multi-GPU exchanges (time_kernels) */
     uint32_t queue_iterations;/* iterations whose relax ran from the active-node queue (FRONTIER_AUTO/QUEUE) */
     uint32_t reserved;
+    uint64_t active_nodes;    /* sum over iterations of active nodes that own virtual nodes (FRONTIER_AUTO/QUEUE) */
 } tigr_stats;
 
 /* Fill *opts with the defaults above. */

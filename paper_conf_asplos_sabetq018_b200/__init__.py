@@ -53,7 +53,8 @@ class tigr_stats(ctypes.Structure):
     _fields_ = [("iterations", ctypes.c_uint32), ("relax_launches", ctypes.c_uint32),
                 ("edges_processed", ctypes.c_uint64), ("updates", ctypes.c_uint64),
                 ("active_vnodes", ctypes.c_uint64), ("ms_total", ctypes.c_double), ("ms_relax", ctypes.c_double),
-                ("ms_exchange", ctypes.c_double), ("queue_iterations", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+                ("ms_exchange", ctypes.c_double), ("queue_iterations", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
+                ("active_nodes", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -688,7 +688,7 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
     if (v == 0) {
         ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
-        ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0;
+        ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0; ctl->nodes = 0;
     }
 }
 
@@ -710,6 +710,7 @@ tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* ou
 // end of one iteration: decide whether to continue; sets the graph's WHILE condition
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle) {
     const uint32_t changed = ctl->changed;
+    ctl->nodes += ctl->qpack[ctl->it & 1u] >> 32;
     ctl->qpack[ctl->it & 1u] = 0ull;  // queue slot consumed by this iteration (frontier.cu)
     uint32_t cont = changed ? 1u : 0u;
     if (changed && ctl->it >= ctl->max_iters) { cont = 0; ctl->notconv = 1; }

@@ -257,6 +257,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         st->ms_total = ms;
         st->ms_relax = ms_relax;
         st->queue_iterations = c.queue_iters;
+        st->active_nodes = c.nodes;
     }
     if (c.notconv) return fail(TIGR_ENOTCONV, "max_iters reached before the fixed point");
     return TIGR_OK;

@@ -23,6 +23,7 @@ struct Ctl {
     unsigned long long qpack[2];
     uint32_t queue_iters;  // iterations the queue-driven (dynamic-mapping) path ran
     uint32_t pad2;
+    unsigned long long nodes;  // sum over iterations of active nodes with arcs (queue entries)
 };
 
 struct GraphKey {
