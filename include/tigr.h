@@ -79,9 +79,21 @@ typedef enum {
                                   Needs 4 | K (else EUNSUPPORTED). */
 } tigr_frontier;
 
+/* Multi-GPU merge of the replicated frontier values after each relax (SURVEY §8(e), §8(f)
+ * NEXT-2; exchange.cu).  PageRank always all-reduces its accumulator (every entry changes). */
+typedef enum {
+    TIGR_EXCHANGE_AUTO = 0,    /* per iteration: SPARSE while all ranks together changed at most
+                                  n/2 nodes, else DENSE (the same verdict on every rank) */
+    TIGR_EXCHANGE_DENSE = 1,   /* in-place MIN/MAX all-reduce of all n values; activity = moved */
+    TIGR_EXCHANGE_SPARSE = 2   /* every rank publishes {node, value} of the nodes it changed
+                                  (8 bytes each); every rank applies all lists with the relax's
+                                  atomic and activates the listed nodes */
+} tigr_exchange;
+
 typedef struct tigr_graph tigr_graph;   /* device CSR; owns its buffers */
 typedef struct tigr_vgraph tigr_vgraph; /* virtual node array + per-node info; refs its graph */
-typedef struct tigr_comm tigr_comm;     /* NCCL communicator + rank/size (multi-GPU) */
+typedef struct tigr_comm tigr_comm;     /* a rank's communicator (NCCL, or a thread group) */
+typedef struct tigr_comm_group tigr_comm_group; /* ranks that are threads of one process */
 
 typedef struct {
     uint32_t max_iters;   /* frontier algorithms: iteration cap (0 = n + 1); exceeded -> TIGR_ENOTCONV */
@@ -98,6 +110,7 @@ typedef struct {
     int time_kernels;     /* 1 = CUDA-event time every relax launch into tigr_stats.ms_relax (host loop) */
     tigr_comm* comm;      /* NULL = single GPU; else this rank's communicator (see tigr_vgraph_partition) */
     void* stream;         /* cudaStream_t */
+    int exchange;         /* tigr_exchange (multi-GPU frontier algorithms; default AUTO) */
 } tigr_run_opts;
 
 typedef struct {
@@ -110,7 +123,7 @@ typedef struct {
     double ms_relax;          /* device time of the relax launches (time_kernels) */
     double ms_exchange;       /* device time of the multi-GPU exchanges (time_kernels) */
     uint32_t queue_iterations;/* iterations whose relax ran from the active-node queue (FRONTIER_AUTO/QUEUE) */
-    uint32_t reserved;
+    uint32_t sparse_exchanges;/* multi-GPU: iterations merged by the sparse (changed-node list) exchange */
     uint64_t active_nodes;    /* sum over iterations of active nodes that own virtual nodes (FRONTIER_AUTO/QUEUE) */
 } tigr_stats;
 
@@ -264,6 +277,20 @@ tigr_status tigr_run(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tig
 tigr_status tigr_comm_unique_id(uint8_t id[128]);
 tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
 void tigr_comm_free(tigr_comm* comm);
+
+/* Thread-group communicator: nranks ranks that are threads of ONE process, each on its own
+ * current device (several ranks may share one GPU).  Exchanges read the peers' buffers directly
+ * (unified addressing; NVLink peer access is enabled between distinct GPUs at init) and a host
+ * barrier orders them; results are identical to the NCCL transport's.  Create the group once,
+ * then every rank thread calls tigr_comm_init_group with its rank: the call returns once all
+ * ranks have joined.  A rank that does not arrive at a barrier within TIGR_GROUP_TIMEOUT seconds
+ * (default 300) fails every rank's run with ENCCL instead of hanging.  The group may be freed
+ * after every rank has its tigr_comm (ranks keep the shared state alive).
+ * Errors: EINVAL (nranks outside [1, 16], rank outside [0, nranks), rank joined twice),
+ * EUNSUPPORTED (two ranks' GPUs without peer access). */
+tigr_status tigr_comm_group_create(int nranks, tigr_comm_group** out);
+tigr_status tigr_comm_init_group(tigr_comm_group* group, int rank, tigr_comm** out);
+void tigr_comm_group_free(tigr_comm_group* group);
 
 /* ----------------------------------------------------------------- misc ---- */
 

@@ -30,6 +30,8 @@ TIGR_OK, TIGR_EINVAL, TIGR_ENOMEM, TIGR_ECUDA, TIGR_ENCCL, TIGR_ERANGE, TIGR_ENO
 TIGR_BFS, TIGR_SSSP, TIGR_CC, TIGR_SSWP, TIGR_PR = 0, 1, 2, 3, 4
 TIGR_LAYOUT_CONSECUTIVE, TIGR_LAYOUT_STRIDED = 0, 1
 TIGR_FRONTIER_AUTO, TIGR_FRONTIER_DENSE, TIGR_FRONTIER_NONE, TIGR_FRONTIER_QUEUE = 0, 1, 2, 3
+TIGR_EXCHANGE_AUTO, TIGR_EXCHANGE_DENSE, TIGR_EXCHANGE_SPARSE = 0, 1, 2
+EXCHANGES = {"auto": TIGR_EXCHANGE_AUTO, "dense": TIGR_EXCHANGE_DENSE, "sparse": TIGR_EXCHANGE_SPARSE}
 ALGOS = {"bfs": TIGR_BFS, "sssp": TIGR_SSSP, "cc": TIGR_CC, "sswp": TIGR_SSWP, "pr": TIGR_PR}
 LAYOUTS = {"consecutive": TIGR_LAYOUT_CONSECUTIVE, "strided": TIGR_LAYOUT_STRIDED}
 INF = 0xFFFFFFFF
@@ -46,14 +48,14 @@ class tigr_run_opts(ctypes.Structure):
     _fields_ = [("max_iters", ctypes.c_uint32), ("pr_iters", ctypes.c_uint32), ("pr_damping", ctypes.c_double),
                 ("pr_dangling", ctypes.c_int), ("schedule", ctypes.c_int), ("frontier", ctypes.c_int),
                 ("use_graph", ctypes.c_int), ("collect_stats", ctypes.c_int), ("time_kernels", ctypes.c_int),
-                ("comm", ctypes.c_void_p), ("stream", ctypes.c_void_p)]
+                ("comm", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("exchange", ctypes.c_int)]
 
 
 class tigr_stats(ctypes.Structure):
     _fields_ = [("iterations", ctypes.c_uint32), ("relax_launches", ctypes.c_uint32),
                 ("edges_processed", ctypes.c_uint64), ("updates", ctypes.c_uint64),
                 ("active_vnodes", ctypes.c_uint64), ("ms_total", ctypes.c_double), ("ms_relax", ctypes.c_double),
-                ("ms_exchange", ctypes.c_double), ("queue_iterations", ctypes.c_uint32), ("reserved", ctypes.c_uint32),
+                ("ms_exchange", ctypes.c_double), ("queue_iterations", ctypes.c_uint32), ("sparse_exchanges", ctypes.c_uint32),
                 ("active_nodes", ctypes.c_uint64)]
 
     def as_dict(self):
@@ -89,6 +91,9 @@ _SIGS = {
     "tigr_comm_unique_id": (_I, [_P]),
     "tigr_comm_init": (_I, [_I, _I, _P, ctypes.POINTER(_P)]),
     "tigr_comm_free": (None, [_P]),
+    "tigr_comm_group_create": (_I, [_I, ctypes.POINTER(_P)]),
+    "tigr_comm_init_group": (_I, [_P, _I, ctypes.POINTER(_P)]),
+    "tigr_comm_group_free": (None, [_P]),
     "tigr_last_error": (ctypes.c_char_p, []),
     "tigr_launch_count": (_U64, []),
     "tigr_release_cached_memory": (None, []),
@@ -201,6 +206,29 @@ class Comm:
     def free(self):
         if self._ptr:
             _lib.tigr_comm_free(self._ptr)
+            self._ptr = ctypes.c_void_p(None)
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+class CommGroup:
+    """Owning wrapper of a tigr_comm_group* (ranks that are threads of this process)."""
+
+    def __init__(self, ptr, nranks):
+        self._ptr = ctypes.c_void_p(ptr)
+        self.nranks = nranks
+
+    @property
+    def ptr(self):
+        return self._ptr
+
+    def free(self):
+        if self._ptr:
+            _lib.tigr_comm_group_free(self._ptr)
             self._ptr = ctypes.c_void_p(None)
 
     def __del__(self):
@@ -379,6 +407,8 @@ def tigr_run(vg: VGraph, algo, source=0, opts: tigr_run_opts | None = None, out=
     for k, v in kw.items():
         if k == "comm":
             v = v.ptr if isinstance(v, Comm) else v
+        elif k == "exchange" and isinstance(v, str):
+            v = EXCHANGES[v]
         setattr(o, k, v)
     if stream is not None:
         o.stream = _stream_ptr(stream)
@@ -402,6 +432,21 @@ def tigr_comm_init(nranks: int, rank: int, uid: bytes) -> Comm:
     out = _P()
     _check(_lib.tigr_comm_init(nranks, rank, buf, ctypes.byref(out)))
     return Comm(out.value, nranks, rank)
+
+
+def tigr_comm_group_create(nranks: int) -> CommGroup:
+    """A group of `nranks` ranks that are threads of this process (one tigr_comm each)."""
+    out = _P()
+    _check(_lib.tigr_comm_group_create(nranks, ctypes.byref(out)))
+    return CommGroup(out.value, nranks)
+
+
+def tigr_comm_init_group(group: CommGroup, rank: int) -> Comm:
+    """Join `group` as `rank` on the calling thread's current CUDA device; returns once every
+    rank has joined (call it from each rank's thread)."""
+    out = _P()
+    _check(_lib.tigr_comm_init_group(group.ptr, rank, ctypes.byref(out)))
+    return Comm(out.value, group.nranks, rank)
 
 
 def tigr_last_error() -> str:

@@ -56,22 +56,29 @@ tigr_status cuda_fail(cudaError_t e, const char* what, const char* file, int lin
 // own cache of cudaMalloc'ed blocks (2 MiB granularity, best fit within +25%).  A freed block
 // records an event on the stream that last used it; reuse from another stream waits on it.
 namespace {
+// Blocks are keyed by device as well as size: one process may drive several GPUs (the
+// thread-group communicator, comm.cu), and a block must only be reused on the device it lives on.
 struct CachedBlock {
     void* p;
     size_t size;
     cudaStream_t s;
     cudaEvent_t ev;
+    int dev;
 };
 std::mutex g_cache_mu;
-std::multimap<size_t, CachedBlock> g_free;       // size -> block
-std::map<void*, size_t> g_live;                 // live block -> size
+std::multimap<std::pair<int, size_t>, CachedBlock> g_free;  // (device, size) -> block
+std::map<void*, std::pair<int, size_t>> g_live;             // live block -> (device, size)
 constexpr size_t kGran = 2u << 20;
 
 void release_cached_locked() {
+    int cur = 0;
+    cudaGetDevice(&cur);
     for (auto& kv : g_free) {
+        cudaSetDevice(kv.second.dev);
         cudaFree(kv.second.p);
         if (kv.second.ev) cudaEventDestroy(kv.second.ev);
     }
+    cudaSetDevice(cur);
     g_free.clear();
 }
 }  // namespace
@@ -80,14 +87,16 @@ void init_pool() {}
 
 void* cache_alloc(size_t nbytes, cudaStream_t s, cudaError_t* err) {
     const size_t size = ((nbytes ? nbytes : 1) + kGran - 1) / kGran * kGran;
+    int dev = 0;
+    cudaGetDevice(&dev);
     std::lock_guard<std::mutex> lk(g_cache_mu);
-    auto it = g_free.lower_bound(size);
-    if (it != g_free.end() && it->first <= size + size / 4 + kGran) {
+    auto it = g_free.lower_bound({dev, size});
+    if (it != g_free.end() && it->first.first == dev && it->first.second <= size + size / 4 + kGran) {
         CachedBlock b = it->second;
         g_free.erase(it);
         if (b.s != s && b.ev) cudaStreamWaitEvent(s, b.ev, 0);
         if (b.ev) cudaEventDestroy(b.ev);
-        g_live[b.p] = b.size;
+        g_live[b.p] = {dev, b.size};
         *err = cudaSuccess;
         return b.p;
     }
@@ -101,7 +110,7 @@ void* cache_alloc(size_t nbytes, cudaStream_t s, cudaError_t* err) {
     }
     *err = e;
     if (e != cudaSuccess) return nullptr;
-    g_live[p] = size;
+    g_live[p] = {dev, size};
     return p;
 }
 
@@ -110,11 +119,11 @@ void cache_free(void* p, cudaStream_t s) {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     auto it = g_live.find(p);
     if (it == g_live.end()) return;
-    CachedBlock b{p, it->second, s, nullptr};
+    CachedBlock b{p, it->second.second, s, nullptr, it->second.first};
     g_live.erase(it);
     if (cudaEventCreateWithFlags(&b.ev, cudaEventDisableTiming) == cudaSuccess) cudaEventRecord(b.ev, s);
     else b.ev = nullptr;
-    g_free.emplace(b.size, b);
+    g_free.emplace(std::make_pair(b.dev, b.size), b);
 }
 
 void cache_release_all() {
@@ -181,6 +190,9 @@ void partition_ranges(uint32_t n, const int64_t* rp, const uint32_t* vp, int nra
 tigr_status comm_unique_id(uint8_t id[128]);
 tigr_status comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
 void comm_free(tigr_comm* c);
+tigr_status comm_group_create(int nranks, tigr_comm_group** out);
+tigr_status comm_init_group(tigr_comm_group* g, int rank, tigr_comm** out);
+void comm_group_free(tigr_comm_group* g);
 
 namespace {
 
@@ -220,6 +232,7 @@ void tigr_run_opts_default(tigr_run_opts* o) {
     o->schedule = 0;
     o->frontier = TIGR_FRONTIER_AUTO;
     o->use_graph = 1;
+    o->exchange = TIGR_EXCHANGE_AUTO;
 }
 
 tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
@@ -476,6 +489,20 @@ tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], tigr_com
 }
 
 void tigr_comm_free(tigr_comm* c) { comm_free(c); }
+
+tigr_status tigr_comm_group_create(int nranks, tigr_comm_group** out) {
+    if (!out) return fail(TIGR_EINVAL, "comm_group_create: NULL");
+    *out = nullptr;
+    return comm_group_create(nranks, out);
+}
+
+tigr_status tigr_comm_init_group(tigr_comm_group* group, int rank, tigr_comm** out) {
+    if (!group || !out) return fail(TIGR_EINVAL, "comm_init_group: NULL");
+    *out = nullptr;
+    return comm_init_group(group, rank, out);
+}
+
+void tigr_comm_group_free(tigr_comm_group* g) { comm_group_free(g); }
 
 const char* tigr_last_error(void) { return t_err.c_str(); }
 

@@ -5,6 +5,7 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <memory>
 #include <string>
 
 #include "tigr.h"
@@ -119,10 +120,23 @@ struct tigr_graph {
     tigr::DevBuf perm_order; // uint32[n]: id here -> original id
 };
 
+namespace tigr { struct LocalGroup; }
+
+// A rank's communicator.  Two transports (comm.cu): NCCL (one process per GPU), or a thread
+// group (ranks are threads of one process; exchanges read the peers' buffers directly through
+// unified addressing / NVLink peer access, synchronised by a host barrier).
 struct tigr_comm {
-    void* nccl = nullptr;    // ncclComm_t
+    void* nccl = nullptr;    // ncclComm_t (NCCL transport)
+    std::shared_ptr<tigr::LocalGroup> local;  // thread-group transport
     int nranks = 1;
     int rank = 0;
+    int device = 0;
+    tigr::DevBuf scratch;    // exchange staging (grown on demand)
+    tigr::DevBuf counts;     // uint32[nranks] (NCCL count all-gather)
+};
+
+struct tigr_comm_group {
+    std::shared_ptr<tigr::LocalGroup> g;
 };
 
 struct tigr_vgraph;  // defined in vgraph.cuh

@@ -80,6 +80,19 @@ tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* ou
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle);
 __global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
                        uint32_t* __restrict__ stamp, Ctl* ctl);
+// multi-GPU merge of the replicated frontier values after a relax (exchange.cu)
+struct ExchangeArgs {
+    tigr_comm* comm;
+    int mode;          // tigr_exchange
+    int algo;
+    uint32_t n;
+    uint32_t* val;
+    uint32_t* prev;
+    uint32_t* stamp;
+    uint2* list;       // uint2[n] records of this rank (sparse mode)
+    Ctl* ctl;
+};
+tigr_status exchange_frontier(const ExchangeArgs& x, cudaStream_t s, bool* sparse_used);
 __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
                           double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl);
 __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double base, double damping,

@@ -82,6 +82,7 @@ RelaxArgs make_args(tigr_vgraph* vg) {
 
 struct FrontierPlan {
     RelaxFn relax;
+    ExchangeArgs xa;       // multi-GPU merge (exchange.cu), when comm
     FqFn fq = nullptr;     // queue / dynamic-mapping relax (frontier.cu); relax unused when set
     FqArgs fa;
     const tigr_vgraph* vg = nullptr;
@@ -95,7 +96,8 @@ struct FrontierPlan {
 
 // enqueue one iteration body; returns number of kernels it launches
 tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditionalHandle h, int use_handle,
-                         int* kernels, cudaEvent_t ev_a = nullptr, cudaEvent_t ev_b = nullptr) {
+                         int* kernels, cudaEvent_t ev_a = nullptr, cudaEvent_t ev_b = nullptr,
+                         uint32_t* sparse_count = nullptr) {
     int k = 0;
     if (p.bsp && !p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * p.n, cudaMemcpyDeviceToDevice, s));
@@ -110,13 +112,10 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
         ++k;
     }
     if (ev_b) TIGR_CK(cudaEventRecord(ev_b, s));
-    if (p.comm) {
-        TIGR_TRY(comm_allreduce(p.c, p.args.val, p.n, p.algo, s));
-        // the local `changed` flag is rank-local: reset it so k_control only sees k_diff's verdict
-        TIGR_CK(cudaMemsetAsync(&p.args.ctl->changed, 0, sizeof(uint32_t), s));
-        k_diff<<<grid_for(p.n), kBlock, 0, s>>>(p.n, p.args.val, (uint32_t*)p.args.prev, p.args.stamp, p.args.ctl);
-        TIGR_CK(cudaGetLastError());
-        ++k;
+    if (p.comm) {  // host loop only (never captured): the exchange decides on the host
+        bool sparse = false;
+        TIGR_TRY(exchange_frontier(p.xa, s, &sparse));  // its kernels count their own launches
+        if (sparse && sparse_count) ++*sparse_count;
     }
     if (p.fq) {  // next iteration's queue from the stamps just written
         TIGR_TRY(compact_launch(p.vg, p.args.ctl, 1, s));
@@ -157,6 +156,14 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     p.relax = relax_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0);
     if (!p.relax) return fail(TIGR_EUNSUPPORTED, "no relax kernel for this option combination");
     p.args = make_args(vg);
+    if (p.comm) {
+        if (o.exchange < TIGR_EXCHANGE_AUTO || o.exchange > TIGR_EXCHANGE_SPARSE)
+            return fail(TIGR_EINVAL, "run: unknown exchange mode");
+        if (o.exchange != TIGR_EXCHANGE_DENSE && !ws.xlist.p)
+            TIGR_TRY(ws.xlist.alloc(sizeof(uint2) * (n ? n : 1), s));
+        p.xa = ExchangeArgs{o.comm, o.exchange, algo, n, p.args.val, (uint32_t*)p.args.prev, p.args.stamp,
+                            ws.xlist.as<uint2>(), p.args.ctl};
+    }
     int per_thread = 1;
     if (RelaxFn mlp = relax_mlp_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0, &per_thread))
         p.relax = mlp;
@@ -179,7 +186,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s));  // iteration 1's queue
 
     int kpi = 0;
-    uint32_t launches = 0;
+    uint32_t launches = 0, sparse_exchanges = 0;
     double ms_relax = 0.0;
     // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
     const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
@@ -225,7 +232,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         for (;;) {
             int k = 0;
             TIGR_TRY(enqueue_body(p, s, 0, 0, &k, o.time_kernels ? ws.ev[2] : nullptr,
-                                  o.time_kernels ? ws.ev[3] : nullptr));
+                                  o.time_kernels ? ws.ev[3] : nullptr, &sparse_exchanges));
             count_launch(k);
             launches += p.grid ? 1 : 0;
             TIGR_CK(cudaMemcpyAsync(ws.ctl_host, p.args.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
@@ -258,6 +265,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         st->ms_relax = ms_relax;
         st->queue_iterations = c.queue_iters;
         st->active_nodes = c.nodes;
+        st->sparse_exchanges = sparse_exchanges;
     }
     if (c.notconv) return fail(TIGR_ENOTCONV, "max_iters reached before the fixed point");
     return TIGR_OK;

@@ -22,7 +22,7 @@ struct Ctl {
     // active-node queue of iteration it (frontier.cu): slot it&1 packs (entries << 32) | vnodes
     unsigned long long qpack[2];
     uint32_t queue_iters;  // iterations the queue-driven (dynamic-mapping) path ran
-    uint32_t pad2;
+    uint32_t xcount;       // multi-GPU sparse exchange: records this rank packed (exchange.cu)
     unsigned long long nodes;  // sum over iterations of active nodes with arcs (queue entries)
 };
 
@@ -56,6 +56,7 @@ struct Workspace {
     bool cid_ready = false;
     DevBuf qv;       // uint32[2][n]: active-node queue (node ids), one slot per iteration parity
     DevBuf qo;       // uint32[2][n]: first queue-space virtual node of each entry (exclusive prefix)
+    DevBuf xlist;    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
     DevBuf ctl;      // Ctl
     Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (thread-local, not owned)
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};

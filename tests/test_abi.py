@@ -70,8 +70,20 @@ def test_opts_default_and_version():
     import paper_conf_asplos_sabetq018_b200 as tigr
     o = tigr.tigr_run_opts_default()
     assert o.pr_iters == 20 and abs(o.pr_damping - 0.85) < 1e-15 and o.use_graph == 1
+    assert o.exchange == tigr.TIGR_EXCHANGE_AUTO
     assert "sm_100a" in tigr.tigr_version()
-    assert ctypes.sizeof(tigr.tigr_run_opts) == 56
+    # the ctypes mirrors of the option / stats structs match the C layout of include/tigr.h
+    os.makedirs(os.path.join(ROOT, "build"), exist_ok=True)
+    src = os.path.join(ROOT, "build", "abi_sizes.c")
+    exe = os.path.join(ROOT, "build", "abi_sizes")
+    with open(src, "w") as f:
+        f.write('#include <stdio.h>\n#include <stddef.h>\n#include "tigr.h"\n'
+                'int main(void){printf("%zu %zu %zu %zu\\n", sizeof(tigr_run_opts), sizeof(tigr_stats),'
+                ' offsetof(tigr_run_opts, exchange), offsetof(tigr_stats, sparse_exchanges));return 0;}\n')
+    subprocess.run(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), src, "-o", exe], check=True)
+    sizes = [int(x) for x in subprocess.run([exe], check=True, capture_output=True, text=True).stdout.split()]
+    assert sizes == [ctypes.sizeof(tigr.tigr_run_opts), ctypes.sizeof(tigr.tigr_stats),
+                     tigr.tigr_run_opts.exchange.offset, tigr.tigr_stats.sparse_exchanges.offset]
 
 
 def _build_c_example():
