@@ -29,6 +29,18 @@
 //
 // The relax itself is Alg. 2/3 unchanged: x = value[v]; for each arc alt = f(x, w); if
 // better(alt, value[nbr]) then atomic{Min,Max} and stamp nbr for the next iteration.
+//
+// BFS settled bitmap.  The relax is bound by the L1/L2 sector traffic of the random 4-byte
+// target gathers (profiles/r01_ncu_frontier_units.csv), so BFS first tests one bit of a 2 MB
+// bitmap (hot targets stay L1-resident) and gathers the level only for targets whose bit is
+// clear.  This is exact because BFS levels are final on first assignment under this
+// worklist, asynchronous schedule included: by induction, the nodes active in iteration it
+// all hold level it-1 (they were lowered to it-1 in iteration it-1, and every candidate of
+// iteration it-1 was it-1), so every candidate of iteration it equals it and can never lower
+// a value assigned earlier; on replicas the same holds rank-wide.  A bit is set next to an
+// atomicMin whose candidate beat the observed level (the level then ends at it, final), so a
+// set bit never hides an improvement; a stale clear bit (another SM's atomicOr not yet
+// visible through this SM's L1) only costs the level gather the plain test would have done.
 #include <algorithm>
 
 #include "devutil.cuh"
@@ -100,6 +112,7 @@ __device__ __forceinline__ void map_round(const uint32_t* __restrict__ qv, const
 template <int A, int LAYOUT, bool BSP, int B, bool STATS, int MINB, bool PRE>
 __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    const bool BITS = A == TIGR_BFS && f.settled != nullptr;  // uniform per launch
     const int lane = threadIdx.x & 31;
     const uint32_t it = a.ctl->it;
     const unsigned long long qp = a.ctl->qpack[it & 1u];
@@ -186,10 +199,20 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             kn[r] = k + 2 * step[r];
             if (STATS && act[r]) ++n_vn;
         }
+        // BFS with a settled bitmap (f.settled): the test reads one bit of a 2 MB array instead
+        // of the 4-byte level (see k_relax_fq's header); cur[q] = 1 means "settled, skip"
         auto gather8 = [&](const uint32_t* nb, uint32_t* cur) {
+            if (BITS) {  // settled targets read as level 0 (never improved); the rest read the level
+                uint32_t b[8];
 #pragma unroll
-            for (int q = 0; q < 8; ++q)
-                cur[q] = (nb[q] == kPad) ? 0u : a.val[nb[q]];
+                for (int q = 0; q < 8; ++q)
+                    b[q] = (nb[q] == kPad) ? 1u : (f.settled[nb[q] >> 5] >> (nb[q] & 31u)) & 1u;
+#pragma unroll
+                for (int q = 0; q < 8; ++q) cur[q] = b[q] ? 0u : a.val[nb[q]];
+                return;
+            }
+#pragma unroll
+            for (int q = 0; q < 8; ++q) cur[q] = (nb[q] == kPad) ? 0u : a.val[nb[q]];
         };
         auto apply8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv, const uint32_t* cur) {
 #pragma unroll
@@ -200,6 +223,8 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                 if (better<A>(alt, cur[q])) {
                     if (A == TIGR_SSWP) atomicMax(a.val + nb[q], alt);
                     else atomicMin(a.val + nb[q], alt);
+                    // the level becomes alt = it, final (see the header): mark it settled
+                    if (BITS) atomicOr(f.settled + (nb[q] >> 5), 1u << (nb[q] & 31u));
                     stamp_next[nb[q]] = it + 1;
                     touched = true;
                     if (STATS) ++n_upd;

@@ -30,6 +30,7 @@ struct FqArgs {
     const uint32_t* qo;   // uint32[2][n] queue-space first virtual node of each entry
     int mode;             // 0 = per iteration (queue if vnodes * dense_div < span), 1 = queue, 2 = dense
     uint32_t dense_div;
+    uint32_t* settled;    // BFS only: bit v set once v's level is final (nullptr: test the value)
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
 FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);

@@ -144,6 +144,12 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         if (e && front == TIGR_FRONTIER_AUTO) p.fa.mode = atoi(e);
         const char* d = getenv("TIGR_FQ_DIV");
         p.fa.dense_div = d ? (uint32_t)atoi(d) : 2u;
+        p.fa.settled = nullptr;
+        const char* bb = getenv("TIGR_BFS_BITS");  // development knob: 0 = test the levels instead
+        if (algo == TIGR_BFS && !(bb && atoi(bb) == 0)) {
+            if (!ws.settled.p) TIGR_TRY(ws.settled.alloc(sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
+            p.fa.settled = ws.settled.as<uint32_t>();
+        }
     } else if (front == TIGR_FRONTIER_QUEUE) {
         return fail(TIGR_EUNSUPPORTED, "frontier QUEUE needs the 16-byte-chunk layout (4 | K)");
     }
@@ -181,6 +187,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
                                           gg->reordered ? gg->perm_cid.as<uint32_t>() : nullptr,
                                           gg->reordered ? gg->perm_order.as<uint32_t>() : nullptr);
     TIGR_CKL("init");
+    if (p.fq && p.fa.settled) TIGR_CK(cudaMemsetAsync(p.fa.settled, 0, sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
     if (p.bsp || p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
     if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s));  // iteration 1's queue
@@ -191,7 +198,8 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
     const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
     if (use_graph) {
-        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0), p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div * 16 : front,
+        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0),
+                     p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div * 16 + (p.fa.settled ? 1 << 30 : 0) : front,
                      p.bsp ? 1 : 0, o.collect_stats ? 1 : 0, p.comm ? 1 : 0, vg->lo, vg->hi};
         auto itg = ws.graphs.find(key);
         if (itg == ws.graphs.end()) {

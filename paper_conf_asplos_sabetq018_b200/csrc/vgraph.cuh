@@ -56,6 +56,7 @@ struct Workspace {
     bool cid_ready = false;
     DevBuf qv;       // uint32[2][n]: active-node queue (node ids), one slot per iteration parity
     DevBuf qo;       // uint32[2][n]: first queue-space virtual node of each entry (exclusive prefix)
+    DevBuf settled;  // uint32[n/32+1]: BFS settled bitmap (frontier.cu)
     DevBuf xlist;    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
     DevBuf ctl;      // Ctl
     Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (thread-local, not owned)
