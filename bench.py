@@ -55,6 +55,7 @@ def parse():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-extra", action="store_true", help="skip the per-algorithm extras")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras, no e2e)")
+    ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs (per_config)")
     return ap.parse_args()
 
 
@@ -404,6 +405,9 @@ def main():
     if not args.no_extra and not args.profile and world == 1:
         result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy(), peak)
 
+    if not args.no_extra and not args.no_configs and not args.profile and world == 1:
+        result["per_config"] = per_config(tigr, torch, s, peak)
+
     if rank == 0 and world == 1 and not args.no_cpu and not args.profile:
         dt, _ = cpu_pr_sample(rec, 2)
         v = 2 * m / dt / 1e9
@@ -503,6 +507,72 @@ def per_algo(tigr, torch, rec, args, s, deg, peak):
                       "note": "SURVEY NEXT-1: in-CSR via tigr_graph_transpose, warp-segmented family sums"}
     vgt.free()
     gt.free()
+    return res
+
+
+def per_config(tigr, torch, s, peak):
+    """GTEPS per algorithm on the other BASELINE configs at one GPU (configs[1], [2], [4]; the
+    scale-24 graph is the main line and per_algo): cfg2 BFS + CC, cfg3 SSSP + SSWP at K = 4, 8,
+    16, 32, cfg5 BFS / SSSP / CC.  Arc list drawn on the device (tigr_rmat_coo), CSR built from
+    it (build_ms), virtual split at K (strided), then per algorithm: one stats run
+    (processed arcs), the median of 3 device-timed runs (CUDA-graph loop), and one run with
+    per-relax CUDA events.  gteps_input = arcs out of reached nodes (CC: all 2m arcs) / time."""
+    import graphgen
+
+    plan = {"cfg2": [("bfs", 8), ("cc", 8)],
+            "cfg3": [(a, K) for K in (4, 8, 16, 32) for a in ("sssp", "sswp")],
+            "cfg5": [("bfs", 8), ("sssp", 8), ("cc", 8)]}
+    res = {}
+    for cfg, runs in plan.items():
+        rec = graphgen.recipe(cfg)
+        n, m = rec.n, rec.m
+        src = torch.empty(m, dtype=torch.int32, device="cuda")
+        dst, w = torch.empty_like(src), torch.empty_like(src)
+        tigr.tigr_rmat_coo(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, src, dst, w, stream=s)
+        deg = torch.bincount(src.long(), minlength=n)
+        out = torch.empty(n, dtype=torch.int32, device="cuda")
+        entry = {"n": n, "m": m, "source": rec.source}
+        graphs = {}
+        for algo, K in runs:
+            sym = algo == "cc"
+            if sym not in graphs:
+                for g in graphs.values():
+                    g.free()
+                graphs.clear()
+                # one untimed build first: the block cache then holds buffers of these sizes
+                tigr.tigr_graph_from_coo(n, src, dst, None if sym else w, symmetrize=sym, stream=s).free()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                graphs[sym] = tigr.tigr_graph_from_coo(n, src, dst, None if sym else w, symmetrize=sym, stream=s)
+                e1.record(s)
+                torch.cuda.synchronize()
+                entry["build_ms_sym" if sym else "build_ms"] = e0.elapsed_time(e1)
+            vg = tigr.tigr_virtualize(graphs[sym], K, "strided", stream=s)
+            _, st = tigr.tigr_run(vg, algo, rec.source, out=out, stream=s, collect_stats=1, return_stats=True)
+            ts = []
+            for _ in range(3):
+                _, st2 = tigr.tigr_run(vg, algo, rec.source, out=out, stream=s, return_stats=True)
+                ts.append(st2["ms_total"])
+            _, st3 = tigr.tigr_run(vg, algo, rec.source, out=out, stream=s, return_stats=True, time_kernels=1)
+            t = statistics.median(ts)
+            if sym:
+                m_in = 2 * m
+            else:
+                reached = out != (0 if algo == "sswp" else -1)
+                m_in = int(deg[reached].sum().item())
+            nbytes = frontier_bytes(algo, st, n)
+            entry[f"{algo}_K{K}"] = {
+                "ms": t, "ms_relax": st3["ms_relax"], "iterations": st["iterations"],
+                "gteps_input": m_in / (t * 1e-3) / 1e9,
+                "gteps_processed": st["edges_processed"] / (t * 1e-3) / 1e9,
+                "roofline_frac": nbytes / (st3["ms_relax"] * 1e-3) / 1e9 / peak if st3["ms_relax"] else None,
+                "nv": vg.info()["nv"]}
+            vg.free()
+        for g in graphs.values():
+            g.free()
+        del src, dst, w, deg, out
+        torch.cuda.synchronize()
+        res[cfg] = entry
     return res
 
 
