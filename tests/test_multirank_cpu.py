@@ -7,6 +7,8 @@ every iteration by an all-reduce (MIN for BFS/SSSP/CC, MAX for SSWP, SUM for the
 accumulator); activity for the next iteration is "value changed by the exchange".  Here the
 per-rank relax is emulated in numpy (test code) and the all-reduce is a real gloo collective,
 so the partition rule and the exchange protocol are checked end to end against the oracle.
+Both merges are covered: the dense all-reduce and the sparse exchange of changed nodes
+(all-gather of {node, value} lists, apply, activate the union).
 """
 import os
 import socket
@@ -56,7 +58,27 @@ def _relax_range(o, vg, lo, hi, algo, val, active, xs=None):
     return new
 
 
-def _worker(rank, world, port, q):
+def _merge_sparse(algo, val, mine):
+    """Sparse exchange (exchange.cu, NEXT-2): every rank publishes {node, value} of the nodes its
+    relax improved; every rank applies all lists with the relax's own combine and activates
+    exactly the listed nodes (the union, identical on every rank)."""
+    changed = np.nonzero(mine != val)[0]
+    lists = [None] * dist.get_world_size()
+    dist.all_gather_object(lists, (changed.tolist(), mine[changed].tolist()))
+    nxt = mine.copy()
+    active = np.zeros(len(val), dtype=bool)
+    for ids, vals in lists:
+        ids = np.asarray(ids, dtype=np.int64)
+        vals = np.asarray(vals, dtype=np.int64)
+        if algo == "sswp":
+            np.maximum.at(nxt, ids, vals)
+        else:
+            np.minimum.at(nxt, ids, vals)
+        active[ids] = True
+    return nxt, active
+
+
+def _worker(rank, world, port, q, mode="dense"):
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import graphgen
@@ -98,10 +120,14 @@ def _worker(rank, world, port, q):
                 val[0] = 0
                 active[0] = True
             while True:
-                mine = torch.from_numpy(_relax_range(g, vg, mylo, myhi, algo, val, active))
-                dist.all_reduce(mine, op=dist.ReduceOp.MAX if algo == "sswp" else dist.ReduceOp.MIN)
-                nxt = mine.numpy()
-                active = nxt != val  # identical on every rank: no extra collective needed
+                mine = _relax_range(g, vg, mylo, myhi, algo, val, active)
+                if mode == "sparse":
+                    nxt, active = _merge_sparse(algo, val, mine)
+                else:
+                    t = torch.from_numpy(mine)
+                    dist.all_reduce(t, op=dist.ReduceOp.MAX if algo == "sswp" else dist.ReduceOp.MIN)
+                    nxt = t.numpy()
+                    active = nxt != val  # identical on every rank: no extra collective needed
                 val = nxt
                 if not active.any():
                     break
@@ -111,15 +137,15 @@ def _worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_partitioned_exchange_matches_oracle(world):
+@pytest.mark.parametrize("world,mode", [(2, "dense"), (3, "dense"), (2, "sparse"), (3, "sparse")])
+def test_partitioned_exchange_matches_oracle(world, mode):
     import graphgen
     import oracle
 
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, mode)) for r in range(world)]
     for p in procs:
         p.start()
     res = [q.get(timeout=600) for _ in range(world)]
