@@ -396,11 +396,15 @@ def main():
             tt = torch.tensor([tp], dtype=torch.float64, device="cuda")
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
             tp = float(tt.item())
-        result["e2e_streaming"] = {"value": 20 * m / (tp * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": tp,
-                                   "steps": ksteps, "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
-                                   "note": "H2D of step i+1 overlapped with step i on a copy stream"}
-        result["e2e"] = {"value": 20 * m / (te * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": te,
-                         "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8}
+        # e2e = the pipelined run (what a user streaming batches gets; every step's H2D and
+        # D2H are inside the timed region); the unpipelined one is reported beside it
+        result["e2e"] = {"value": 20 * m / (tp * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": tp,
+                         "steps": ksteps, "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
+                         "note": "H2D of step i+1 (pinned host arc list) overlapped with step i on a copy "
+                                 "stream; each step's ranks read back to pinned host memory"}
+        result["e2e_serial"] = {"value": 20 * m / (te * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": te,
+                                "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
+                                "note": "H2D -> step -> D2H with nothing overlapped"}
 
     if not args.no_extra and not args.profile and world == 1:
         result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy(), peak)
