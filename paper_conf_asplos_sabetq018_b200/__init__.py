@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtigr.so")
+LIB_PATH = os.environ.get("TIGR_LIB") or os.path.join(_HERE, "libtigr.so")  # TIGR_LIB: A/B builds (development)
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

@@ -233,25 +233,10 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         s_dstart[t] = wofs + v - tile_cnt;
         if (FILT && t == kST - 1) s_dstart[kMaxRadix] = wofs + v;  // the tile's kept items
     }
-    // decoupled look-back for this digit
-    if (t < radix) {
-        uint64_t excl = 0;
-        if (tile > 0) {
-            for (int64_t p = (int64_t)tile - 1; p >= 0; --p) {
-                const volatile uint64_t* sp = reinterpret_cast<const volatile uint64_t*>(&status[(uint64_t)p * kMaxRadix + t]);
-                uint64_t st = *sp;
-                while ((st >> 48) != epoch || (st & (3ull << 46)) == 0) st = *sp;
-                excl += st & kValMask;
-                if (st & kFlagInc) break;
-            }
-            *reinterpret_cast<volatile uint64_t*>(&status[(uint64_t)tile * kMaxRadix + t]) =
-                (epoch << 48) | kFlagInc | (excl + tile_cnt);
-        }
-        s_gofs[t] = digit_base[t] + excl;
-    }
     asm volatile("cp.async.wait_all;" ::: "memory");
     __syncthreads();
-    // reorder the tile by digit in shared memory
+    // reorder the tile by digit in shared memory (needs no global offset: done before the
+    // look-back, so that the predecessors have had that much longer to publish)
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
         const uint32_t li = wp * (SI * 32) + r * 32 + lane;
@@ -261,6 +246,26 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
             s_key[lp] = key[r];
             s_val[lp] = s_vin[li];
         }
+    }
+    // decoupled look-back for this digit (a short sleep between polls keeps the spinning
+    // blocks from flooding L2 while the predecessor tiles finish)
+    if (t < radix) {
+        uint64_t excl = 0;
+        if (tile > 0) {
+            for (int64_t p = (int64_t)tile - 1; p >= 0; --p) {
+                const volatile uint64_t* sp = reinterpret_cast<const volatile uint64_t*>(&status[(uint64_t)p * kMaxRadix + t]);
+                uint64_t st = *sp;
+                while ((st >> 48) != epoch || (st & (3ull << 46)) == 0) {
+                    __nanosleep(64);
+                    st = *sp;
+                }
+                excl += st & kValMask;
+                if (st & kFlagInc) break;
+            }
+            *reinterpret_cast<volatile uint64_t*>(&status[(uint64_t)tile * kMaxRadix + t]) =
+                (epoch << 48) | kFlagInc | (excl + tile_cnt);
+        }
+        s_gofs[t] = digit_base[t] + excl;
     }
     __syncthreads();
     const uint32_t nvalid = FILT ? s_dstart[kMaxRadix] : cnt;
