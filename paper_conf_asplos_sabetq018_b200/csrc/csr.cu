@@ -8,6 +8,8 @@
 // From an arc list the CSR is built by a stable radix sort on the source (sort.cu), so the
 // arcs of a source keep their input order: the canonical CSR, element-identical to a stable
 // counting sort.
+#include <algorithm>
+
 #include "internal.cuh"
 
 namespace tigr {
@@ -83,37 +85,76 @@ __global__ void k_padded_to_csr(const int64_t* __restrict__ rp, uint32_t n, uint
     }
 }
 
-// canonical arc list (src, dst, w) of a device CSR: thread per node for short segments, a
-// whole warp per long one (ballot loop), so every write is coalesced
-__global__ void k_expand_arcs(const int64_t* __restrict__ rp, const uint32_t* __restrict__ cptr, uint32_t n,
-                              const uint32_t* __restrict__ col, const uint32_t* __restrict__ wt,
-                              uint32_t* __restrict__ src, uint32_t* __restrict__ dst, uint32_t* __restrict__ w) {
-    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
-    const int lane = threadIdx.x & 31;
-    uint64_t beg = 0, cb = 0;
-    uint32_t d = 0;
-    if (v < n) { beg = (uint64_t)rp[v]; d = (uint32_t)(rp[v + 1] - rp[v]); cb = (uint64_t)cptr[v] * kChunk; }
-    const bool big = d > 32;
-    if (!big)
-        for (uint32_t p = 0; p < d; ++p) {
-            src[beg + p] = v;
-            dst[beg + p] = col[cb + p];
-            if (w) w[beg + p] = wt[cb + p];
-        }
-    uint32_t mask = __ballot_sync(0xffffffffu, big);
-    while (mask) {
-        const int l = __ffs(mask) - 1;
-        mask &= mask - 1;
-        const uint64_t b = __shfl_sync(0xffffffffu, beg, l);
-        const uint64_t c = __shfl_sync(0xffffffffu, cb, l);
-        const uint32_t dd = __shfl_sync(0xffffffffu, d, l);
-        const uint32_t vv = __shfl_sync(0xffffffffu, v, l);
-        for (uint32_t p = lane; p < dd; p += 32) {
-            src[b + p] = vv;
-            dst[b + p] = col[c + p];
-            if (w) w[b + p] = wt[c + p];
-        }
+// canonical arc list (src, dst, w) of a device CSR, arc-parallel (balanced whatever the
+// degrees: one hub's 371 K arcs are spread over many blocks).  Block b owns arc positions
+// [b*kExpTile, (b+1)*kExpTile); one thread finds the node owning the first position (binary
+// search over row_ptr), the block stages the row offsets of the nodes its tile spans in shared
+// memory, and each arc finds its source there by a short binary search.  Tiles that span more
+// nodes than the stage holds (long runs of zero-degree nodes) search row_ptr in global memory.
+constexpr uint32_t kExpTile = 2048;
+constexpr uint32_t kExpStage = 2048;
+
+__device__ __forceinline__ uint32_t owner_of(const int64_t* __restrict__ rp, uint32_t lo, uint32_t hi, uint64_t p) {
+    // last v in [lo, hi] with rp[v] <= p
+    while (lo < hi) {
+        const uint32_t mid = lo + (hi - lo + 1) / 2;
+        if ((uint64_t)rp[mid] <= p) lo = mid; else hi = mid - 1;
     }
+    return lo;
+}
+
+__global__ void __launch_bounds__(256) k_expand_arcs(const int64_t* __restrict__ rp, const uint32_t* __restrict__ cptr,
+                                                     uint32_t n, uint64_t m, const uint32_t* __restrict__ col,
+                                                     const uint32_t* __restrict__ wt, uint32_t* __restrict__ src,
+                                                     uint32_t* __restrict__ dst, uint32_t* __restrict__ w) {
+    __shared__ int64_t s_rp[kExpStage + 1];
+    __shared__ uint32_t s_v[2];
+    for (uint64_t t0 = (uint64_t)blockIdx.x * kExpTile; t0 < m; t0 += (uint64_t)gridDim.x * kExpTile) {
+        const uint64_t t1 = min(t0 + kExpTile, m);
+        if (threadIdx.x == 0) s_v[0] = owner_of(rp, 0, n - 1, t0);
+        if (threadIdx.x == 1) s_v[1] = owner_of(rp, 0, n - 1, t1 - 1);
+        __syncthreads();
+        const uint32_t v0 = s_v[0], v1 = s_v[1];
+        const bool staged = v1 - v0 < kExpStage;
+        if (staged)
+            for (uint32_t i = threadIdx.x; i <= v1 - v0; i += blockDim.x) s_rp[i] = rp[v0 + i];
+        __syncthreads();
+        for (uint64_t p = t0 + threadIdx.x; p < t1; p += blockDim.x) {
+            uint32_t v;
+            int64_t beg;
+            if (staged) {
+                uint32_t lo = 0, hi = v1 - v0;
+                while (lo < hi) {
+                    const uint32_t mid = lo + (hi - lo + 1) / 2;
+                    if ((uint64_t)s_rp[mid] <= p) lo = mid; else hi = mid - 1;
+                }
+                v = v0 + lo;
+                beg = s_rp[lo];
+            } else {
+                v = owner_of(rp, v0, v1, p);
+                beg = rp[v];
+            }
+            const uint64_t c = (uint64_t)cptr[v] * kChunk + (p - (uint64_t)beg);
+            src[p] = v;
+            dst[p] = col[c];
+            if (w) w[p] = wt[c];
+        }
+        __syncthreads();  // s_rp / s_v reused by the next tile
+    }
+}
+
+tigr_status expand_arcs(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w, cudaStream_t s) {
+    if (g->m == 0 || g->n == 0) return TIGR_OK;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t tiles = (g->m + kExpTile - 1) / kExpTile;
+    const unsigned grid = (unsigned)std::min<uint64_t>(tiles, (uint64_t)sms * 8);
+    k_expand_arcs<<<grid, 256, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), g->n, g->m,
+                                       g->col.as<uint32_t>(), g->weighted ? g->wt.as<uint32_t>() : nullptr, src, dst,
+                                       w);
+    TIGR_CKL("expand arcs");
+    return TIGR_OK;
 }
 
 // ---- UDT (physical uniform-degree-tree transformation, §3.2 Alg. 1) ----
@@ -332,10 +373,7 @@ tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_gra
     TIGR_TRY(src.alloc(sizeof(uint32_t) * (m ? m : 1), s));
     TIGR_TRY(dst.alloc(sizeof(uint32_t) * (m ? m : 1), s));
     if (g->weighted) TIGR_TRY(w.alloc(sizeof(uint32_t) * (m ? m : 1), s));
-    k_expand_arcs<<<grid_for(g->n), kBlock, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), g->n,
-                                                    g->col.as<uint32_t>(), g->wt.as<uint32_t>(), src.as<uint32_t>(),
-                                                    dst.as<uint32_t>(), g->weighted ? w.as<uint32_t>() : nullptr);
-    TIGR_CKL("expand arcs");
+    TIGR_TRY(expand_arcs(g, src.as<uint32_t>(), dst.as<uint32_t>(), g->weighted ? w.as<uint32_t>() : nullptr, s));
     tigr_graph* t = nullptr;
     TIGR_TRY(graph_from_coo_device(g->n, m, dst.as<uint32_t>(), src.as<uint32_t>(),
                                    g->weighted ? w.as<uint32_t>() : nullptr, 0, s, &t));
@@ -385,10 +423,7 @@ tigr_status graph_reorder_device(const tigr_graph* g, cudaStream_t s, tigr_graph
     TIGR_TRY(src.alloc(sizeof(uint32_t) * (m ? m : 1), s));
     TIGR_TRY(dst.alloc(sizeof(uint32_t) * (m ? m : 1), s));
     if (g->weighted) TIGR_TRY(w.alloc(sizeof(uint32_t) * (m ? m : 1), s));
-    k_expand_arcs<<<grid_for(n), kBlock, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), n,
-                                                 g->col.as<uint32_t>(), g->wt.as<uint32_t>(), src.as<uint32_t>(),
-                                                 dst.as<uint32_t>(), g->weighted ? w.as<uint32_t>() : nullptr);
-    TIGR_CKL("reorder expand");
+    TIGR_TRY(expand_arcs(g, src.as<uint32_t>(), dst.as<uint32_t>(), g->weighted ? w.as<uint32_t>() : nullptr, s));
     if (m) {
         k_relabel<<<capped_grid(m), kBlock, 0, s>>>(src.as<uint32_t>(), dst.as<uint32_t>(), m, cid.as<uint32_t>());
         TIGR_CKL("reorder relabel");
