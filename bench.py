@@ -192,9 +192,23 @@ def run_reference(args, rank, world):
         "config": config_obj(args, rec),
         "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                          "sample": "1 of the 20 PageRank iterations per step on the full cfg4 graph "
-                                   "(oracle/oracle.c or_pagerank, single thread)"},
+                                   "(oracle/oracle.c or_pagerank, single thread)", "host": host_cpu()},
         "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
+
+
+def host_cpu():
+    """'<model>, <N> logical cores' of this host (the oracle uses 1 of them)."""
+    model = "unknown CPU"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return f"{model}, {os.cpu_count()} logical cores (oracle on 1)"
 
 
 def metric_name(args):
@@ -324,13 +338,14 @@ def main():
 
     result = {
         "metric": metric_name(args), "value": gteps, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": t_step, "higher_is_better": True,
+        "warmup": args.warmup, "ms_per_step": t_step, "ms_per_step_median": statistics.median(step_ms),
+        "ms_per_step_min": min(step_ms), "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": config_obj(args, rec),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                      "traffic": traffic, "kernel": "k_relax_pr_cid (PageRank push relax, pr.cu)",
                      "algorithmic_bytes_per_launch": bytes_launch, "avg_launch_ms": relax_avg_ms,
-                     "peak_source": peak_src},
+                     "peak_source": peak_src, "frac_vs_8000_GBps": achieved / 8000.0},
         "breakdown_ms": {"csr_build": statistics.mean(phase[0]), "virtualize": statistics.mean(phase[1]),
                          "pagerank_20it": statistics.mean(phase[2]), "relax_total": relax_ms / args.steps},
         "algo_gteps": 20 * m / (statistics.mean(phase[2]) * 1e-3) / 1e9,
@@ -417,7 +432,8 @@ def main():
         v = 2 * m / dt / 1e9
         result["cpu_baseline"] = {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                                   "sample": "2 of the 20 PageRank iterations on the full cfg4 graph "
-                                            f"({dt:.1f} s; oracle/oracle.c or_pagerank, single thread)"}
+                                            f"({dt:.1f} s; oracle/oracle.c or_pagerank, single thread)",
+                                  "host": host_cpu()}
     if rank == 0:
         print(json.dumps(result), flush=True)
     if world > 1:
