@@ -208,3 +208,35 @@ def test_exchange_modes_single_rank_nccl(tigr, exchange):
             assert st["sparse_exchanges"] == st["iterations"]
     assert np.array_equal(tigr.tigr_run(vgs, "cc", comm=comm, exchange=exchange), want["cc"])
     comm.free()
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("exchange", ["sparse", "auto"])
+def test_group_cfg2_full(tigr, exchange):
+    """Config 2 at full size (R-MAT scale 20: 16.8 M arcs, 33.6 M symmetrised) on 4 ranks:
+    BFS and CC bit-exact on every rank, plus SSSP through the source-range build."""
+    rec = graphgen.recipe("cfg2")
+    src, dst, w = graphgen.generate(rec)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    want = {"bfs": oracle.bfs(o, 0), "sssp": oracle.sssp(o, 0), "cc": oracle.cc(rec.n, src, dst)}
+    P = 4
+    cuts = tigr.tigr_coo_source_cuts(rec.n, src, dst, P)
+
+    def body(r, comm, s):
+        g = tigr.tigr_graph_from_coo(rec.n, src, dst, w, stream=s)
+        vg = tigr.tigr_virtualize(g, 8, "strided", stream=s)
+        tigr.tigr_vgraph_partition(vg, P, r)
+        gs = tigr.tigr_graph_from_coo(rec.n, src, dst, None, symmetrize=True, stream=s)
+        vgs = tigr.tigr_virtualize(gs, 8, "strided", stream=s)
+        tigr.tigr_vgraph_partition(vgs, P, r)
+        gp = tigr.tigr_graph_from_coo_part(rec.n, src, dst, w, src_lo=int(cuts[r]), src_hi=int(cuts[r + 1]),
+                                           stream=s)
+        vgp = tigr.tigr_virtualize(gp, 8, "strided", stream=s)
+        return {"bfs": tigr.tigr_run(vg, "bfs", 0, comm=comm, exchange=exchange, stream=s),
+                "cc": tigr.tigr_run(vgs, "cc", comm=comm, exchange=exchange, stream=s),
+                "sssp": tigr.tigr_run(vgp, "sssp", 0, comm=comm, exchange=exchange, stream=s)}
+
+    res = _run_group(tigr, P, body)
+    for rank, got in enumerate(res):
+        for a in ("bfs", "sssp", "cc"):
+            assert np.array_equal(got[a], want[a]), (rank, a)
