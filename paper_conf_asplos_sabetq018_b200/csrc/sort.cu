@@ -285,7 +285,31 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
 // degrees from the runs of the sorted keys: start/end of each present key
 __global__ void k_runs(const uint32_t* __restrict__ key, uint64_t M, uint32_t* __restrict__ start,
                        uint32_t* __restrict__ end) {
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
+    // four keys per thread and step (one 16-byte load; neighbours across the group from the
+    // adjacent lanes' registers, the first / last lane reads one extra key)
+    const uint64_t M4 = M / 4;
+    const int lane = threadIdx.x & 31;
+    for (uint64_t b = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); b < M4;
+         b += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t g = b + lane;
+        uint4 k4 = make_uint4(0, 0, 0, 0);
+        if (g < M4) k4 = reinterpret_cast<const uint4*>(key)[g];
+        uint32_t prev = __shfl_up_sync(0xffffffffu, k4.w, 1);
+        uint32_t next = __shfl_down_sync(0xffffffffu, k4.x, 1);
+        if (g < M4) {
+            const uint64_t i0 = 4 * g;
+            if (lane == 0) prev = i0 ? key[i0 - 1] : ~k4.x;
+            if (lane == 31 || g + 1 == M4) next = (i0 + 4 < M) ? key[i0 + 4] : ~k4.w;
+            const uint32_t k[6] = {prev, k4.x, k4.y, k4.z, k4.w, next};
+#pragma unroll
+            for (int q = 1; q <= 4; ++q) {
+                if (k[q - 1] != k[q]) start[k[q]] = (uint32_t)(i0 + q - 1);
+                if (k[q + 1] != k[q]) end[k[q]] = (uint32_t)(i0 + q);
+            }
+        }
+    }
+    for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
+         i += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t k = key[i];
         if (i == 0 || key[i - 1] != k) start[k] = (uint32_t)i;
         if (i + 1 == M || key[i + 1] != k) end[k] = (uint32_t)(i + 1);
@@ -303,10 +327,31 @@ template <bool W>
 __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>::T* __restrict__ val, uint64_t M,
                         const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ cptr,
                         uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
-    for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
+    typedef typename ValT<W>::T VT;
+    // four arcs per thread and step: 16-byte key loads, all node-record reads in flight together
+    const uint64_t M4 = M / 4;
+    for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < M4; g += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 k4 = reinterpret_cast<const uint4*>(key)[g];
+        const uint32_t v[4] = {k4.x, k4.y, k4.z, k4.w};
+        VT x[4];
+        uint64_t base[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            x[q] = val[4 * g + q];
+            base[q] = (uint64_t)cptr[v[q]] * kChunk - (uint64_t)row_ptr[v[q]];
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const uint64_t pos = base[q] + 4 * g + q;
+            col[pos] = (uint32_t)x[q];
+            if constexpr (W) wt[pos] = (uint32_t)(x[q] >> 32);
+        }
+    }
+    for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
+         i += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t v = key[i];
         const uint64_t pos = (uint64_t)cptr[v] * kChunk + (i - (uint64_t)row_ptr[v]);
-        const typename ValT<W>::T x = val[i];
+        const VT x = val[i];
         col[pos] = (uint32_t)x;
         if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
     }
