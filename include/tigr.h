@@ -85,9 +85,13 @@ typedef enum {
     TIGR_EXCHANGE_AUTO = 0,    /* per iteration: SPARSE while all ranks together changed at most
                                   n/2 nodes, else DENSE (the same verdict on every rank) */
     TIGR_EXCHANGE_DENSE = 1,   /* in-place MIN/MAX all-reduce of all n values; activity = moved */
-    TIGR_EXCHANGE_SPARSE = 2   /* every rank publishes {node, value} of the nodes it changed
+    TIGR_EXCHANGE_SPARSE = 2,  /* every rank publishes {node, value} of the nodes it changed
                                   (8 bytes each); every rank applies all lists with the relax's
                                   atomic and activates the listed nodes */
+    TIGR_EXCHANGE_FUSED = 3    /* no exchange step: the relax kernel applies each improvement to
+                                  every peer's replica too (peer atomics, over NVLink between GPUs)
+                                  and activates it there; a barrier ends each iteration.
+                                  Thread-group communicator and 4 | K only (else EUNSUPPORTED). */
 } tigr_exchange;
 
 typedef struct tigr_graph tigr_graph;   /* device CSR; owns its buffers */

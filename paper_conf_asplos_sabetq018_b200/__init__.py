@@ -30,8 +30,9 @@ TIGR_OK, TIGR_EINVAL, TIGR_ENOMEM, TIGR_ECUDA, TIGR_ENCCL, TIGR_ERANGE, TIGR_ENO
 TIGR_BFS, TIGR_SSSP, TIGR_CC, TIGR_SSWP, TIGR_PR = 0, 1, 2, 3, 4
 TIGR_LAYOUT_CONSECUTIVE, TIGR_LAYOUT_STRIDED = 0, 1
 TIGR_FRONTIER_AUTO, TIGR_FRONTIER_DENSE, TIGR_FRONTIER_NONE, TIGR_FRONTIER_QUEUE = 0, 1, 2, 3
-TIGR_EXCHANGE_AUTO, TIGR_EXCHANGE_DENSE, TIGR_EXCHANGE_SPARSE = 0, 1, 2
-EXCHANGES = {"auto": TIGR_EXCHANGE_AUTO, "dense": TIGR_EXCHANGE_DENSE, "sparse": TIGR_EXCHANGE_SPARSE}
+TIGR_EXCHANGE_AUTO, TIGR_EXCHANGE_DENSE, TIGR_EXCHANGE_SPARSE, TIGR_EXCHANGE_FUSED = 0, 1, 2, 3
+EXCHANGES = {"auto": TIGR_EXCHANGE_AUTO, "dense": TIGR_EXCHANGE_DENSE, "sparse": TIGR_EXCHANGE_SPARSE,
+             "fused": TIGR_EXCHANGE_FUSED}
 ALGOS = {"bfs": TIGR_BFS, "sssp": TIGR_SSSP, "cc": TIGR_CC, "sswp": TIGR_SSWP, "pr": TIGR_PR}
 LAYOUTS = {"consecutive": TIGR_LAYOUT_CONSECUTIVE, "strided": TIGR_LAYOUT_STRIDED}
 INF = 0xFFFFFFFF

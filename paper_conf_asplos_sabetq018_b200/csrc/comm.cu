@@ -38,6 +38,7 @@ struct LocalGroup {
     uint64_t gen = 0;
     bool broken = false;
     std::vector<const void*> ptr;  // published device pointers (one per rank)
+    std::vector<const void*> ptrk; // published pointer sets (kMaxSet per rank)
     std::vector<uint32_t> cnt;     // published counts
     std::vector<int> dev;          // device of each rank
     std::vector<char> joined;
@@ -184,6 +185,7 @@ tigr_status comm_group_create(int nranks, tigr_comm_group** out) {
     auto g = std::make_shared<LocalGroup>();
     g->P = nranks;
     g->ptr.assign(nranks, nullptr);
+    g->ptrk.assign((size_t)nranks * 8, nullptr);
     g->cnt.assign(nranks, 0);
     g->dev.assign(nranks, -1);
     g->joined.assign(nranks, 0);
@@ -317,6 +319,25 @@ tigr_status comm_share_lists(tigr_comm* c, const void* mine, const uint32_t* cou
         off += counts[r];
     }
     return nccl_check(g_nccl.groupEnd(), "ncclGroupEnd");
+}
+
+// every rank's set of k (<= 8) device pointers: all[r * k + i] (thread group only)
+tigr_status comm_share_ptrs(tigr_comm* c, const void* const* mine, int k, const void** all) {
+    if (!c->local) return fail(TIGR_EUNSUPPORTED, "pointer exchange needs the thread-group communicator");
+    if (k < 1 || k > 8) return fail(TIGR_EINVAL, "comm_share_ptrs: 1..8 pointers");
+    LocalGroup& g = *c->local;
+    for (int i = 0; i < k; ++i) g.ptrk[(size_t)c->rank * 8 + i] = mine[i];
+    TIGR_TRY(g.barrier());
+    for (int r = 0; r < g.P; ++r)
+        for (int i = 0; i < k; ++i) all[r * k + i] = g.ptrk[(size_t)r * 8 + i];
+    return g.barrier();  // slots may be rewritten after this
+}
+
+// host barrier of the thread group after this rank's stream has drained (no-op for NCCL)
+tigr_status comm_sync_barrier(tigr_comm* c, cudaStream_t s) {
+    if (!c->local) return TIGR_OK;
+    TIGR_CK(cudaStreamSynchronize(s));
+    return c->local->barrier();
 }
 
 // the lists shared by comm_share_lists are no longer read by this rank's stream

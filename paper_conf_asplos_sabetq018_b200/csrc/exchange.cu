@@ -33,6 +33,8 @@ tigr_status comm_allgather_count(tigr_comm* c, const uint32_t* dev_count, uint32
 tigr_status comm_share_lists(tigr_comm* c, const void* mine, const uint32_t* counts, const void** ptrs,
                              cudaStream_t s);
 tigr_status comm_release_lists(tigr_comm* c, cudaStream_t s);
+tigr_status comm_share_ptrs(tigr_comm* c, const void* const* mine, int k, const void** all);
+tigr_status comm_sync_barrier(tigr_comm* c, cudaStream_t s);
 
 namespace {
 
@@ -89,6 +91,13 @@ __global__ void k_lists_prev(Lists L, const uint32_t* __restrict__ val, uint32_t
     }
 }
 
+// fused exchange, end of an iteration: this rank's verdict is every rank's flag for it
+__global__ void k_fused_settle(Ctl* ctl) {
+    const uint32_t slot = ctl->it & 1u;
+    ctl->changed = ctl->xchanged[slot];
+    ctl->xchanged[slot] = 0;  // no rank writes this slot again before iteration it + 2
+}
+
 tigr_status dense(const ExchangeArgs& x, cudaStream_t s) {
     TIGR_TRY(comm_allreduce(x.comm, x.val, x.n, x.algo, s));
     // the local `changed` flag is rank-local: reset it so k_control only sees k_diff's verdict
@@ -99,6 +108,44 @@ tigr_status dense(const ExchangeArgs& x, cudaStream_t s) {
 }
 
 }  // namespace
+
+// Fused exchange (TIGR_EXCHANGE_FUSED; thread-group transport).  There is no exchange step:
+// the relax itself applies each improvement to every peer's replica and stamp array
+// (frontier.cu push_peers) and raises every rank's xchanged flag.  What remains per iteration
+// is ordering: a barrier once every rank's relax has drained (all remote updates have landed),
+// then each rank reads the common verdict.  Before the first iteration every replica must be
+// initialised (barrier after init); in BSP mode the snapshot is taken between two barriers so
+// that no peer's update of the new iteration leaks into it.
+tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, DevBuf& peers_buf,
+                        cudaStream_t s, const FusedPeers** out) {
+    if (!c->local) return fail(TIGR_EUNSUPPORTED, "fused exchange needs the thread-group communicator");
+    if (c->nranks > kMaxPeers) return fail(TIGR_EUNSUPPORTED, "fused exchange: more than 16 ranks");
+    const void* mine[3] = {val, stamp, ctl};
+    const void* all[3 * kMaxPeers] = {};
+    TIGR_TRY(comm_share_ptrs(c, mine, 3, all));
+    FusedPeers h{};
+    h.P = c->nranks;
+    h.me = c->rank;
+    for (int r = 0; r < c->nranks; ++r) {
+        h.val[r] = const_cast<uint32_t*>(static_cast<const uint32_t*>(all[3 * r]));
+        h.stamp[r] = const_cast<uint32_t*>(static_cast<const uint32_t*>(all[3 * r + 1]));
+        h.ctl[r] = const_cast<Ctl*>(static_cast<const Ctl*>(all[3 * r + 2]));
+    }
+    if (!peers_buf.p) TIGR_TRY(peers_buf.alloc(sizeof(FusedPeers), s));
+    TIGR_CK(cudaMemcpyAsync(peers_buf.p, &h, sizeof(FusedPeers), cudaMemcpyHostToDevice, s));
+    TIGR_CK(cudaStreamSynchronize(s));  // h is a stack copy
+    *out = peers_buf.as<FusedPeers>();
+    return TIGR_OK;
+}
+
+tigr_status fused_barrier(tigr_comm* c, cudaStream_t s) { return comm_sync_barrier(c, s); }
+
+tigr_status fused_end_iteration(tigr_comm* c, Ctl* ctl, cudaStream_t s) {
+    TIGR_TRY(comm_sync_barrier(c, s));
+    k_fused_settle<<<1, 1, 0, s>>>(ctl);
+    TIGR_CKL("fused settle");
+    return TIGR_OK;
+}
 
 tigr_status exchange_frontier(const ExchangeArgs& x, cudaStream_t s, bool* sparse_used) {
     *sparse_used = false;

@@ -104,6 +104,22 @@ __device__ __forceinline__ void map_round(const uint32_t* __restrict__ qv, const
     k += (uint32_t)__shfl_sync(kFull, e, 31);
 }
 
+// Fused exchange (TIGR_EXCHANGE_FUSED, exchange.cu): an improvement found by this rank is
+// applied, in the same branch, to every peer's replica with the relax's own atomic (over
+// NVLink when the peer is another GPU) and activates the node there too -- the peers see it
+// like an update from one more SM.  Only improvements travel: bytes ~ updates x (P-1) x 8.
+template <int A>
+__device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, uint32_t n, uint32_t it, uint32_t v,
+                                           uint32_t alt) {
+    const uint64_t slot = (uint64_t)((it + 1) & 1u) * n;
+    for (int r = 0; r < pp->P; ++r) {
+        if (r == pp->me) continue;
+        if (A == TIGR_SSWP) atomicMax(pp->val[r] + v, alt);
+        else atomicMin(pp->val[r] + v, alt);
+        pp->stamp[r][slot + v] = it + 1;
+    }
+}
+
 }  // namespace
 
 // ------------------------------------------------------------------------------------------
@@ -223,6 +239,7 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                 if (better<A>(alt, cur[q])) {
                     if (A == TIGR_SSWP) atomicMax(a.val + nb[q], alt);
                     else atomicMin(a.val + nb[q], alt);
+                    if (f.peers) push_peers<A>(f.peers, a.n, it, nb[q], alt);
                     // the level becomes alt = it, final (see the header): mark it settled
                     if (BITS) atomicOr(f.settled + (nb[q] >> 5), 1u << (nb[q] & 31u));
                     stamp_next[nb[q]] = it + 1;
@@ -275,7 +292,14 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             }
         }
     }
-    if (__any_sync(kFull, touched) && lane == 0) a.ctl->changed = 1;
+    if (__any_sync(kFull, touched) && lane == 0) {
+        if (f.peers) {  // every rank's verdict for this iteration, read after the group barrier
+            for (int r = 0; r < f.peers->P; ++r)
+                *reinterpret_cast<volatile uint32_t*>(&f.peers->ctl[r]->xchanged[it & 1u]) = 1u;
+        } else {
+            a.ctl->changed = 1;
+        }
+    }
     if (STATS) {
         unsigned long long e = n_edges, u = n_upd, q = n_vn;
 #pragma unroll

@@ -687,6 +687,7 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
     }
     if (v == 0) {
         ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
+        ctl->xchanged[0] = 0; ctl->xchanged[1] = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
         ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0; ctl->nodes = 0;
     }

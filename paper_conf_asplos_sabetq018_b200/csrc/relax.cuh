@@ -24,6 +24,16 @@ struct RelaxArgs {
 
 typedef void (*RelaxFn)(RelaxArgs);
 
+struct Ctl;
+// fused multi-GPU exchange (exchange.cu): the replicas of every rank of a thread group
+constexpr int kMaxPeers = 16;
+struct FusedPeers {
+    int P, me;
+    uint32_t* val[kMaxPeers];
+    uint32_t* stamp[kMaxPeers];
+    Ctl* ctl[kMaxPeers];
+};
+
 // queue-driven frontier relax with dynamic virtual-node mapping (frontier.cu)
 struct FqArgs {
     const uint32_t* qv;   // uint32[2][n] queue node ids (slot = iteration parity)
@@ -31,6 +41,7 @@ struct FqArgs {
     int mode;             // 0 = per iteration (queue if vnodes * dense_div < span), 1 = queue, 2 = dense
     uint32_t dense_div;
     uint32_t* settled;    // BFS only: bit v set once v's level is final (nullptr: test the value)
+    const FusedPeers* peers;  // fused exchange: every improvement is also applied to the peers' replicas
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
 FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);
@@ -94,6 +105,10 @@ struct ExchangeArgs {
     Ctl* ctl;
 };
 tigr_status exchange_frontier(const ExchangeArgs& x, cudaStream_t s, bool* sparse_used);
+tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, DevBuf& peers_buf,
+                        cudaStream_t s, const FusedPeers** out);
+tigr_status fused_barrier(tigr_comm* c, cudaStream_t s);
+tigr_status fused_end_iteration(tigr_comm* c, Ctl* ctl, cudaStream_t s);
 __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
                           double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl);
 __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double base, double damping,

@@ -89,6 +89,7 @@ struct FrontierPlan {
     RelaxArgs args;
     unsigned grid;
     bool bsp, comm;
+    bool fused = false;    // TIGR_EXCHANGE_FUSED: the relax updates the peers' replicas itself
     int algo;
     tigr_comm* c;
     uint32_t n;
@@ -99,8 +100,9 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
                          int* kernels, cudaEvent_t ev_a = nullptr, cudaEvent_t ev_b = nullptr,
                          uint32_t* sparse_count = nullptr) {
     int k = 0;
-    if (p.bsp && !p.comm)
+    if (p.bsp && (!p.comm || p.fused))
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * p.n, cudaMemcpyDeviceToDevice, s));
+    if (p.bsp && p.fused) TIGR_TRY(fused_barrier(p.c, s));  // every snapshot taken before any remote update
     if (ev_a) TIGR_CK(cudaEventRecord(ev_a, s));
     if (p.grid && p.fq) {
         p.fq<<<p.grid, relax_fq_threads(), 0, s>>>(p.args, p.fa);
@@ -112,7 +114,9 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
         ++k;
     }
     if (ev_b) TIGR_CK(cudaEventRecord(ev_b, s));
-    if (p.comm) {  // host loop only (never captured): the exchange decides on the host
+    if (p.fused) {  // host loop only: wait for every rank's relax (and its remote updates)
+        TIGR_TRY(fused_end_iteration(p.c, p.args.ctl, s));
+    } else if (p.comm) {  // host loop only (never captured): the exchange decides on the host
         bool sparse = false;
         TIGR_TRY(exchange_frontier(p.xa, s, &sparse));  // its kernels count their own launches
         if (sparse && sparse_count) ++*sparse_count;
@@ -145,6 +149,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         const char* d = getenv("TIGR_FQ_DIV");
         p.fa.dense_div = d ? (uint32_t)atoi(d) : 2u;
         p.fa.settled = nullptr;
+        p.fa.peers = nullptr;
         const char* bb = getenv("TIGR_BFS_BITS");  // development knob: 0 = test the levels instead
         if (algo == TIGR_BFS && !(bb && atoi(bb) == 0)) {
             if (!ws.settled.p) TIGR_TRY(ws.settled.alloc(sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
@@ -163,8 +168,16 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     if (!p.relax) return fail(TIGR_EUNSUPPORTED, "no relax kernel for this option combination");
     p.args = make_args(vg);
     if (p.comm) {
-        if (o.exchange < TIGR_EXCHANGE_AUTO || o.exchange > TIGR_EXCHANGE_SPARSE)
+        if (o.exchange < TIGR_EXCHANGE_AUTO || o.exchange > TIGR_EXCHANGE_FUSED)
             return fail(TIGR_EINVAL, "run: unknown exchange mode");
+        if (o.exchange == TIGR_EXCHANGE_FUSED) {
+            if (!p.fq)
+                return fail(TIGR_EUNSUPPORTED, "fused exchange needs the queue/dense frontier relax (4 | K, FRONTIER_AUTO/QUEUE)");
+            const FusedPeers* fp = nullptr;
+            TIGR_TRY(fused_setup(o.comm, p.args.val, p.args.stamp, p.args.ctl, ws.peers, s, &fp));
+            p.fa.peers = fp;
+            p.fused = true;
+        }
         if (o.exchange != TIGR_EXCHANGE_DENSE && !ws.xlist.p)
             TIGR_TRY(ws.xlist.alloc(sizeof(uint2) * (n ? n : 1), s));
         p.xa = ExchangeArgs{o.comm, o.exchange, algo, n, p.args.val, (uint32_t*)p.args.prev, p.args.stamp,
@@ -191,6 +204,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     if (p.bsp || p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
     if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s));  // iteration 1's queue
+    if (p.fused) TIGR_TRY(fused_barrier(p.c, s));  // every replica initialised before any remote update
 
     int kpi = 0;
     uint32_t launches = 0, sparse_exchanges = 0;

@@ -16,7 +16,8 @@ struct Ctl {
     uint32_t max_iters;
     uint32_t cont;         // 1 while the loop should continue (host-loop mode reads it)
     uint32_t notconv;      // 1 if the cap was hit while values still changed
-    uint32_t pad[3];
+    uint32_t xchanged[2];  // fused multi-GPU exchange: set by any rank's relax in iteration it (slot it&1)
+    uint32_t pad;
     unsigned long long edges, updates, vnodes;
     double dsum[2];        // PR: dangling mass of the iterate (parity of the iteration)
     // active-node queue of iteration it (frontier.cu): slot it&1 packs (entries << 32) | vnodes
@@ -57,7 +58,8 @@ struct Workspace {
     DevBuf qv;       // uint32[2][n]: active-node queue (node ids), one slot per iteration parity
     DevBuf qo;       // uint32[2][n]: first queue-space virtual node of each entry (exclusive prefix)
     DevBuf settled;  // uint32[n/32+1]: BFS settled bitmap (frontier.cu)
-    DevBuf xlist;    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
+    DevBuf xlist;
+    DevBuf peers;    // FusedPeers (fused multi-GPU exchange, exchange.cu)    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
     DevBuf ctl;      // Ctl
     Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (thread-local, not owned)
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};

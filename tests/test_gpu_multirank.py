@@ -90,7 +90,7 @@ def _check(want, res, algos=("bfs", "sssp", "sswp", "cc", "pr")):
 
 @pytest.mark.parametrize("graph", ["cfg1", "s16"])
 @pytest.mark.parametrize("P", [2, 3])
-@pytest.mark.parametrize("exchange", ["dense", "sparse", "auto"])
+@pytest.mark.parametrize("exchange", ["dense", "sparse", "auto", "fused"])
 def test_group_vnode_partition(tigr, graph, P, exchange):
     """Full graph on every rank, virtual node range per rank (tigr_vgraph_partition)."""
     n, src, dst, w = _graph(graph)
@@ -116,7 +116,7 @@ def test_group_vnode_partition(tigr, graph, P, exchange):
     for r in res:
         for a, st in r["stats"].items():
             assert st["iterations"] == res[0]["stats"][a]["iterations"]  # same termination on every rank
-            if exchange == "dense":
+            if exchange in ("dense", "fused"):
                 assert st["sparse_exchanges"] == 0
             elif exchange == "sparse":
                 assert st["sparse_exchanges"] == st["iterations"], (a, st)
@@ -142,7 +142,11 @@ def test_group_source_partition_bsp_and_queue(tigr, P):
             res[a] = tigr.tigr_run(vg, a, 0, comm=comm, exchange="sparse", schedule=1, stream=s)
             q = tigr.tigr_run(vg, a, 0, comm=comm, exchange="auto", frontier=tigr.TIGR_FRONTIER_QUEUE, stream=s)
             assert np.array_equal(q, res[a]), a
+            for sched in (0, 1):  # fused exchange, asynchronous and BSP
+                fz = tigr.tigr_run(vg, a, 0, comm=comm, exchange="fused", schedule=sched, stream=s)
+                assert np.array_equal(fz, res[a]), (a, sched)
         res["cc"] = tigr.tigr_run(vgs, "cc", comm=comm, exchange="sparse", stream=s)
+        assert np.array_equal(tigr.tigr_run(vgs, "cc", comm=comm, exchange="fused", stream=s), res["cc"])
         res["pr"] = tigr.tigr_run(vg, "pr", comm=comm, stream=s)
         return res
 
@@ -163,6 +167,9 @@ def test_group_consecutive_layout_and_odd_K(tigr):
             for a in ("bfs", "sssp", "sswp"):
                 got = tigr.tigr_run(vg, a, 0, comm=comm, exchange="sparse", stream=s)
                 assert np.array_equal(got, want[a]), (K, layout, a)
+            with pytest.raises(tigr.TigrError) as e:  # fused needs the 16-byte-chunk relax (4 | K)
+                tigr.tigr_run(vg, "bfs", 0, comm=comm, exchange="fused", stream=s)
+            assert e.value.status == tigr.TIGR_EUNSUPPORTED
             out[K] = True
         return out
 
@@ -207,11 +214,14 @@ def test_exchange_modes_single_rank_nccl(tigr, exchange):
         if exchange == "sparse":
             assert st["sparse_exchanges"] == st["iterations"]
     assert np.array_equal(tigr.tigr_run(vgs, "cc", comm=comm, exchange=exchange), want["cc"])
+    with pytest.raises(tigr.TigrError) as e:  # fused needs peer pointers: thread group only
+        tigr.tigr_run(vg, "bfs", 0, comm=comm, exchange="fused")
+    assert e.value.status == tigr.TIGR_EUNSUPPORTED
     comm.free()
 
 
 @pytest.mark.slow
-@pytest.mark.parametrize("exchange", ["sparse", "auto"])
+@pytest.mark.parametrize("exchange", ["sparse", "auto", "fused"])
 def test_group_cfg2_full(tigr, exchange):
     """Config 2 at full size (R-MAT scale 20: 16.8 M arcs, 33.6 M symmetrised) on 4 ranks:
     BFS and CC bit-exact on every rank, plus SSSP through the source-range build."""
