@@ -296,6 +296,18 @@ tigr_status tigr_comm_group_create(int nranks, tigr_comm_group** out);
 tigr_status tigr_comm_init_group(tigr_comm_group* group, int rank, tigr_comm** out);
 void tigr_comm_group_free(tigr_comm_group* group);
 
+/* Node communicator: nranks PROCESSES of one node (normally one per GPU, e.g. under torchrun),
+ * without NCCL.  Rank 0 creates the POSIX shared-memory segment "/tigr_<name>" (name: unique per
+ * job, <= 200 chars), the other ranks attach to it; it holds a barrier and one slot per rank.
+ * Device buffers are shared as CUDA IPC handles (mapped once per peer allocation, NVLink peer
+ * access between distinct GPUs), so every exchange mode -- dense, sparse and fused -- reads or
+ * updates the peers' replicas directly, exactly as the thread-group communicator does.  Each
+ * rank calls it on its own current device; it returns once all ranks have joined.
+ * Errors: EINVAL (name, nranks outside [1, 16], rank outside [0, nranks), nranks differs from
+ * rank 0's), ENCCL (segment not created / barrier timeout, TIGR_GROUP_TIMEOUT seconds),
+ * EUNSUPPORTED (GPUs without peer access).  tigr_comm_free detaches (rank 0 unlinks). */
+tigr_status tigr_comm_init_node(const char* name, int nranks, int rank, tigr_comm** out);
+
 /* ----------------------------------------------------------------- misc ---- */
 
 const char* tigr_last_error(void);

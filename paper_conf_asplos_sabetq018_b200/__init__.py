@@ -95,6 +95,7 @@ _SIGS = {
     "tigr_comm_group_create": (_I, [_I, ctypes.POINTER(_P)]),
     "tigr_comm_init_group": (_I, [_P, _I, ctypes.POINTER(_P)]),
     "tigr_comm_group_free": (None, [_P]),
+    "tigr_comm_init_node": (_I, [ctypes.c_char_p, _I, _I, ctypes.POINTER(_P)]),
     "tigr_last_error": (ctypes.c_char_p, []),
     "tigr_launch_count": (_U64, []),
     "tigr_release_cached_memory": (None, []),
@@ -448,6 +449,14 @@ def tigr_comm_init_group(group: CommGroup, rank: int) -> Comm:
     out = _P()
     _check(_lib.tigr_comm_init_group(group.ptr, rank, ctypes.byref(out)))
     return Comm(out.value, group.nranks, rank)
+
+
+def tigr_comm_init_node(name: str, nranks: int, rank: int) -> Comm:
+    """Join the node communicator `name` (ranks = processes of this node, CUDA IPC + shared
+    memory, no NCCL) as `rank` on the current CUDA device; returns once all ranks joined."""
+    out = _P()
+    _check(_lib.tigr_comm_init_node(name.encode(), nranks, rank, ctypes.byref(out)))
+    return Comm(out.value, nranks, rank)
 
 
 def tigr_last_error() -> str:

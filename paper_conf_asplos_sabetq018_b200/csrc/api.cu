@@ -126,6 +126,21 @@ void cache_free(void* p, cudaStream_t s) {
     g_free.emplace(std::make_pair(b.dev, b.size), b);
 }
 
+// the live libtigr allocation containing p: its base and p's offset in it (CUDA IPC exports
+// whole allocations)
+bool cache_base(const void* p, void** base, size_t* off) {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    auto it = g_live.upper_bound(const_cast<void*>(p));
+    if (it == g_live.begin()) return false;
+    --it;
+    const char* b = static_cast<const char*>(it->first);
+    const char* q = static_cast<const char*>(p);
+    if (q < b || q >= b + it->second.second) return false;
+    *base = it->first;
+    *off = (size_t)(q - b);
+    return true;
+}
+
 void cache_release_all() {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     cudaDeviceSynchronize();
@@ -191,6 +206,7 @@ tigr_status comm_unique_id(uint8_t id[128]);
 tigr_status comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
 void comm_free(tigr_comm* c);
 tigr_status comm_group_create(int nranks, tigr_comm_group** out);
+tigr_status comm_init_node(const char* name, int nranks, int rank, tigr_comm** out);
 tigr_status comm_init_group(tigr_comm_group* g, int rank, tigr_comm** out);
 void comm_group_free(tigr_comm_group* g);
 
@@ -503,6 +519,12 @@ tigr_status tigr_comm_init_group(tigr_comm_group* group, int rank, tigr_comm** o
 }
 
 void tigr_comm_group_free(tigr_comm_group* g) { comm_group_free(g); }
+
+tigr_status tigr_comm_init_node(const char* name, int nranks, int rank, tigr_comm** out) {
+    if (!out) return fail(TIGR_EINVAL, "comm_init_node: NULL");
+    *out = nullptr;
+    return comm_init_node(name, nranks, rank, out);
+}
 
 const char* tigr_last_error(void) { return t_err.c_str(); }
 

@@ -16,11 +16,16 @@
 //     kernels read the peers' buffers directly (same device, or NVLink peer access enabled at
 //     init).  This is also what lets the multi-rank protocol run on a single GPU.
 #include <dlfcn.h>
+#include <fcntl.h>
 #include <nccl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <chrono>
 #include <condition_variable>
+#include <map>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -29,23 +34,42 @@
 
 namespace tigr {
 
-// ------------------------------------------------------------------------------ thread group
-struct LocalGroup {
+constexpr int kMaxGroupRanks = 16;
+
+// ------------------------------------------------------------------------------ peer groups
+// Ranks that can read each other's device memory: a published pointer of rank r becomes usable
+// on every rank after the next barrier.  Two implementations: ranks as threads of one process
+// (LocalGroup) and ranks as processes of one node (NodeGroup: POSIX shared memory for slots and
+// barrier, CUDA IPC for the device pointers).
+struct PeerGroup {
     int P = 1;
+    virtual ~PeerGroup() {}
+    virtual tigr_status barrier() = 0;
+    virtual tigr_status publish(int me, const void* const* ptrs, int k) = 0;
+    virtual tigr_status peer(int me, int r, int k, const void** out) = 0;
+    virtual void publish_count(int me, uint32_t c) = 0;
+    virtual uint32_t count(int r) = 0;
+};
+
+static int group_timeout_s() {
+    const char* e = getenv("TIGR_GROUP_TIMEOUT");
+    return e ? atoi(e) : 300;
+}
+
+struct LocalGroup : PeerGroup {
     std::mutex mu;
     std::condition_variable cv;
     int arrived = 0;
     uint64_t gen = 0;
     bool broken = false;
-    std::vector<const void*> ptr;  // published device pointers (one per rank)
-    std::vector<const void*> ptrk; // published pointer sets (kMaxSet per rank)
+    std::vector<const void*> ptrk; // published pointer sets (8 per rank)
     std::vector<uint32_t> cnt;     // published counts
     std::vector<int> dev;          // device of each rank
     std::vector<char> joined;
 
     // all P ranks arrive before any leaves; a rank that waits longer than the timeout marks
     // the group broken (a peer failed or never called), and every later barrier fails at once
-    tigr_status barrier() {
+    tigr_status barrier() override {
         std::unique_lock<std::mutex> lk(mu);
         if (broken) return fail(TIGR_ENCCL, "thread-group communicator: a rank failed earlier");
         const uint64_t g = gen;
@@ -55,14 +79,107 @@ struct LocalGroup {
             cv.notify_all();
             return TIGR_OK;
         }
-        const int secs = getenv("TIGR_GROUP_TIMEOUT") ? atoi(getenv("TIGR_GROUP_TIMEOUT")) : 300;
-        if (!cv.wait_for(lk, std::chrono::seconds(secs), [&] { return gen != g || broken; }) || broken) {
+        if (!cv.wait_for(lk, std::chrono::seconds(group_timeout_s()), [&] { return gen != g || broken; }) ||
+            broken) {
             broken = true;
             cv.notify_all();
             return fail(TIGR_ENCCL, "thread-group communicator: barrier timed out (a rank did not arrive)");
         }
         return TIGR_OK;
     }
+    tigr_status publish(int me, const void* const* ptrs, int k) override {
+        for (int i = 0; i < k; ++i) ptrk[(size_t)me * 8 + i] = ptrs[i];
+        return TIGR_OK;
+    }
+    tigr_status peer(int, int r, int k, const void** out) override {
+        for (int i = 0; i < k; ++i) out[i] = ptrk[(size_t)r * 8 + i];
+        return TIGR_OK;
+    }
+    void publish_count(int me, uint32_t c) override { cnt[me] = c; }
+    uint32_t count(int r) override { return cnt[r]; }
+};
+
+bool cache_base(const void* p, void** base, size_t* off);  // api.cu: allocation containing p
+
+// Ranks as processes of one node.  The shared segment holds a sense-counting barrier and one
+// slot per rank; device pointers travel as CUDA IPC handles of their allocation plus an offset
+// and are mapped once per (rank, allocation) with cudaIpcOpenMemHandle.
+struct NodeShm {
+    static constexpr uint32_t kMagic = 0x54494752u;  // "TIGR"
+    std::atomic<uint32_t> magic;
+    uint32_t P;
+    std::atomic<uint32_t> arrived, gen, broken, joined;
+    struct Slot {
+        int dev;
+        uint32_t count;
+        cudaIpcMemHandle_t h[8];
+        uint64_t off[8];
+    } slot[kMaxGroupRanks];
+};
+
+struct NodeGroup : PeerGroup {
+    std::string name;
+    NodeShm* shm = nullptr;
+    int me = 0;
+    bool owner = false;
+    std::vector<const void*> mine = std::vector<const void*>(8, nullptr);
+    std::map<std::string, void*> opened;  // IPC handle bytes -> mapped base
+
+    ~NodeGroup() override {
+        for (auto& kv : opened) cudaIpcCloseMemHandle(kv.second);
+        if (shm) munmap(shm, sizeof(NodeShm));
+        if (owner) shm_unlink(name.c_str());
+    }
+    tigr_status barrier() override {
+        if (shm->broken.load()) return fail(TIGR_ENCCL, "node communicator: a rank failed earlier");
+        const uint32_t g = shm->gen.load(std::memory_order_acquire);
+        if (shm->arrived.fetch_add(1, std::memory_order_acq_rel) + 1 == (uint32_t)P) {
+            shm->arrived.store(0, std::memory_order_relaxed);
+            shm->gen.fetch_add(1, std::memory_order_acq_rel);
+            return TIGR_OK;
+        }
+        const auto t0 = std::chrono::steady_clock::now();
+        int spins = 0;
+        while (shm->gen.load(std::memory_order_acquire) == g) {
+            if (shm->broken.load()) return fail(TIGR_ENCCL, "node communicator: a rank failed earlier");
+            if (++spins > 1000) {
+                usleep(20);
+                if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(group_timeout_s())) {
+                    shm->broken.store(1);
+                    return fail(TIGR_ENCCL, "node communicator: barrier timed out (a rank did not arrive)");
+                }
+            }
+        }
+        return TIGR_OK;
+    }
+    tigr_status publish(int r, const void* const* ptrs, int k) override {
+        for (int i = 0; i < k; ++i) {
+            mine[i] = ptrs[i];
+            void* base = nullptr;
+            size_t off = 0;
+            if (!cache_base(ptrs[i], &base, &off))
+                return fail(TIGR_EINVAL, "node communicator: buffer not allocated by libtigr");
+            TIGR_CK(cudaIpcGetMemHandle(&shm->slot[r].h[i], base));
+            shm->slot[r].off[i] = off;
+        }
+        return TIGR_OK;
+    }
+    tigr_status peer(int self, int r, int k, const void** out) override {
+        for (int i = 0; i < k; ++i) {
+            if (r == self) { out[i] = mine[i]; continue; }
+            const std::string key(reinterpret_cast<const char*>(&shm->slot[r].h[i]), sizeof(cudaIpcMemHandle_t));
+            auto it = opened.find(key);
+            if (it == opened.end()) {
+                void* p = nullptr;
+                TIGR_CK(cudaIpcOpenMemHandle(&p, shm->slot[r].h[i], cudaIpcMemLazyEnablePeerAccess));
+                it = opened.emplace(key, p).first;
+            }
+            out[i] = static_cast<const char*>(it->second) + shm->slot[r].off[i];
+        }
+        return TIGR_OK;
+    }
+    void publish_count(int r, uint32_t c) override { shm->slot[r].count = c; }
+    uint32_t count(int r) override { return shm->slot[r].count; }
 };
 
 namespace {
@@ -127,15 +244,16 @@ tigr_status nccl_check(ncclResult_t r, const char* what) {
 }
 
 // ------------------------------------------------------------------------------ group kernels
-constexpr int kMaxGroup = 16;
+constexpr int kMaxGroup = kMaxGroupRanks;
 struct PeerPtrs {
     const void* p[kMaxGroup];
 };
 
-// out[i] = op over ranks 0..P-1 (in rank order, so every rank computes the same bits) of in_r[i]
+// out[i] = op over ranks 0..P-1 (in rank order, so every rank computes the same bits) of in_r[i],
+// for i in [lo, hi)
 template <class T, int OP>  // OP: 0 min, 1 max, 2 sum
-__global__ void k_group_reduce(PeerPtrs in, int P, size_t count, T* __restrict__ out) {
-    for (size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (size_t)gridDim.x * blockDim.x) {
+__global__ void k_group_reduce(PeerPtrs in, int P, size_t lo, size_t hi, T* __restrict__ out) {
+    for (size_t i = lo + (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < hi; i += (size_t)gridDim.x * blockDim.x) {
         T v = static_cast<const T*>(in.p[0])[i];
         for (int r = 1; r < P; ++r) {
             const T x = static_cast<const T*>(in.p[r])[i];
@@ -145,6 +263,17 @@ __global__ void k_group_reduce(PeerPtrs in, int P, size_t count, T* __restrict__
         }
         out[i] = v;
     }
+}
+
+// buf[i] = src_r[i] for i in rank r's slice, every r != me (16-byte copies where aligned)
+template <class T>
+__global__ void k_group_gather(PeerPtrs src, int P, int me, size_t count, T* __restrict__ buf) {
+    const int r = blockIdx.y;
+    if (r == me) return;
+    const size_t lo = count * (size_t)r / (size_t)P, hi = count * (size_t)(r + 1) / (size_t)P;
+    const T* __restrict__ s = static_cast<const T*>(src.p[r]);
+    for (size_t i = lo + (size_t)blockIdx.x * blockDim.x + threadIdx.x; i < hi; i += (size_t)gridDim.x * blockDim.x)
+        buf[i] = s[i];
 }
 
 tigr_status scratch_bytes(tigr_comm* c, size_t bytes, cudaStream_t s) {
@@ -184,12 +313,24 @@ tigr_status comm_group_create(int nranks, tigr_comm_group** out) {
     if (nranks < 1 || nranks > kMaxGroup) return fail(TIGR_EINVAL, "comm_group_create: nranks outside [1, 16]");
     auto g = std::make_shared<LocalGroup>();
     g->P = nranks;
-    g->ptr.assign(nranks, nullptr);
     g->ptrk.assign((size_t)nranks * 8, nullptr);
     g->cnt.assign(nranks, 0);
     g->dev.assign(nranks, -1);
     g->joined.assign(nranks, 0);
     *out = new tigr_comm_group{g};
+    return TIGR_OK;
+}
+
+static tigr_status enable_peers(int dev, const std::vector<int>& devs) {
+    for (int d : devs) {
+        if (d == dev || d < 0) continue;
+        int can = 0;
+        TIGR_CK(cudaDeviceCanAccessPeer(&can, dev, d));
+        if (!can) return fail(TIGR_EUNSUPPORTED, "communicator: no peer access between the ranks' GPUs");
+        cudaError_t e = cudaDeviceEnablePeerAccess(d, 0);
+        if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+        else TIGR_CK(e);
+    }
     return TIGR_OK;
 }
 
@@ -205,15 +346,7 @@ tigr_status comm_init_group(tigr_comm_group* grp, int rank, tigr_comm** out) {
         g.dev[rank] = dev;
     }
     TIGR_TRY(g.barrier());  // every rank's device is known after this
-    for (int r = 0; r < g.P; ++r) {
-        if (g.dev[r] == dev) continue;
-        int can = 0;
-        TIGR_CK(cudaDeviceCanAccessPeer(&can, dev, g.dev[r]));
-        if (!can) return fail(TIGR_EUNSUPPORTED, "comm_init_group: no peer access between the ranks' GPUs");
-        cudaError_t e = cudaDeviceEnablePeerAccess(g.dev[r], 0);
-        if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
-        else TIGR_CK(e);
-    }
+    TIGR_TRY(enable_peers(dev, g.dev));
     tigr_comm* tc = new tigr_comm();
     tc->local = grp->g;
     tc->nranks = g.P;
@@ -225,6 +358,71 @@ tigr_status comm_init_group(tigr_comm_group* grp, int rank, tigr_comm** out) {
 
 void comm_group_free(tigr_comm_group* g) { delete g; }
 
+// Node communicator: rank 0 creates the shared segment "/tigr_<name>", the others attach to it
+// (waiting up to TIGR_GROUP_TIMEOUT seconds for it to appear), every rank records its device,
+// and the call returns once all nranks have joined.
+tigr_status comm_init_node(const char* name, int nranks, int rank, tigr_comm** out) {
+    if (!name || !*name || strlen(name) > 200) return fail(TIGR_EINVAL, "comm_init_node: bad name");
+    if (nranks < 1 || nranks > kMaxGroupRanks || rank < 0 || rank >= nranks)
+        return fail(TIGR_EINVAL, "comm_init_node: nranks outside [1, 16] or rank outside [0, nranks)");
+    int dev = 0;
+    TIGR_CK(cudaGetDevice(&dev));
+    auto g = std::make_shared<NodeGroup>();
+    g->name = std::string("/tigr_") + name;
+    g->P = nranks;
+    g->me = rank;
+    int fd = -1;
+    if (rank == 0) {
+        shm_unlink(g->name.c_str());  // a stale segment of an earlier job with this name
+        fd = shm_open(g->name.c_str(), O_CREAT | O_EXCL | O_RDWR, 0600);
+        if (fd < 0 || ftruncate(fd, sizeof(NodeShm)) != 0) {
+            if (fd >= 0) close(fd);
+            return fail(TIGR_ENCCL, "comm_init_node: cannot create the shared segment");
+        }
+        g->owner = true;
+    } else {
+        const auto t0 = std::chrono::steady_clock::now();
+        while ((fd = shm_open(g->name.c_str(), O_RDWR, 0600)) < 0) {
+            if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(group_timeout_s()))
+                return fail(TIGR_ENCCL, "comm_init_node: rank 0 never created the shared segment");
+            usleep(1000);
+        }
+    }
+    void* m = mmap(nullptr, sizeof(NodeShm), PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+    close(fd);
+    if (m == MAP_FAILED) return fail(TIGR_ENCCL, "comm_init_node: mmap failed");
+    g->shm = static_cast<NodeShm*>(m);
+    if (rank == 0) {
+        g->shm->P = (uint32_t)nranks;
+        g->shm->arrived.store(0);
+        g->shm->gen.store(0);
+        g->shm->broken.store(0);
+        g->shm->joined.store(0);
+        g->shm->magic.store(NodeShm::kMagic, std::memory_order_release);
+    } else {
+        const auto t0 = std::chrono::steady_clock::now();
+        while (g->shm->magic.load(std::memory_order_acquire) != NodeShm::kMagic) {
+            if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(group_timeout_s()))
+                return fail(TIGR_ENCCL, "comm_init_node: the shared segment was never initialised");
+            usleep(1000);
+        }
+        if (g->shm->P != (uint32_t)nranks) return fail(TIGR_EINVAL, "comm_init_node: nranks differs from rank 0's");
+    }
+    g->shm->slot[rank].dev = dev;
+    g->shm->joined.fetch_add(1);
+    TIGR_TRY(g->barrier());  // every rank's device is known after this
+    std::vector<int> devs(nranks);
+    for (int r = 0; r < nranks; ++r) devs[r] = g->shm->slot[r].dev;
+    TIGR_TRY(enable_peers(dev, devs));
+    tigr_comm* tc = new tigr_comm();
+    tc->local = g;
+    tc->nranks = nranks;
+    tc->rank = rank;
+    tc->device = dev;
+    *out = tc;
+    return TIGR_OK;
+}
+
 void comm_free(tigr_comm* c) {
     if (!c) return;
     if (c->nccl && g_nccl.commDestroy) g_nccl.commDestroy((ncclComm_t)c->nccl);
@@ -233,32 +431,50 @@ void comm_free(tigr_comm* c) {
 
 // ------------------------------------------------------------------------------ operations
 // in-place all-reduce of a replicated array: MIN (BFS/SSSP/CC), MAX (SSWP) of uint32, SUM of
-// float64 (PR).  Thread group: every rank reduces all replicas in rank order into scratch (so
-// the float64 sums are bit-identical on every rank), then, once no peer still reads, copies back.
+// float64 (PR).  Peer groups run it as a reduce-scatter + all-gather over peer memory (each
+// rank moves ~2x its array, as a ring would): rank r reduces slice r of all replicas, in rank
+// order, into its scratch (so the float64 sums are bit-identical on every rank); once every
+// slice is reduced, every rank copies the other slices from their owners' scratch.
 tigr_status comm_allreduce(tigr_comm* c, void* buf, size_t count, int algo, cudaStream_t s) {
     if (c->local) {
-        LocalGroup& g = *c->local;
+        PeerGroup& g = *c->local;
+        const int P = g.P, me = c->rank;
         const size_t esz = algo == TIGR_PR ? sizeof(double) : sizeof(uint32_t);
         TIGR_TRY(scratch_bytes(c, count * esz, s));
-        g.ptr[c->rank] = buf;
+        const void* mine[2] = {buf, c->scratch.p};
+        TIGR_TRY(g.publish(me, mine, 2));
         TIGR_CK(cudaStreamSynchronize(s));
         TIGR_TRY(g.barrier());
-        PeerPtrs pp{};
-        for (int r = 0; r < g.P; ++r) pp.p[r] = g.ptr[r];
-        if (count) {
-            const unsigned grid = (unsigned)std::min<size_t>((count + kBlock - 1) / kBlock, 148 * 8);
+        PeerPtrs rep{}, scr{};
+        for (int r = 0; r < P; ++r) {
+            const void* two[2];
+            TIGR_TRY(g.peer(me, r, 2, two));
+            rep.p[r] = two[0];
+            scr.p[r] = two[1];
+        }
+        const size_t lo = count * (size_t)me / (size_t)P, hi = count * (size_t)(me + 1) / (size_t)P;
+        if (hi > lo) {
+            const unsigned grid = (unsigned)std::min<size_t>((hi - lo + kBlock - 1) / kBlock, 148 * 8);
             if (algo == TIGR_PR)
-                k_group_reduce<double, 2><<<grid, kBlock, 0, s>>>(pp, g.P, count, c->scratch.as<double>());
+                k_group_reduce<double, 2><<<grid, kBlock, 0, s>>>(rep, P, lo, hi, c->scratch.as<double>());
             else if (algo == TIGR_SSWP)
-                k_group_reduce<uint32_t, 1><<<grid, kBlock, 0, s>>>(pp, g.P, count, c->scratch.as<uint32_t>());
+                k_group_reduce<uint32_t, 1><<<grid, kBlock, 0, s>>>(rep, P, lo, hi, c->scratch.as<uint32_t>());
             else
-                k_group_reduce<uint32_t, 0><<<grid, kBlock, 0, s>>>(pp, g.P, count, c->scratch.as<uint32_t>());
-            TIGR_CKL("group all-reduce");
+                k_group_reduce<uint32_t, 0><<<grid, kBlock, 0, s>>>(rep, P, lo, hi, c->scratch.as<uint32_t>());
+            TIGR_CKL("group reduce-scatter");
+            TIGR_CK(cudaMemcpyAsync(static_cast<char*>(buf) + lo * esz, c->scratch.as<char>() + lo * esz,
+                                    (hi - lo) * esz, cudaMemcpyDeviceToDevice, s));
         }
         TIGR_CK(cudaStreamSynchronize(s));
-        TIGR_TRY(g.barrier());  // every peer has finished reading this rank's buffer
-        if (count) TIGR_CK(cudaMemcpyAsync(buf, c->scratch.p, count * esz, cudaMemcpyDeviceToDevice, s));
-        return TIGR_OK;
+        TIGR_TRY(g.barrier());  // every slice reduced; no peer reads the replicas any more
+        if (count && P > 1) {
+            const dim3 grid((unsigned)std::min<size_t>((count / P + kBlock) / kBlock, 148 * 4), (unsigned)P);
+            if (algo == TIGR_PR) k_group_gather<double><<<grid, kBlock, 0, s>>>(scr, P, me, count, static_cast<double*>(buf));
+            else k_group_gather<uint32_t><<<grid, kBlock, 0, s>>>(scr, P, me, count, static_cast<uint32_t*>(buf));
+            TIGR_CKL("group all-gather");
+        }
+        TIGR_CK(cudaStreamSynchronize(s));
+        return g.barrier();  // no peer reads this rank's scratch any more
     }
     TIGR_TRY(nccl_ready());
     ncclDataType_t t = ncclUint32;
@@ -272,12 +488,12 @@ tigr_status comm_allreduce(tigr_comm* c, void* buf, size_t count, int algo, cuda
 tigr_status comm_allgather_count(tigr_comm* c, const uint32_t* dev_count, uint32_t* host_counts, cudaStream_t s) {
     uint32_t mine = 0;
     if (c->local) {
-        LocalGroup& g = *c->local;
+        PeerGroup& g = *c->local;
         TIGR_CK(cudaMemcpyAsync(&mine, dev_count, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
         TIGR_CK(cudaStreamSynchronize(s));
-        g.cnt[c->rank] = mine;
+        g.publish_count(c->rank, mine);
         TIGR_TRY(g.barrier());
-        for (int r = 0; r < g.P; ++r) host_counts[r] = g.cnt[r];
+        for (int r = 0; r < g.P; ++r) host_counts[r] = g.count(r);
         TIGR_TRY(g.barrier());  // slots may be rewritten after this
         return TIGR_OK;
     }
@@ -295,11 +511,11 @@ tigr_status comm_allgather_count(tigr_comm* c, const uint32_t* dev_count, uint32
 tigr_status comm_share_lists(tigr_comm* c, const void* mine, const uint32_t* counts, const void** ptrs,
                              cudaStream_t s) {
     if (c->local) {
-        LocalGroup& g = *c->local;
-        g.ptr[c->rank] = mine;
+        PeerGroup& g = *c->local;
+        TIGR_TRY(g.publish(c->rank, &mine, 1));
         TIGR_CK(cudaStreamSynchronize(s));  // the list is complete before peers read it
         TIGR_TRY(g.barrier());
-        for (int r = 0; r < g.P; ++r) ptrs[r] = g.ptr[r];
+        for (int r = 0; r < g.P; ++r) TIGR_TRY(g.peer(c->rank, r, 1, &ptrs[r]));
         return TIGR_OK;
     }
     TIGR_TRY(nccl_ready());
@@ -321,19 +537,18 @@ tigr_status comm_share_lists(tigr_comm* c, const void* mine, const uint32_t* cou
     return nccl_check(g_nccl.groupEnd(), "ncclGroupEnd");
 }
 
-// every rank's set of k (<= 8) device pointers: all[r * k + i] (thread group only)
+// every rank's set of k (<= 8) device pointers: all[r * k + i] (peer groups only)
 tigr_status comm_share_ptrs(tigr_comm* c, const void* const* mine, int k, const void** all) {
-    if (!c->local) return fail(TIGR_EUNSUPPORTED, "pointer exchange needs the thread-group communicator");
+    if (!c->local) return fail(TIGR_EUNSUPPORTED, "pointer exchange needs a thread-group or node communicator");
     if (k < 1 || k > 8) return fail(TIGR_EINVAL, "comm_share_ptrs: 1..8 pointers");
-    LocalGroup& g = *c->local;
-    for (int i = 0; i < k; ++i) g.ptrk[(size_t)c->rank * 8 + i] = mine[i];
+    PeerGroup& g = *c->local;
+    TIGR_TRY(g.publish(c->rank, mine, k));
     TIGR_TRY(g.barrier());
-    for (int r = 0; r < g.P; ++r)
-        for (int i = 0; i < k; ++i) all[r * k + i] = g.ptrk[(size_t)r * 8 + i];
+    for (int r = 0; r < g.P; ++r) TIGR_TRY(g.peer(c->rank, r, k, all + r * k));
     return g.barrier();  // slots may be rewritten after this
 }
 
-// host barrier of the thread group after this rank's stream has drained (no-op for NCCL)
+// host barrier of a peer group after this rank's stream has drained (no-op for NCCL)
 tigr_status comm_sync_barrier(tigr_comm* c, cudaStream_t s) {
     if (!c->local) return TIGR_OK;
     TIGR_CK(cudaStreamSynchronize(s));

@@ -109,7 +109,7 @@ tigr_status dense(const ExchangeArgs& x, cudaStream_t s) {
 
 }  // namespace
 
-// Fused exchange (TIGR_EXCHANGE_FUSED; thread-group transport).  There is no exchange step:
+// Fused exchange (TIGR_EXCHANGE_FUSED; peer-group transports: thread group or node group).  There is no exchange step:
 // the relax itself applies each improvement to every peer's replica and stamp array
 // (frontier.cu push_peers) and raises every rank's xchanged flag.  What remains per iteration
 // is ordering: a barrier once every rank's relax has drained (all remote updates have landed),
@@ -118,7 +118,7 @@ tigr_status dense(const ExchangeArgs& x, cudaStream_t s) {
 // that no peer's update of the new iteration leaks into it.
 tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, DevBuf& peers_buf,
                         cudaStream_t s, const FusedPeers** out) {
-    if (!c->local) return fail(TIGR_EUNSUPPORTED, "fused exchange needs the thread-group communicator");
+    if (!c->local) return fail(TIGR_EUNSUPPORTED, "fused exchange needs a thread-group or node communicator");
     if (c->nranks > kMaxPeers) return fail(TIGR_EUNSUPPORTED, "fused exchange: more than 16 ranks");
     const void* mine[3] = {val, stamp, ctl};
     const void* all[3 * kMaxPeers] = {};

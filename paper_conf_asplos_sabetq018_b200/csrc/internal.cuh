@@ -120,14 +120,14 @@ struct tigr_graph {
     tigr::DevBuf perm_order; // uint32[n]: id here -> original id
 };
 
-namespace tigr { struct LocalGroup; }
+namespace tigr { struct PeerGroup; struct LocalGroup; }
 
 // A rank's communicator.  Two transports (comm.cu): NCCL (one process per GPU), or a thread
 // group (ranks are threads of one process; exchanges read the peers' buffers directly through
 // unified addressing / NVLink peer access, synchronised by a host barrier).
 struct tigr_comm {
     void* nccl = nullptr;    // ncclComm_t (NCCL transport)
-    std::shared_ptr<tigr::LocalGroup> local;  // thread-group transport
+    std::shared_ptr<tigr::PeerGroup> local;   // peer-group transport (thread group or node group)
     int nranks = 1;
     int rank = 0;
     int device = 0;

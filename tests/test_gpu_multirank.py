@@ -250,3 +250,52 @@ def test_group_cfg2_full(tigr, exchange):
     for rank, got in enumerate(res):
         for a in ("bfs", "sssp", "cc"):
             assert np.array_equal(got[a], want[a]), (rank, a)
+
+
+# ------------------------------------------------------------------------------ node communicator
+def _node_worker(name, P, r, exchange, q):
+    import os
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    try:
+        import torch as t
+        import paper_conf_asplos_sabetq018_b200 as tg
+        t.cuda.set_device(0)
+        n, src, dst, w = _graph("s16")
+        comm = tg.tigr_comm_init_node(name, P, r)
+        g = tg.tigr_graph_from_coo(n, src, dst, w)
+        gs = tg.tigr_graph_from_coo(n, src, dst, None, symmetrize=True)
+        vg = tg.tigr_virtualize(g, 8, "strided")
+        vgs = tg.tigr_virtualize(gs, 8, "strided")
+        tg.tigr_vgraph_partition(vg, P, r)
+        tg.tigr_vgraph_partition(vgs, P, r)
+        out = {a: tg.tigr_run(vg, a, 0, comm=comm, exchange=exchange) for a in ("bfs", "sssp", "sswp")}
+        out["cc"] = tg.tigr_run(vgs, "cc", comm=comm, exchange=exchange)
+        out["pr"] = tg.tigr_run(vg, "pr", comm=comm)
+        t.cuda.synchronize()
+        comm.free()
+        q.put((r, out, None))
+    except Exception as e:  # pragma: no cover - reported by the parent
+        q.put((r, None, repr(e)))
+
+
+@pytest.mark.parametrize("exchange", ["dense", "sparse", "fused"])
+def test_node_communicator_processes(tigr, exchange):
+    """Ranks as separate PROCESSES (both on cuda:0): shared-memory barrier + CUDA IPC buffers,
+    no NCCL -- every exchange mode through real cross-process peer mappings."""
+    import os
+    import torch.multiprocessing as mp
+
+    P = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    name = f"pytest_{os.getpid()}_{exchange}"
+    procs = [ctx.Process(target=_node_worker, args=(name, P, r, exchange, q)) for r in range(P)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=600) for _ in range(P)]
+    for p in procs:
+        p.join(timeout=120)
+    errs = [(r, e) for r, _, e in res if e]
+    assert not errs, errs
+    _check(_want("s16"), [out for _, out, _ in sorted(res, key=lambda x: x[0])])
