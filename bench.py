@@ -56,6 +56,9 @@ def parse():
     ap.add_argument("--no-extra", action="store_true", help="skip the per-algorithm extras")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras, no e2e)")
     ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs (per_config)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "node"],
+                    help="N > 1: PageRank exchange over NCCL (default) or the node communicator (CUDA IPC + "
+                         "shared memory; torch.distributed on gloo; ranks may share a GPU -- for testing)")
     return ap.parse_args()
 
 
@@ -219,8 +222,10 @@ def config_obj(args, rec):
     return {"workload": f"{args.config}: R-MAT n={rec.n:,} m={rec.m:,} (a,b,c)=({rec.a},{rec.b},{rec.c}) "
                         f"PageRank 20 iterations, K={args.K}, {args.layout} layout",
             "algorithm": "pagerank", "K": args.K, "layout": args.layout, "n": rec.n, "m": rec.m,
-            "parallelism": ("source-range partitioned CSR build per rank (arc-balanced cuts) + NCCL all-reduce "
-                            "of the PageRank accumulator each iteration") if args.gpus > 1 else "single GPU",
+            "parallelism": ("source-range partitioned CSR build per rank (arc-balanced cuts) + "
+                            + ("NCCL all-reduce" if args.transport == "nccl" else
+                               "peer-memory reduce-scatter/all-gather (node communicator)")
+                            + " of the PageRank accumulator each iteration") if args.gpus > 1 else "single GPU",
             "l2": "flushed between steps (512 MiB write outside the timed events); arc list 2.1 GB > L2"}
 
 
@@ -240,13 +245,25 @@ def main():
     import graphgen
     import paper_conf_asplos_sabetq018_b200 as tigr
 
+    local = local % max(torch.cuda.device_count(), 1)
     torch.cuda.set_device(local)
     comm = None
-    if world > 1:
+    if world > 1 and args.transport == "nccl":
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         uid = [tigr.tigr_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         comm = tigr.tigr_comm_init(world, rank, uid[0])
+    elif world > 1:
+        dist.init_process_group("gloo")
+        comm = tigr.tigr_comm_init_node(job_name("pr"), world, rank)
+
+    def allmax(x):
+        """max over ranks of a host float (device tensor for NCCL, host tensor for gloo)."""
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda" if args.transport == "nccl" else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
 
     rec = graphgen.recipe(args.config)
     n, m = rec.n, rec.m
@@ -313,11 +330,7 @@ def main():
     launches = tigr.tigr_launch_count() - l0
     clk = clocks.stop()
 
-    t_step = sum(step_ms) / len(step_ms)
-    if world > 1:
-        tt = torch.tensor([t_step], dtype=torch.float64, device="cuda")
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        t_step = float(tt.item())
+    t_step = allmax(sum(step_ms) / len(step_ms))
     gteps = 20 * m / (t_step * 1e-3) / 1e9
 
     # roofline of the dominant kernel (PR relax), live CUDA-event durations from the timed region
@@ -336,6 +349,10 @@ def main():
     if os.path.exists(tpath):
         traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
 
+    if world > torch.cuda.device_count():
+        rec_note = f"{world} ranks share {torch.cuda.device_count()} GPU(s): a protocol test, not a scaling number"
+    else:
+        rec_note = None
     result = {
         "metric": metric_name(args), "value": gteps, "unit": "GTEPS", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": t_step, "ms_per_step_median": statistics.median(step_ms),
@@ -351,6 +368,8 @@ def main():
         "algo_gteps": 20 * m / (statistics.mean(phase[2]) * 1e-3) / 1e9,
         "nv": my_nv, "gpu_launches": launches, "clocks": clk,
     }
+    if rec_note:
+        result["note"] = rec_note
 
     # e2e through the public API with HOST buffers (pinned), H2D and D2H inside the timed region
     if not args.no_e2e and not args.profile:
@@ -367,11 +386,7 @@ def main():
             e1.record(s)
             torch.cuda.synchronize()
             e2e.append(e0.elapsed_time(e1))
-        te = sum(e2e) / len(e2e)
-        if world > 1:
-            tt = torch.tensor([te], dtype=torch.float64, device="cuda")
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            te = float(tt.item())
+        te = allmax(sum(e2e) / len(e2e))
         # Streaming variant (reported beside, not instead): step i+1's arc list is copied on a
         # second stream while step i computes -- the same public API on device buffers, every
         # step's H2D and D2H still inside the timed region (first copy to last readback).
@@ -406,11 +421,7 @@ def main():
             freed[i % 2].record(s)
         p1.record(s)
         torch.cuda.synchronize()
-        tp = p0.elapsed_time(p1) / ksteps
-        if world > 1:
-            tt = torch.tensor([tp], dtype=torch.float64, device="cuda")
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            tp = float(tt.item())
+        tp = allmax(p0.elapsed_time(p1) / ksteps)
         # e2e = the pipelined run (what a user streaming batches gets; every step's H2D and
         # D2H are inside the timed region); the unpipelined one is reported beside it
         result["e2e"] = {"value": 20 * m / (tp * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": tp,
@@ -423,6 +434,9 @@ def main():
 
     if not args.no_extra and not args.profile and world == 1:
         result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy(), peak)
+
+    if not args.no_extra and not args.profile and world > 1:
+        result["per_algo_multi"] = per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax)
 
     if not args.no_extra and not args.no_configs and not args.profile and world == 1:
         result["per_config"] = per_config(tigr, torch, s, peak)
@@ -439,6 +453,60 @@ def main():
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def job_name(tag):
+    """A name unique to this torchrun job (node communicator shared-memory segment)."""
+    return f"bench_{tag}_{os.environ.get('MASTER_PORT', '0')}_{os.environ.get('TORCHELASTIC_RUN_ID', 'x')}"
+
+
+def per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax):
+    """N > 1: BFS / SSSP / CC on the scale-24 graph across the ranks with the FUSED exchange
+    (the relax applies each improvement to every peer replica over NVLink; node communicator,
+    CUDA IPC) -- the multi-GPU frontier path.  Every rank holds the whole graph and relaxes its
+    arc-balanced virtual node range; time = max over ranks of the device time of the run;
+    matches_single_gpu: every rank's values equal a one-GPU run of the same graph on its GPU.
+    Failures are recorded, not raised, after every rank has reached the same point."""
+    os.environ.setdefault("TIGR_GROUP_TIMEOUT", "120")
+    n, m = rec.n, rec.m
+    res = {"exchange": "fused", "transport": "node (CUDA IPC + shared memory)"}
+    try:
+        comm = tigr.tigr_comm_init_node(job_name("frontier"), world, rank)
+    except Exception as e:  # every rank fails the same way (segment or barrier timeout)
+        res["error"] = repr(e)
+        return res
+    for algo in ("bfs", "sssp", "cc"):
+        sym = algo == "cc"
+        entry = {}
+        try:
+            g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax,
+                                     weighted=not sym, symmetrize=sym, stream=s)
+            vg1 = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+            ref = torch.empty(n, dtype=torch.int32, device="cuda")
+            tigr.tigr_run(vg1, algo, 0, out=ref, stream=s)
+            vg1.free()
+            vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+            tigr.tigr_vgraph_partition(vg, world, rank)
+            out = torch.empty(n, dtype=torch.int32, device="cuda")
+            ts = []
+            for _ in range(3):
+                _, st = tigr.tigr_run(vg, algo, 0, out=out, comm=comm, exchange="fused", stream=s,
+                                      return_stats=True)
+                ts.append(st["ms_total"])
+            torch.cuda.synchronize()
+            entry = {"ms_rank": statistics.median(ts), "iterations": st["iterations"],
+                     "matches_single_gpu": bool(torch.equal(out, ref))}
+            vg.free()
+            g.free()
+        except Exception as e:
+            entry = {"error": repr(e)}
+        t = allmax(entry.get("ms_rank", float("inf")))
+        ok = allmax(0.0 if entry.get("matches_single_gpu") else 1.0) == 0.0
+        m_arcs = 2 * m if sym else m
+        res[algo] = {"ms": t, "gteps_arcs": m_arcs / (t * 1e-3) / 1e9 if t != float("inf") else None,
+                     "matches_single_gpu_all_ranks": ok, **{k: v for k, v in entry.items() if k != "ms_rank"}}
+    comm.free()
+    return res
 
 
 def frontier_bytes(algo, st, n):
