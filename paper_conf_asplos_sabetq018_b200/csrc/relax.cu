@@ -749,14 +749,15 @@ __device__ __forceinline__ void block_add(double v, double* dst) {
 }
 
 __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
-                          double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl) {
+                          double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl,
+                          const uint32_t* __restrict__ oid) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
     double dang = 0.0;
     if (v < n) {
         const double x0 = 1.0 / (double)n;
         const uint32_t d = deg[v];
         x[v] = x0;
-        contrib[v] = d ? __ddiv_rn(x0, (double)d) : 0.0;
+        contrib[oid ? oid[v] : v] = d ? __ddiv_rn(x0, (double)d) : 0.0;
         acc[v] = 0.0;
         if (!d) dang = x0;
     }
@@ -766,7 +767,8 @@ __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* 
 // x = (1-d)/n + d*(acc + dsum/n);  contrib = x/deg;  acc = 0;  next dangling mass -> dsum_next
 __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double base, double damping,
                            int dangling, double* __restrict__ x, double* __restrict__ contrib,
-                           double* __restrict__ acc, const double* dsum_cur, double* dsum_next) {
+                           double* __restrict__ acc, const double* dsum_cur, double* dsum_next,
+                           const uint32_t* __restrict__ oid) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
     double dang = 0.0;
     if (v < n) {
@@ -775,7 +777,7 @@ __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double 
         const double r = __dadd_rn(base, __dmul_rn(damping, s));  // no FMA: matches the oracle
         const uint32_t d = deg[v];
         x[v] = r;
-        contrib[v] = d ? __ddiv_rn(r, (double)d) : 0.0;
+        contrib[oid ? oid[v] : v] = d ? __ddiv_rn(r, (double)d) : 0.0;
         acc[v] = 0.0;
         if (!d) dang = r;
     }

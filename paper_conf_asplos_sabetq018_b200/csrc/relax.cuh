@@ -109,10 +109,14 @@ tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, 
                         cudaStream_t s, const FusedPeers** out);
 tigr_status fused_barrier(tigr_comm* c, cudaStream_t s);
 tigr_status fused_end_iteration(tigr_comm* c, Ctl* ctl, cudaStream_t s);
+// oid (nullable): contrib is stored at oid[v] instead of v (pull PageRank's source order, pr.cu)
 __global__ void k_pr_init(uint32_t n, const uint32_t* __restrict__ deg, double* __restrict__ x,
-                          double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl);
+                          double* __restrict__ contrib, double* __restrict__ acc, Ctl* ctl,
+                          const uint32_t* __restrict__ oid);
 __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double base, double damping,
                            int dangling, double* __restrict__ x, double* __restrict__ contrib,
-                           double* __restrict__ acc, const double* dsum_cur, double* dsum_next);
+                           double* __restrict__ acc, const double* dsum_cur, double* dsum_next,
+                           const uint32_t* __restrict__ oid);
+tigr_status pr_pull_prepare(tigr_vgraph* vg, cudaStream_t s);  // oid order + remapped in-arcs (pr.cu)
 
 }  // namespace tigr

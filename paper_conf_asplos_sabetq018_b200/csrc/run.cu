@@ -310,6 +310,15 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         TIGR_TRY(pr_cid_prepare(vg, s));
         cp = pr_cid_plan(vg);
     }
+    // pull: sources in out-degree order (pr.cu pr_pull_prepare); TIGR_PR_PULL_OID=0 disables
+    const char* po = getenv("TIGR_PR_PULL_OID");
+    const bool pull_oid = pull && vg->vec && !(po && atoi(po) == 0);
+    const uint32_t* oid = nullptr;
+    if (pull_oid) {
+        TIGR_TRY(pr_pull_prepare(vg, s));
+        oid = ws.cid.as<uint32_t>();
+        a.col = ws.col_pr.as<uint32_t>();
+    }
     const PrHotConfig hc =
         (pull || o.collect_stats || use_cid) ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
     const RelaxHotFn hot = hc.fn;
@@ -350,7 +359,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     TIGR_CK(cudaEventRecord(t0, s));
     TIGR_CK(cudaMemsetAsync(a.ctl, 0, sizeof(Ctl), s));
     k_pr_init<<<grid_for(n), kBlock, 0, s>>>(n, out_deg, ws.x.as<double>(), ws.contrib.as<double>(),
-                                             ws.acc.as<double>(), a.ctl);
+                                             ws.acc.as<double>(), a.ctl, oid);
     TIGR_CKL("pr init");
     trace(s, "pr: prepare+init");
     double ms_relax = 0.0, ms_ex = 0.0;
@@ -390,7 +399,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         }
         k_pr_apply<<<grid_for(n), kBlock, 0, s>>>(n, out_deg, base, o.pr_damping, o.pr_dangling,
                                                   ws.x.as<double>(), ws.contrib.as<double>(), ws.acc.as<double>(),
-                                                  dcur, dnext);
+                                                  dcur, dnext, oid);
         TIGR_CKL("pr apply");
     }
     TIGR_CK(cudaEventRecord(t1, s));
