@@ -30,12 +30,15 @@ import numpy as np  # noqa: E402
 # Algorithmic bytes of the push relax (fixed before measurement; DESIGN.md
 # "Roofline"): per processed arc s_e + s_v (read the target value) -- PageRank: s_e + 2 s_v
 # (RED = read + write of acc[dst]); per virtual node 4 (vn_phys); per node with d > 0 the
-# source value + its row_ptr pair (s_v + 8).
+# source value + its row_ptr pair (s_v + 8).  The PageRank relax runs with the apply fused in
+# (pr.cu PrFuse): its source value is derived from the previous accumulator, so per node with
+# d > 0 it reads acc_prev[cid[v]] (8) + cid[v] (4) + the row pair (8) instead of contrib (8) +
+# the row pair.
 S_E = 4
 
 
-def relax_bytes_pr(m, nv, n_out):
-    return m * (S_E + 16) + nv * 4 + n_out * (8 + 8)
+def relax_bytes_pr(m, nv, n_out, fused=True):
+    return m * (S_E + 16) + nv * 4 + n_out * ((8 + 4 + 8) if fused else (8 + 8))
 
 
 def pr_apply_bytes(n):
@@ -360,7 +363,8 @@ def main():
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": config_obj(args, rec),
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": traffic, "kernel": "k_relax_pr_cid (PageRank push relax, pr.cu)",
+                     "traffic": traffic,
+                     "kernel": "k_relax_pr_cid (PageRank push relax with the apply fused in, pr.cu)",
                      "algorithmic_bytes_per_launch": bytes_launch, "avg_launch_ms": relax_avg_ms,
                      "peak_source": peak_src, "frac_vs_8000_GBps": achieved / 8000.0},
         "breakdown_ms": {"csr_build": statistics.mean(phase[0]), "virtualize": statistics.mean(phase[1]),

@@ -82,9 +82,14 @@ __global__ void k_build_col_pr(const uint4* __restrict__ c4, uint64_t nchunks, c
     }
 }
 
+// Fused apply (PrFuse): the relax of iteration t+1 computes each source's contribution from
+// the previous iteration's accumulator itself -- x = (1-d)/n + d*acc_t[cid[v]], contrib =
+// x/deg_v, the apply's exact arithmetic (no FMA) -- so the separate apply pass disappears;
+// x is materialised once, after the last iteration.  mode 0: read contrib[v] (unfused);
+// 1: first iteration, x = x0; 2: from acc_prev.
 template <int LAYOUT, int B, int T, int SLOTS, int MINB>
 __global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uint32_t* __restrict__ col_pr,
-                                                                   uint32_t tiles) {
+                                                                   uint32_t tiles, PrFuse fz) {
     extern __shared__ __align__(16) double s_acc[];  // SLOTS entries (dynamic: 64 KB)
     const int t = threadIdx.x;
     for (int i = t; i < SLOTS; i += T) s_acc[i] = 0.0;
@@ -105,11 +110,29 @@ __global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uin
         }
         uint4 info[B];
         double x[B];
+        uint32_t cv[B];
 #pragma unroll
         for (int r = 0; r < B; ++r) {
             info[r] = make_uint4(0, 0, 0, 1);
             x[r] = 0.0;
-            if (v[r] != kPad) { info[r] = __ldg(a.vinfo + v[r]); x[r] = __ldg(a.contrib + v[r]); }
+            cv[r] = 0xFFFFFFFFu;
+            if (v[r] != kPad) {
+                info[r] = __ldg(a.vinfo + v[r]);
+                if (fz.mode == 0) x[r] = __ldg(a.contrib + v[r]);
+                else if (fz.mode == 2) cv[r] = __ldg(fz.cid + v[r]);
+            }
+        }
+        if (fz.mode != 0) {
+#pragma unroll
+            for (int r = 0; r < B; ++r) {
+                if (v[r] == kPad) continue;
+                double xv = fz.x0;
+                if (fz.mode == 2) {
+                    const double s = cv[r] < fz.n_in ? __ldg(fz.prev + cv[r]) : 0.0;
+                    xv = __dadd_rn(fz.base, __dmul_rn(fz.damping, s));  // = k_pr_apply_cid's x
+                }
+                x[r] = __ddiv_rn(xv, (double)info[r].y);                 // = its contrib (deg > 0 here)
+            }
         }
         uint4 c0[B], c1[B];
         uint32_t kn[B], kend[B], step[B];
@@ -298,6 +321,7 @@ tigr_status pr_pull_prepare(tigr_vgraph* vg, cudaStream_t s) {
 
 template <int B, int T, int SLOTS, int MINB>
 static void fill_plan(PrCidPlan& p, int layout) {
+    static_assert(B >= 1, "");
     p.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, B, T, SLOTS, MINB>
                                          : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, B, T, SLOTS, MINB>;
     p.threads = T;
@@ -331,15 +355,16 @@ PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
 }
 
 tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,
-                         double* dsum_next, cudaStream_t s) {
+                         double* dsum_next, cudaStream_t s, double* acc, bool reset) {
     Workspace& ws = vg->ws;
     const uint32_t n = vg->g->n;
+    if (!acc) acc = ws.acc.as<double>();
     k_pr_apply_cid<<<grid_for(n), kBlock, 0, s>>>(n, vg->g->deg.as<uint32_t>(), ws.cid.as<uint32_t>(), ws.n_in, base,
                                                   damping, dangling, ws.x.as<double>(), ws.contrib.as<double>(),
-                                                  ws.acc.as<double>(), dsum_cur, dsum_next);
+                                                  acc, dsum_cur, dsum_next);
     TIGR_CKL("pr apply (cid)");
     // only the first n_in accumulator entries are ever written
-    TIGR_CK(cudaMemsetAsync(ws.acc.p, 0, sizeof(double) * ws.n_in, s));
+    if (reset) TIGR_CK(cudaMemsetAsync(acc, 0, sizeof(double) * ws.n_in, s));
     return TIGR_OK;
 }
 

@@ -67,8 +67,15 @@ struct PrHotConfig {
 };
 PrHotConfig relax_pr_hot_config(int layout, bool vec);
 // PageRank push with an in-degree-ordered accumulator (pr.cu)
+struct PrFuse {
+    int mode = 0;               // 0 read contrib, 1 first iteration (x = x0), 2 from prev
+    uint32_t n_in = 0;
+    const double* prev = nullptr;  // accumulator of the previous iteration (cid order)
+    const uint32_t* cid = nullptr;
+    double base = 0.0, damping = 0.0, x0 = 0.0;
+};
 struct PrCidPlan {
-    void (*fn)(RelaxArgs, const uint32_t*, uint32_t) = nullptr;
+    void (*fn)(RelaxArgs, const uint32_t*, uint32_t, PrFuse) = nullptr;
     unsigned grid = 0, tiles = 0;
     int threads = 256, per_thread = 4;
     size_t smem = 0;
@@ -78,7 +85,7 @@ RelaxFn relax_pr_pull_kernel(int layout, int* per_thread);   // pull PageRank (p
 tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s);
 PrCidPlan pr_cid_plan(tigr_vgraph* vg);
 tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,
-                         double* dsum_next, cudaStream_t s);
+                         double* dsum_next, cudaStream_t s, double* acc = nullptr, bool reset = true);
 uint32_t pr_hot_max();        // capacity of the workspace's hot-id list (>= any config's max_ids)
 tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uint32_t max_ids, uint32_t* cnt_tmp,
                           uint32_t* hist_tmp, uint32_t* hot_ids, uint32_t* n_hot, cudaStream_t s);

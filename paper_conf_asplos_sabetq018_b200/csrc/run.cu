@@ -310,6 +310,11 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         TIGR_TRY(pr_cid_prepare(vg, s));
         cp = pr_cid_plan(vg);
     }
+    // fused apply (pr.cu PrFuse): the relax derives contributions from the previous accumulator;
+    // two accumulators alternate; dangling-mass redistribution keeps the separate apply
+    const char* fe = getenv("TIGR_PR_FUSE");
+    const bool fuse = use_cid && !o.pr_dangling && !(fe && atoi(fe) == 0) && o.pr_iters > 0;
+    if (fuse && !ws.acc2.p) TIGR_TRY(ws.acc2.alloc(sizeof(double) * (n ? n : 1), s));
     // pull: sources in out-degree order (pr.cu pr_pull_prepare); TIGR_PR_PULL_OID=0 disables
     const char* po = getenv("TIGR_PR_PULL_OID");
     const bool pull_oid = pull && vg->vec && !(po && atoi(po) == 0);
@@ -373,8 +378,22 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     }
     for (uint32_t t = 0; t < o.pr_iters; ++t) {
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t], s));
+        double* acc_cur = ws.acc.as<double>();
+        PrFuse fz;
+        if (fuse) {
+            acc_cur = (t & 1) ? ws.acc2.as<double>() : ws.acc.as<double>();
+            fz.mode = t == 0 ? 1 : 2;
+            fz.n_in = ws.n_in;
+            fz.prev = (t & 1) ? ws.acc.as<double>() : ws.acc2.as<double>();
+            fz.cid = ws.cid.as<uint32_t>();
+            fz.base = base;
+            fz.damping = o.pr_damping;
+            fz.x0 = 1.0 / (double)n;
+            if (t > 0) TIGR_CK(cudaMemsetAsync(acc_cur, 0, sizeof(double) * ws.n_in, s));
+            a.acc = acc_cur;
+        }
         if (use_cid && cp.tiles) {
-            cp.fn<<<cp.grid, cp.threads, cp.smem, s>>>(a, ws.col_pr.as<uint32_t>(), cp.tiles);
+            cp.fn<<<cp.grid, cp.threads, cp.smem, s>>>(a, ws.col_pr.as<uint32_t>(), cp.tiles, fz);
             TIGR_CKL("pr relax (cid)");
             ++launches;
         } else if (hot && hot_tiles) {
@@ -388,11 +407,15 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         }
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t + 1], s));
         // in accumulator-id order only the first n_in entries are ever written (pr.cu)
-        if (comm) TIGR_TRY(comm_allreduce(o.comm, ws.acc.p, use_cid ? ws.n_in : n, TIGR_PR, s));
+        if (comm) TIGR_TRY(comm_allreduce(o.comm, acc_cur, use_cid ? ws.n_in : n, TIGR_PR, s));
         if (o.time_kernels) TIGR_CK(cudaEventRecord(ws.tev[3 * t + 2], s));
         double* dcur = &a.ctl->dsum[t & 1];
         double* dnext = &a.ctl->dsum[(t + 1) & 1];
         if (o.pr_dangling) TIGR_CK(cudaMemsetAsync(dnext, 0, sizeof(double), s));
+        if (fuse) {  // x itself only after the last iteration
+            if (t + 1 == o.pr_iters) TIGR_TRY(pr_cid_apply(vg, base, o.pr_damping, 0, dcur, dnext, s, acc_cur, false));
+            continue;
+        }
         if (use_cid) {
             TIGR_TRY(pr_cid_apply(vg, base, o.pr_damping, o.pr_dangling, dcur, dnext, s));
             continue;

@@ -50,6 +50,7 @@ struct Workspace {
     DevBuf x;        // double[n] PR rank
     DevBuf contrib;  // double[n] PR x/deg
     DevBuf acc;      // double[n] PR accumulator
+    DevBuf acc2;     // double[n] second accumulator (fused apply alternates the two; pr.cu)
     DevBuf hot;      // uint32: PR hot-destination selection {count[n], hist[33], n_hot, ids[max]}
     DevBuf cid;      // uint32[n]: PR accumulator id (in-degree order; pr.cu)
     DevBuf col_pr;   // uint32[4 * nchunks]: arc targets as accumulator ids (PR only)
