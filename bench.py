@@ -459,9 +459,19 @@ def main():
         dist.destroy_process_group()
 
 
+_JOB_TOKEN = []
+
+
 def job_name(tag):
-    """A name unique to this torchrun job (node communicator shared-memory segment)."""
-    return f"bench_{tag}_{os.environ.get('MASTER_PORT', '0')}_{os.environ.get('TORCHELASTIC_RUN_ID', 'x')}"
+    """A name unique to this job (node communicator shared-memory segment): rank 0 draws a
+    random token and broadcasts it, so no rank can attach to a stale segment of another run."""
+    import torch.distributed as dist
+    if not _JOB_TOKEN:
+        import uuid
+        tok = [uuid.uuid4().hex[:16] if dist.get_rank() == 0 else None]
+        dist.broadcast_object_list(tok, src=0)
+        _JOB_TOKEN.append(tok[0])
+    return f"bench_{tag}_{_JOB_TOKEN[0]}"
 
 
 def per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax):
