@@ -296,6 +296,24 @@ def test_pr_dangling_redistribute(tigr):
     assert abs(got.sum() - 1.0) < 1e-9  # redistribute conserves mass
 
 
+@pytest.mark.parametrize("fuse", ["0", "1"])
+def test_pr_iteration_counts_and_fused_apply(tigr, fuse, monkeypatch):
+    """PageRank after 0, 1, 2, 3 and 20 iterations, with the apply fused into the relax
+    (default) and separate (TIGR_PR_FUSE=0): the two accumulators alternate correctly and x is
+    materialised after the last iteration; damping 0.5 and 1.0 exercise the constants."""
+    monkeypatch.setenv("TIGR_PR_FUSE", fuse)
+    rec = graphgen.recipe("cfg1")
+    src, dst, _ = graphgen.generate(rec)
+    o = oracle.csr_build(rec.n, src, dst)
+    vg = tigr.tigr_virtualize(tigr.tigr_graph_from_coo(rec.n, src, dst, None), 8)
+    for iters in (0, 1, 2, 3, 20):
+        got = tigr.tigr_run(vg, "pr", pr_iters=iters)
+        assert np.abs(got - oracle.pagerank(o, iters)).max() <= 1e-15, iters
+    for d in (0.5, 1.0):
+        got = tigr.tigr_run(vg, "pr", pr_iters=7, pr_damping=d)
+        assert np.abs(got - oracle.pagerank(o, 7, d)).max() <= 1e-15, d
+
+
 def test_errors(tigr):
     src, dst, w = graphgen.random_small(10, 30, 1)
     g = tigr.tigr_graph_from_coo(10, src, dst, None)
