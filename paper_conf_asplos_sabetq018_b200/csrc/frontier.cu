@@ -41,6 +41,9 @@
 // atomicMin whose candidate beat the observed level (the level then ends at it, final), so a
 // set bit never hides an improvement; a stale clear bit (another SM's atomicOr not yet
 // visible through this SM's L1) only costs the level gather the plain test would have done.
+// CC uses the same bitmap for one exact case: a label lowered to 0, the smallest id, is
+// final (nothing is better than 0), and on power-law graphs the giant component -- most
+// targets -- carries label 0 after the first iterations.
 #include <algorithm>
 
 #include "devutil.cuh"
@@ -128,7 +131,7 @@ __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, ui
 template <int A, int LAYOUT, bool BSP, int B, bool STATS, int MINB, bool PRE>
 __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
-    const bool BITS = A == TIGR_BFS && f.settled != nullptr;  // uniform per launch
+    const bool BITS = (A == TIGR_BFS || A == TIGR_CC) && f.settled != nullptr;  // uniform per launch
     const int lane = threadIdx.x & 31;
     const uint32_t it = a.ctl->it;
     const unsigned long long qp = a.ctl->qpack[it & 1u];
@@ -241,7 +244,8 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                     else atomicMin(a.val + nb[q], alt);
                     if (f.peers) push_peers<A>(f.peers, a.n, it, nb[q], alt);
                     // the level becomes alt = it, final (see the header): mark it settled
-                    if (BITS) atomicOr(f.settled + (nb[q] >> 5), 1u << (nb[q] & 31u));
+                    if (BITS && (A == TIGR_BFS || alt == 0u))  // CC: only label 0 is final
+                        atomicOr(f.settled + (nb[q] >> 5), 1u << (nb[q] & 31u));
                     stamp_next[nb[q]] = it + 1;
                     touched = true;
                     if (STATS) ++n_upd;

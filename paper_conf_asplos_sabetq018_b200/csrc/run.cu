@@ -150,8 +150,8 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         p.fa.dense_div = d ? (uint32_t)atoi(d) : 2u;
         p.fa.settled = nullptr;
         p.fa.peers = nullptr;
-        const char* bb = getenv("TIGR_BFS_BITS");  // development knob: 0 = test the levels instead
-        if (algo == TIGR_BFS && !(bb && atoi(bb) == 0)) {
+        const char* bb = getenv("TIGR_BFS_BITS");  // development knob: 0 = test the values instead
+        if ((algo == TIGR_BFS || algo == TIGR_CC) && !(bb && atoi(bb) == 0)) {
             if (!ws.settled.p) TIGR_TRY(ws.settled.alloc(sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
             p.fa.settled = ws.settled.as<uint32_t>();
         }
