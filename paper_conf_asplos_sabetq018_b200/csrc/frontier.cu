@@ -384,8 +384,8 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
 
 // Kernel shape per algorithm (cfg4 sweep, tools/dev/fq_sweep.sh): the relax
 // is bound by L1tex wavefronts of the random target-value gathers and by latency, so
-// occupancy matters more than per-thread depth.  CC: 4 vnodes per thread, 80 registers,
-// 3 blocks/SM; BFS: see pick_fq.  Weighted (SSSP, SSWP; one more 16-byte load per chunk): 2 vnodes
+// occupancy matters more than per-thread depth.  BFS and CC (settled bitmap): see pick_fq;
+// BSP / stats variants: 4 vnodes per thread, 80 registers, 3 blocks/SM.  Weighted (SSSP, SSWP; one more 16-byte load per chunk): 2 vnodes
 // per thread with all target gathers of both issued before the first atomic, 3 blocks/SM.
 template <int A, int LAYOUT>
 static FqFn pick_fq(bool bsp, bool stats) {
@@ -394,10 +394,10 @@ static FqFn pick_fq(bool bsp, bool stats) {
     constexpr bool PRE = W;
     if (!bsp && !stats) {  // development knob: alternative shapes (TIGR_FQ_SHAPE)
         const char* e = getenv("TIGR_FQ_SHAPE");
-        // BFS with its settled bitmap is latency-bound rather than L1/L2-bound
+        // BFS and CC with their settled bitmap are latency-bound rather than L1/L2-bound
         // (profiles/README.md): 2 virtual nodes per thread with all gathers issued first,
-        // 4 blocks/SM (64 registers, no spills), 1.47 -> 1.34 ms at cfg4
-        const int dflt = (A == TIGR_BFS) ? 1 : 0;
+        // 4 blocks/SM (64 registers, no spills); cfg4 BFS 1.47 -> 1.34 ms, CC 3.44 -> 3.07 ms
+        const int dflt = (A == TIGR_BFS || A == TIGR_CC) ? 1 : 0;
         switch (e ? atoi(e) : dflt) {
             case 1: return &k_relax_fq<A, LAYOUT, false, 2, false, 4, true>;
             case 2: return &k_relax_fq<A, LAYOUT, false, 4, false, 4, false>;
