@@ -631,7 +631,9 @@ def per_config(tigr, torch, s, peak):
     16, 32, cfg5 BFS / SSSP / CC.  Arc list drawn on the device (tigr_rmat_coo), CSR built from
     it (build_ms), virtual split at K (strided), then per algorithm: one stats run
     (processed arcs), the median of 3 device-timed runs (CUDA-graph loop), and one run with
-    per-relax CUDA events.  gteps_input = arcs out of reached nodes (CC: all 2m arcs) / time."""
+    per-relax CUDA events; then the median of 3 runs on the in-degree-reordered copy
+    (tigr_graph_reorder, its one-off cost in reorder_ms; results in original ids).
+    gteps_input = arcs out of reached nodes (CC: all 2m arcs) / time."""
     import graphgen
 
     plan = {"cfg2": [("bfs", 8), ("cc", 8)],
@@ -662,6 +664,12 @@ def per_config(tigr, torch, s, peak):
                 e1.record(s)
                 torch.cuda.synchronize()
                 entry["build_ms_sym" if sym else "build_ms"] = e0.elapsed_time(e1)
+                # the in-degree-reordered copy (one-off cost reported like the build)
+                e0.record(s)
+                graphs[(sym, "r")] = tigr.tigr_graph_reorder(graphs[sym], stream=s)
+                e1.record(s)
+                torch.cuda.synchronize()
+                entry["reorder_ms_sym" if sym else "reorder_ms"] = e0.elapsed_time(e1)
             vg = tigr.tigr_virtualize(graphs[sym], K, "strided", stream=s)
             _, st = tigr.tigr_run(vg, algo, rec.source, out=out, stream=s, collect_stats=1, return_stats=True)
             ts = []
@@ -683,6 +691,16 @@ def per_config(tigr, torch, s, peak):
                 "roofline_frac": nbytes / (st3["ms_relax"] * 1e-3) / 1e9 / peak if st3["ms_relax"] else None,
                 "nv": vg.info()["nv"]}
             vg.free()
+            # same run on the reordered graph (values come back in original ids)
+            vgr = tigr.tigr_virtualize(graphs[(sym, "r")], K, "strided", stream=s)
+            tr = []
+            for _ in range(3):
+                _, st4 = tigr.tigr_run(vgr, algo, rec.source, out=out, stream=s, return_stats=True)
+                tr.append(st4["ms_total"])
+            tr_med = statistics.median(tr)
+            entry[f"{algo}_K{K}"]["ms_reordered"] = tr_med
+            entry[f"{algo}_K{K}"]["gteps_input_reordered"] = m_in / (tr_med * 1e-3) / 1e9
+            vgr.free()
         for g in graphs.values():
             g.free()
         del src, dst, w, deg, out
