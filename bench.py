@@ -523,11 +523,23 @@ def per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax):
             torch.cuda.synchronize()
             entry = {"ms_rank": statistics.median(ts), "iterations": st["iterations"],
                      "matches_single_gpu": bool(torch.equal(out, ref))}
+            for mode in ("sparse", "dense"):  # the other exchanges, for comparison
+                tm = []
+                for _ in range(3):
+                    _, stm = tigr.tigr_run(vg, algo, 0, out=out, comm=comm, exchange=mode, stream=s,
+                                           return_stats=True)
+                    tm.append(stm["ms_total"])
+                torch.cuda.synchronize()
+                entry[f"ms_rank_{mode}"] = statistics.median(tm)
+                entry["matches_single_gpu"] = entry["matches_single_gpu"] and bool(torch.equal(out, ref))
             vg.free()
             g.free()
         except Exception as e:
             entry = {"error": repr(e)}
         t = allmax(entry.get("ms_rank", float("inf")))
+        for mode in ("sparse", "dense"):
+            if f"ms_rank_{mode}" in entry or "error" in entry:
+                entry[f"ms_{mode}"] = allmax(entry.pop(f"ms_rank_{mode}", float("inf")))
         ok = allmax(0.0 if entry.get("matches_single_gpu") else 1.0) == 0.0
         m_arcs = 2 * m if sym else m
         res[algo] = {"ms": t, "gteps_arcs": m_arcs / (t * 1e-3) / 1e9 if t != float("inf") else None,
