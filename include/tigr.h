@@ -219,6 +219,13 @@ tigr_status tigr_graph_permutation(const tigr_graph* g, uint32_t* cid, uint32_t*
 tigr_status tigr_graph_udt(const tigr_graph* g, uint32_t K, uint32_t dumb_weight, uint32_t unit_weight,
                            void* stream, tigr_graph** out);
 
+/* Copy the arc list out in CSR order: src[m], dst[m], w[m] (w only if weighted and != NULL);
+ * arc e is the e-th arc of the canonical CSR (Fig. 10a), so (src, dst, w) rebuilt by
+ * tigr_graph_from_coo gives the same graph.  Buffers are caller-owned, host or device
+ * (is_device_ptr), any of them may be NULL.  Errors: EINVAL (NULL graph). */
+tigr_status tigr_graph_export_coo(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w,
+                                  int is_device_ptr, void* stream);
+
 /* Copy the CSR out (row_ptr[n+1], col[m], w[m] if weighted and w != NULL), arcs of a
  * source contiguous in the graph's internal order. */
 tigr_status tigr_graph_export_csr(const tigr_graph* g, int64_t* row_ptr, uint32_t* col, uint32_t* w,

@@ -79,6 +79,7 @@ _SIGS = {
     "tigr_graph_reorder": (_I, [_P, _P, ctypes.POINTER(_P)]),
     "tigr_graph_permutation": (_I, [_P, _P, _P, _I, _P]),
     "tigr_graph_export_csr": (_I, [_P, _P, _P, _P, _I, _P]),
+    "tigr_graph_export_coo": (_I, [_P, _P, _P, _P, _I, _P]),
     "tigr_graph_free": (None, [_P]),
     "tigr_virtualize": (_I, [_P, _U32, _I, _P, ctypes.POINTER(_P)]),
     "tigr_vgraph_info": (_I, [_P, ctypes.POINTER(_U64), ctypes.POINTER(_U64), ctypes.POINTER(_D),
@@ -352,6 +353,18 @@ def tigr_graph_export_csr(g: Graph, stream=None):
     _check(_lib.tigr_graph_export_csr(g.ptr, rp.ctypes.data, col.ctypes.data,
                                       None if w is None else w.ctypes.data, 0, _stream_ptr(stream)))
     return rp, col, w
+
+
+def tigr_graph_export_coo(g: Graph, stream=None):
+    """Host copies (src uint32[m], dst uint32[m], w uint32[m] or None) in canonical CSR order."""
+    info = g.info()
+    m = info["m"]
+    src = np.empty(max(m, 1), dtype=np.uint32)
+    dst = np.empty(max(m, 1), dtype=np.uint32)
+    w = np.empty(max(m, 1), dtype=np.uint32) if info["weighted"] else None
+    _check(_lib.tigr_graph_export_coo(g.ptr, src.ctypes.data, dst.ctypes.data,
+                                      None if w is None else w.ctypes.data, 0, _stream_ptr(stream)))
+    return src[:m], dst[:m], (None if w is None else w[:m])
 
 
 def tigr_virtualize(g: Graph, K: int = 8, layout="strided", stream=None) -> VGraph:

@@ -189,6 +189,7 @@ tigr_status coo_source_cuts(uint32_t n, uint64_t m, const uint32_t* src, const u
 tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col, const uint32_t* w,
                                   int symmetric_hint, cudaStream_t s, tigr_graph** out);
 tigr_status graph_export_csr_device(const tigr_graph* g, int64_t* rp, uint32_t* col, uint32_t* w, cudaStream_t s);
+tigr_status expand_arcs(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w, cudaStream_t s);
 tigr_status graph_transpose_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out);
 tigr_status graph_reorder_device(const tigr_graph* g, cudaStream_t s, tigr_graph** out);
 tigr_status graph_udt_device(const tigr_graph* g, uint32_t K, uint32_t dumb, uint32_t unit, cudaStream_t s,
@@ -354,6 +355,28 @@ tigr_status tigr_graph_info(const tigr_graph* g, uint32_t* n, uint64_t* m, int* 
     if (symmetric) *symmetric = g->symmetric;
     if (transposed) *transposed = g->transposed;
     if (device_bytes) *device_bytes = g->row_ptr.bytes + g->deg.bytes + g->cptr.bytes + g->col.bytes + g->wt.bytes;
+    return TIGR_OK;
+}
+
+tigr_status tigr_graph_export_coo(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w,
+                                  int is_device_ptr, void* stream) {
+    if (!g) return fail(TIGR_EINVAL, "graph_export_coo: NULL graph");
+    cudaStream_t s = (cudaStream_t)stream;
+    const size_t bytes = sizeof(uint32_t) * (g->m ? g->m : 1);
+    TmpBuf ds, dd, dw;  // the expansion writes all three; unwanted ones go to scratch
+    uint32_t* ps = (is_device_ptr && src) ? src : nullptr;
+    uint32_t* pd = (is_device_ptr && dst) ? dst : nullptr;
+    uint32_t* pw = (is_device_ptr && w) ? w : nullptr;
+    if (!ps) { TIGR_TRY(ds.alloc(bytes, s)); ps = ds.as<uint32_t>(); }
+    if (!pd) { TIGR_TRY(dd.alloc(bytes, s)); pd = dd.as<uint32_t>(); }
+    if (g->weighted && !pw) { TIGR_TRY(dw.alloc(bytes, s)); pw = dw.as<uint32_t>(); }
+    TIGR_TRY(expand_arcs(g, ps, pd, g->weighted ? pw : nullptr, s));
+    if (!is_device_ptr && g->m) {
+        if (src) TIGR_CK(cudaMemcpyAsync(src, ps, sizeof(uint32_t) * g->m, cudaMemcpyDeviceToHost, s));
+        if (dst) TIGR_CK(cudaMemcpyAsync(dst, pd, sizeof(uint32_t) * g->m, cudaMemcpyDeviceToHost, s));
+        if (w && g->weighted) TIGR_CK(cudaMemcpyAsync(w, pw, sizeof(uint32_t) * g->m, cudaMemcpyDeviceToHost, s));
+    }
+    TIGR_CK(cudaStreamSynchronize(s));
     return TIGR_OK;
 }
 

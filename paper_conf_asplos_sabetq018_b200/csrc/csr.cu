@@ -14,6 +14,8 @@
 
 namespace tigr {
 
+tigr_status expand_arcs(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w, cudaStream_t s);
+
 tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double b, double c,
                        uint64_t seed, uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src,
                        uint32_t* dst, uint32_t* w, cudaStream_t s);
@@ -143,19 +145,6 @@ __global__ void __launch_bounds__(256) k_expand_arcs(const int64_t* __restrict__
     }
 }
 
-tigr_status expand_arcs(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w, cudaStream_t s) {
-    if (g->m == 0 || g->n == 0) return TIGR_OK;
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const uint64_t tiles = (g->m + kExpTile - 1) / kExpTile;
-    const unsigned grid = (unsigned)std::min<uint64_t>(tiles, (uint64_t)sms * 8);
-    k_expand_arcs<<<grid, 256, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), g->n, g->m,
-                                       g->col.as<uint32_t>(), g->weighted ? g->wt.as<uint32_t>() : nullptr, src, dst,
-                                       w);
-    TIGR_CKL("expand arcs");
-    return TIGR_OK;
-}
 
 // ---- UDT (physical uniform-degree-tree transformation, §3.2 Alg. 1) ----
 // Node v of out-degree d > K gets t = ceil((d-K)/(K-1)) new split nodes.  Alg. 1's queue is
@@ -280,6 +269,20 @@ __global__ void k_relabel(uint32_t* __restrict__ src, uint32_t* __restrict__ dst
 }
 
 }  // namespace
+
+tigr_status expand_arcs(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint32_t* w, cudaStream_t s) {
+    if (g->m == 0 || g->n == 0) return TIGR_OK;
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t tiles = (g->m + kExpTile - 1) / kExpTile;
+    const unsigned grid = (unsigned)std::min<uint64_t>(tiles, (uint64_t)sms * 8);
+    k_expand_arcs<<<grid, 256, 0, s>>>(g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), g->n, g->m,
+                                       g->col.as<uint32_t>(), g->weighted ? g->wt.as<uint32_t>() : nullptr, src, dst,
+                                       w);
+    TIGR_CKL("expand arcs");
+    return TIGR_OK;
+}
 
 // src_lo/src_hi: keep only the arcs whose source lies in [src_lo, src_hi) (multi-GPU partitioned
 // builds); the in-degree sketch and the id validation still cover every arc
