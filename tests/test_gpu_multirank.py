@@ -299,3 +299,23 @@ def test_node_communicator_processes(tigr, exchange):
     errs = [(r, e) for r, _, e in res if e]
     assert not errs, errs
     _check(_want("s16"), [out for _, out, _ in sorted(res, key=lambda x: x[0])])
+
+
+def test_node_communicator_errors_and_single_rank(tigr):
+    import os
+    with pytest.raises(tigr.TigrError) as e:
+        tigr.tigr_comm_init_node("", 2, 0)
+    assert e.value.status == tigr.TIGR_EINVAL
+    with pytest.raises(tigr.TigrError) as e:
+        tigr.tigr_comm_init_node("x", 17, 0)
+    assert e.value.status == tigr.TIGR_EINVAL
+    with pytest.raises(tigr.TigrError) as e:
+        tigr.tigr_comm_init_node("x", 2, 2)
+    assert e.value.status == tigr.TIGR_EINVAL
+    c = tigr.tigr_comm_init_node(f"pytest1_{os.getpid()}", 1, 0)  # one rank: no peer, no wait
+    n, src, dst, w = _graph("cfg1")
+    vg = tigr.tigr_virtualize(tigr.tigr_graph_from_coo(n, src, dst, w), 8)
+    for ex in ("dense", "sparse", "fused", "auto"):
+        assert np.array_equal(tigr.tigr_run(vg, "sssp", 0, comm=c, exchange=ex), _want("cfg1")["sssp"]), ex
+    assert np.abs(tigr.tigr_run(vg, "pr", comm=c) - _want("cfg1")["pr"]).max() <= 1e-6
+    c.free()
