@@ -488,20 +488,36 @@ def job_name(tag):
 
 
 def per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax):
+    import graphgen
     """N > 1: BFS / SSSP / CC on the scale-24 graph across the ranks with the FUSED exchange
     (the relax applies each improvement to every peer replica over NVLink; node communicator,
     CUDA IPC) -- the multi-GPU frontier path.  Every rank holds the whole graph and relaxes its
     arc-balanced virtual node range; time = max over ranks of the device time of the run;
     matches_single_gpu: every rank's values equal a one-GPU run of the same graph on its GPU.
     Failures are recorded, not raised, after every rank has reached the same point."""
-    os.environ.setdefault("TIGR_GROUP_TIMEOUT", "120")
     n, m = rec.n, rec.m
     res = {"exchange": "fused", "transport": "node (CUDA IPC + shared memory)"}
+    # probe first, with a short barrier timeout: if shared memory or CUDA IPC is unavailable
+    # here, every rank learns it within seconds and the section is skipped on all of them
+    os.environ["TIGR_GROUP_TIMEOUT"] = "30"
+    comm, err = None, None
     try:
         comm = tigr.tigr_comm_init_node(job_name("frontier"), world, rank)
-    except Exception as e:  # every rank fails the same way (segment or barrier timeout)
-        res["error"] = repr(e)
+        small = graphgen.recipe("cfg1")
+        gs = tigr.tigr_graph_rmat(small.n, small.m, small.a, small.b, small.c, small.seed, small.wseed,
+                                  stream=s)
+        vgs = tigr.tigr_virtualize(gs, args.K, args.layout, stream=s)
+        tigr.tigr_vgraph_partition(vgs, world, rank)
+        tigr.tigr_run(vgs, "sssp", 0, comm=comm, exchange="fused", stream=s)
+        tigr.tigr_run(vgs, "sssp", 0, comm=comm, exchange="sparse", stream=s)
+        vgs.free()
+        gs.free()
+    except Exception as e:
+        err = repr(e)
+    if allmax(1.0 if err else 0.0) != 0.0:
+        res["error"] = err or "a peer rank failed the node-communicator probe"
         return res
+    os.environ["TIGR_GROUP_TIMEOUT"] = "120"
     for algo in ("bfs", "sssp", "cc"):
         sym = algo == "cc"
         entry = {}
