@@ -10,6 +10,9 @@ processed every iteration).  The other configs are parity-test cases (tests/).
 
   python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--config cfg4]
 Multi-GPU: torchrun --nproc-per-node N bench.py --gpus N ...  (vnode ranges, NCCL all-reduce).
+
+The algorithmic byte model of every relax launch is computed inside libtigr
+(tigr_stats.bytes_alg, run.cu), so the roofline fractions here and the library agree.
 """
 from __future__ import annotations
 
@@ -27,22 +30,24 @@ sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402
 
-# Algorithmic bytes of the push relax (fixed before measurement; DESIGN.md
-# "Roofline"): per processed arc s_e + s_v (read the target value) -- PageRank: s_e + 2 s_v
-# (RED = read + write of acc[dst]); per virtual node 4 (vn_phys); per node with d > 0 the
-# source value + its row_ptr pair (s_v + 8).  The PageRank relax runs with the apply fused in
-# (pr.cu PrFuse): its source value is derived from the previous accumulator, so per node with
-# d > 0 it reads acc_prev[cid[v]] (8) + cid[v] (4) + the row pair (8) instead of contrib (8) +
-# the row pair.
-S_E = 4
-
-
-def relax_bytes_pr(m, nv, n_out, fused=True):
-    return m * (S_E + 16) + nv * 4 + n_out * ((8 + 4 + 8) if fused else (8 + 8))
-
-
-def pr_apply_bytes(n):
-    return n * 28
+# Paper context (never the target): Tigr-V+ on an NVIDIA Quadro P4000 (Pascal,
+# sm_61, CUDA 8), Table 4 runtimes (L1276-1310) and Fig. 13's average SSSP
+# speedup over the same engine without the transformation (L1341-1367, L1398-1412).
+PAPER_CONTEXT = {
+    "gpu": "NVIDIA Quadro P4000 (Pascal GP104, sm_61, ~243 GB/s), CUDA 8.0 (PAPER.md L1244-1249)",
+    "table4_tigr_v_plus_ms": {
+        "source": "PAPER.md Table 4, L1276-1310 (real graphs; GTEPS = m / t is BASELINE.md's derivation)",
+        "sssp_livejournal": {"ms": 62.21, "n": 4.0e6, "m": 69e6, "derived_gteps": 1.11},
+        "sswp_livejournal": {"ms": 65.67, "n": 4.0e6, "m": 69e6, "derived_gteps": 1.05},
+        "bfs_twitter": {"ms": 178.53, "n": 21e6, "m": 530e6, "derived_gteps": 2.97},
+        "sssp_twitter": {"ms": 269.75, "n": 21e6, "m": 530e6, "derived_gteps": 1.96},
+        "cc_twitter": {"ms": 573.53, "n": 21e6, "m": 530e6, "derived_gteps": 0.92},
+        "pr_twitter": {"ms": 221.49, "n": 21e6, "m": 530e6, "derived_gteps_per_run": 2.39},
+    },
+    "fig13_sssp_speedup_over_no_transform": {"tigr_v_plus": 2.1, "tigr_v": 1.7, "tigr_udt": 1.2,
+                                             "source": "PAPER.md Fig. 13, L1341-1367, L1398-1412"},
+    "note": "context only: other GPU, real graphs; this build's own ablation is DESIGN.md §12",
+}
 
 
 def parse():
@@ -59,6 +64,7 @@ def parse():
     ap.add_argument("--no-extra", action="store_true", help="skip the per-algorithm extras")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras, no e2e)")
     ap.add_argument("--no-configs", action="store_true", help="skip the other BASELINE configs (per_config)")
+    ap.add_argument("--no-cfg5-multi", action="store_true", help="N > 1: skip the cfg5 BFS/SSSP/CC/SSWP leg")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "node"],
                     help="N > 1: PageRank exchange over NCCL (default) or the node communicator (CUDA IPC + "
                          "shared memory; torch.distributed on gloo; ranks may share a GPU -- for testing)")
@@ -156,19 +162,33 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------------------------------ reference arm
-def cpu_pr_sample(rec, iters, threads_note=True):
-    """The oracle as it stands (single-threaded C power iteration) on the same workload:
-    host generator -> oracle CSR (untimed) -> `iters` PageRank iterations (timed)."""
-    import graphgen
+class pinned_to_one_core:
+    """`taskset -c 0` for the timed oracle call (SURVEY.md §8(d) "Oracle timing"): the calling
+    thread is pinned to one core (core 0 when the process may use it) and restored after."""
+
+    def __enter__(self):
+        self.saved = os.sched_getaffinity(0)
+        self.core = 0 if 0 in self.saved else min(self.saved)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.saved)
+        return False
+
+
+def cpu_pr_sample(src, dst, n, iters):
+    """The oracle as it stands (single-threaded C power iteration) on the same workload: the
+    arc list the GPU used -> oracle CSR (untimed) -> `iters` PageRank iterations (timed, pinned
+    to one core)."""
     import oracle
 
-    src, dst, _ = graphgen.generate(rec, weighted=False)
-    g = oracle.csr_build(rec.n, src, dst)
-    del src, dst
-    t0 = time.perf_counter()
-    oracle.pagerank(g, iters)
-    dt = time.perf_counter() - t0
-    return dt, g
+    g = oracle.csr_build(n, src, dst)
+    with pinned_to_one_core() as pin:
+        t0 = time.perf_counter()
+        oracle.pagerank(g, iters)
+        dt = time.perf_counter() - t0
+    return dt, pin.core
 
 
 def run_reference(args, rank, world):
@@ -183,12 +203,13 @@ def run_reference(args, rank, world):
     g = oracle.csr_build(rec.n, src, dst)
     del src, dst
     times = []
-    for i in range(args.warmup + args.steps):
-        t0 = time.perf_counter()
-        oracle.pagerank(g, 1)  # one power iteration per step: a bounded sample of the 20-iteration run
-        dt = time.perf_counter() - t0
-        if i >= args.warmup:
-            times.append(dt)
+    with pinned_to_one_core() as pin:
+        for i in range(args.warmup + args.steps):
+            t0 = time.perf_counter()
+            oracle.pagerank(g, 1)  # one power iteration per step: a bounded sample of the 20-iteration run
+            dt = time.perf_counter() - t0
+            if i >= args.warmup:
+                times.append(dt)
     t = sum(times) / len(times)
     val = rec.m / t / 1e9
     print(json.dumps({
@@ -198,7 +219,8 @@ def run_reference(args, rank, world):
         "config": config_obj(args, rec),
         "cpu_baseline": {"value": val, "unit": "GTEPS", "cores": 1, "kind": "oracle",
                          "sample": "1 of the 20 PageRank iterations per step on the full cfg4 graph "
-                                   "(oracle/oracle.c or_pagerank, single thread)", "host": host_cpu()},
+                                   f"(oracle/oracle.c or_pagerank, single thread pinned to core {pin.core})",
+                         "host": host_cpu()},
         "e2e": {"value": val, "unit": "GTEPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -233,6 +255,34 @@ def config_obj(args, rec):
 
 
 # ------------------------------------------------------------------------------------------ main arm
+def peak_hbm():
+    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(peaks_path):
+        return json.load(open(peaks_path))["hbm_gbs"], "MEASURED_PEAKS.json hbm_gbs (measured copy)"
+    return 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+
+
+def gather_ceiling():
+    """Measured random 4-byte gather rates (G gathers/s) from tools/micro/gather_ceiling.cu
+    (build/libmicro.so, built by build()): uniform indices into a 2 MB, 64 MB (L2-resident) and
+    1 GB array.  The frontier relax kernels gather one 4-byte target value per processed arc."""
+    import ctypes
+    path = os.path.join(ROOT, "build", "libmicro.so")
+    if not os.path.exists(path):
+        return None
+    lib = ctypes.CDLL(path)
+    lib.micro_gather.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int, ctypes.POINTER(ctypes.c_double)]
+    lib.micro_gather.restype = ctypes.c_int
+    out = {"source": "tools/micro/gather_ceiling.cu: uniform random u32 gathers, 8 in flight per thread, "
+                     "148 x 8 blocks of 256 threads, best of 5"}
+    gathers = 1 << 30
+    for name, nbytes in (("l1_2MB", 2 << 20), ("l2_64MB", 64 << 20), ("hbm_1GB", 1 << 30)):
+        ms = ctypes.c_double()
+        rc = lib.micro_gather(nbytes // 4, gathers, 5, ctypes.byref(ms))
+        out[name + "_ggather_s"] = gathers / (ms.value * 1e-3) / 1e9 if rc == 0 else None
+    return out
+
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
@@ -255,7 +305,7 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
         uid = [tigr.tigr_comm_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
-        comm = tigr.tigr_comm_init(world, rank, uid[0])
+        comm = tigr.tigr_comm_init(world, rank, uid[0], device=local)
     elif world > 1:
         dist.init_process_group("gloo")
         comm = tigr.tigr_comm_init_node(job_name("pr"), world, rank)
@@ -282,21 +332,25 @@ def main():
     opts.time_kernels = 1
     if comm is not None:
         opts.comm = comm.ptr.value
+    cuts = None
+    if comm is not None:  # each rank sorts only the arcs of its source range (arc-balanced cuts)
+        cuts = tigr.tigr_coo_source_cuts(n, src, dst, world, stream=s)
 
-    def one_step(src_t, dst_t, out_t, host=False):
-        """a1 CSR build -> a2-a5 virtualize -> a6-a10 PageRank; returns per-phase events."""
+    def one_step(src_t, dst_t, out_t, run_opts=opts):
+        """a1 CSR build -> a2-a5 virtualize -> a6-a10 PageRank through the C ABI; returns
+        per-phase events.  Host src_t / dst_t / out_t: the library copies the arc list in (in
+        chunks, overlapped with its arc-list scan) and the ranks out, inside the call."""
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)]
         ev[0].record(s)
         if comm is None:
             g = tigr.tigr_graph_from_coo(n, src_t, dst_t, None, stream=s)
-        else:  # e: each rank sorts only the arcs of its source range (arc-balanced cuts)
-            cuts = tigr.tigr_coo_source_cuts(n, src_t, dst_t, world, stream=s)
+        else:
             g = tigr.tigr_graph_from_coo_part(n, src_t, dst_t, None, src_lo=int(cuts[rank]),
                                               src_hi=int(cuts[rank + 1]), stream=s)
         ev[1].record(s)
         vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
         ev[2].record(s)
-        _, st = tigr.tigr_run(vg, "pr", 0, opts=opts, out=out_t, return_stats=True)
+        _, st = tigr.tigr_run(vg, "pr", 0, opts=run_opts, out=out_t, return_stats=True)
         ev[3].record(s)
         vi = vg.info()
         nv = (vi["hi"] - vi["lo"], g.info()["m"])  # this rank's virtual nodes and arcs
@@ -309,12 +363,10 @@ def main():
         one_step(src, dst, out)
     torch.cuda.synchronize()
 
-    deg_t = torch.bincount(src, minlength=n)
-    n_out = int(torch.count_nonzero(deg_t).item())
     clocks = ClockSampler(local, gpu_uuid(torch, local))
     clocks.start()
     l0 = tigr.tigr_launch_count()
-    step_ms, phase, relax_ms, relax_launches, nv = [], [[], [], []], 0.0, 0, 0
+    step_ms, phase, relax_ms, relax_launches, relax_bytes, nv = [], [[], [], []], 0.0, 0, 0, 0
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -327,6 +379,7 @@ def main():
             phase[i].append(ev[i].elapsed_time(ev[i + 1]))
         relax_ms += st["ms_relax"]
         relax_launches += st["relax_launches"]
+        relax_bytes += st["bytes_alg"]
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -336,20 +389,17 @@ def main():
     t_step = allmax(sum(step_ms) / len(step_ms))
     gteps = 20 * m / (t_step * 1e-3) / 1e9
 
-    # roofline of the dominant kernel (PR relax), live CUDA-event durations from the timed region
+    # roofline of the dominant kernel (PR relax): the library's algorithmic bytes of the relax
+    # launches (tigr_stats.bytes_alg) / their live CUDA-event durations in the timed region
     relax_avg_ms = relax_ms / max(relax_launches, 1)
-    my_nv, my_m = nv
-    bytes_launch = relax_bytes_pr(my_m, my_nv, n_out // world if world > 1 else n_out)
-    peaks_path = os.path.join(ROOT, "MEASURED_PEAKS.json")
-    if os.path.exists(peaks_path):
-        peak = json.load(open(peaks_path))["hbm_gbs"]
-        peak_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)"
-    else:
-        peak, peak_src = 6650.0, "fallback 6.65 TB/s (B200_PROFILING.md)"
+    bytes_launch = relax_bytes / max(relax_launches, 1)
+    peak, peak_src = peak_hbm()
     achieved = bytes_launch / (relax_avg_ms * 1e-3) / 1e9
+    # DRAM traffic of one launch from the committed ncu --set full capture: only for the
+    # configuration it was captured on (one GPU, cfg4, K = 8, strided)
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "relax_pr_traffic.json")
-    if os.path.exists(tpath):
+    if world == 1 and args.config == "cfg4" and args.K == 8 and args.layout == "strided" and os.path.exists(tpath):
         traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
 
     if world > torch.cuda.device_count():
@@ -366,39 +416,65 @@ def main():
                      "traffic": traffic,
                      "kernel": "k_relax_pr_cid (PageRank push relax with the apply fused in, pr.cu)",
                      "algorithmic_bytes_per_launch": bytes_launch, "avg_launch_ms": relax_avg_ms,
+                     "byte_model": "tigr_stats.bytes_alg: per arc 20 (target 4 + f64 RED read+write 16), per "
+                                   "virtual node 4, per node with arcs 20 (SURVEY.md §8(d); DESIGN.md §5)",
                      "peak_source": peak_src, "frac_vs_8000_GBps": achieved / 8000.0},
         "breakdown_ms": {"csr_build": statistics.mean(phase[0]), "virtualize": statistics.mean(phase[1]),
                          "pagerank_20it": statistics.mean(phase[2]), "relax_total": relax_ms / args.steps},
         "algo_gteps": 20 * m / (statistics.mean(phase[2]) * 1e-3) / 1e9,
-        "nv": my_nv, "gpu_launches": launches, "clocks": clk,
+        "nv": nv[0], "gpu_launches": launches, "clocks": clk,
+        "paper_context": PAPER_CONTEXT,
     }
     if rec_note:
         result["note"] = rec_note
 
-    # e2e through the public API with HOST buffers (pinned), H2D and D2H inside the timed region
+    # e2e through the C ABI with HOST buffers: every step passes the pinned host arc list to
+    # tigr_graph_from_coo (the library copies it in, chunk by chunk, overlapped with its
+    # arc-list scan) and receives the 20-iteration ranks in a pinned host array from tigr_run
+    # (D2H inside the call); the timed region is the whole call sequence, per step.
     if not args.no_e2e and not args.profile:
         hsrc = src.cpu().pin_memory()
         hdst = dst.cpu().pin_memory()
         hout = torch.empty(n, dtype=torch.float64).pin_memory()
+        e2e_opts = tigr.tigr_run_opts_default()
+        e2e_opts.stream = s.cuda_stream
+        if comm is not None:
+            e2e_opts.comm = comm.ptr.value
         e2e = []
-        for _ in range(max(1, min(args.steps, 5))):
+        for _ in range(max(3, min(args.steps, 5))):
             flush.fill_(1)
             torch.cuda.synchronize()
+            if world > 1:
+                dist.barrier()
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(s)
-            one_step(hsrc, hdst, hout)
+            one_step(hsrc, hdst, hout, e2e_opts)
             e1.record(s)
             torch.cuda.synchronize()
             e2e.append(e0.elapsed_time(e1))
         te = allmax(sum(e2e) / len(e2e))
-        # Pipelined variant: step i+1's arc list is copied in on one copy stream and step i-1's
-        # ranks are read back on another while step i computes -- the same public API on
-        # device buffers, every step's H2D and D2H inside the timed region (first copy to
-        # last readback).
+        result["e2e"] = {"value": 20 * m / (te * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": te,
+                         "steps": len(e2e), "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
+                         "path": "C ABI with host buffers: tigr_graph_from_coo(pinned host src/dst) -> "
+                                 "tigr_virtualize -> tigr_run(out = pinned host array)",
+                         "h2d_bound_ms": None}
+        # the PCIe floor of this step: the H2D of the arc list alone (same pinned buffers)
+        dbuf = torch.empty_like(src)
+        c0, c1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        c0.record(s)
+        dbuf.copy_(hsrc, non_blocking=True)
+        dbuf.copy_(hdst, non_blocking=True)
+        c1.record(s)
+        torch.cuda.synchronize()
+        result["e2e"]["h2d_bound_ms"] = c0.elapsed_time(c1)
+        del dbuf
+        # Pipelined variant (context, not the e2e key): step i+1's arc list is copied in on one
+        # copy stream and step i-1's ranks read back on another while step i computes, with the
+        # device-buffer API calls; every step's H2D and D2H are inside the timed region.
         ksteps = max(2, min(args.steps, 6))
         cs = torch.cuda.Stream()
         rs = torch.cuda.Stream()
-        dbuf = [(torch.empty_like(src), torch.empty_like(dst)) for _ in range(2)]
+        dbufs = [(torch.empty_like(src), torch.empty_like(dst)) for _ in range(2)]
         dres = [torch.empty(n, dtype=torch.float64, device="cuda") for _ in range(2)]
         hres = [torch.empty(n, dtype=torch.float64).pin_memory() for _ in range(2)]
         copied = [torch.cuda.Event() for _ in range(2)]
@@ -417,8 +493,8 @@ def main():
             with torch.cuda.stream(cs):
                 if i >= 2:
                     cs.wait_event(freed[b])
-                dbuf[b][0].copy_(hsrc, non_blocking=True)
-                dbuf[b][1].copy_(hdst, non_blocking=True)
+                dbufs[b][0].copy_(hsrc, non_blocking=True)
+                dbufs[b][1].copy_(hdst, non_blocking=True)
                 copied[b].record(cs)
 
         h2d(0)
@@ -429,7 +505,7 @@ def main():
             s.wait_event(copied[b])
             if i >= 2:
                 s.wait_event(read[b])  # step i-2's ranks have left dres[b]
-            one_step(dbuf[b][0], dbuf[b][1], dres[b])
+            one_step(dbufs[b][0], dbufs[b][1], dres[b], e2e_opts)
             freed[b].record(s)
             with torch.cuda.stream(rs):  # read the ranks back while the next step computes
                 rs.wait_event(freed[b])
@@ -439,31 +515,36 @@ def main():
         p1.record(s)
         torch.cuda.synchronize()
         tp = allmax(p0.elapsed_time(p1) / ksteps)
-        # e2e = the pipelined run (what a user streaming batches gets; every step's H2D and
-        # D2H are inside the timed region); the unpipelined one is reported beside it
-        result["e2e"] = {"value": 20 * m / (tp * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": tp,
-                         "steps": ksteps, "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
-                         "note": "H2D of step i+1 (pinned host arc list) and D2H of step i-1's ranks (to "
-                                 "pinned host memory) on two copy streams, overlapped with step i"}
-        result["e2e_serial"] = {"value": 20 * m / (te * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": te,
-                                "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
-                                "note": "H2D -> step -> D2H with nothing overlapped"}
+        result["e2e_pipelined"] = {"value": 20 * m / (tp * 1e-3) / 1e9, "unit": "GTEPS", "ms_per_step": tp,
+                                   "steps": ksteps, "h2d_bytes_per_step": 2 * m * 4, "d2h_bytes_per_step": n * 8,
+                                   "note": "context, not the e2e key: H2D of step i+1 and D2H of step i-1 on two "
+                                           "torch copy streams, overlapped with step i (device-buffer API calls)"}
+        del dbufs, dres, hres
 
     if not args.no_extra and not args.profile and world == 1:
-        result["per_algo"] = per_algo(tigr, torch, rec, args, s, deg_t.cpu().numpy(), peak)
+        peak_g = gather_ceiling()
+        result["gather_ceiling"] = peak_g
+        result["per_algo"] = per_algo(tigr, torch, rec, args, s, peak, peak_g)
 
     if not args.no_extra and not args.profile and world > 1:
-        result["per_algo_multi"] = per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax)
+        result["per_algo_multi"] = {"cfg4": per_algo_multi(tigr, torch, dist, graphgen.recipe("cfg4"), args, s,
+                                                           rank, world, allmax, comm)}
+        if not args.no_cfg5_multi:
+            result["per_algo_multi"]["cfg5"] = per_algo_multi(tigr, torch, dist, graphgen.recipe("cfg5"), args, s,
+                                                              rank, world, allmax, comm)
 
     if not args.no_extra and not args.no_configs and not args.profile and world == 1:
         result["per_config"] = per_config(tigr, torch, s, peak)
 
     if rank == 0 and world == 1 and not args.no_cpu and not args.profile:
-        dt, _ = cpu_pr_sample(rec, 2)
+        hs = src.cpu().numpy().view(np.uint32)  # the device-drawn arc list the GPU ran on
+        hd = dst.cpu().numpy().view(np.uint32)
+        dt, core = cpu_pr_sample(hs, hd, n, 2)
         v = 2 * m / dt / 1e9
         result["cpu_baseline"] = {"value": v, "unit": "GTEPS", "cores": 1, "kind": "oracle",
-                                  "sample": "2 of the 20 PageRank iterations on the full cfg4 graph "
-                                            f"({dt:.1f} s; oracle/oracle.c or_pagerank, single thread)",
+                                  "sample": "2 of the 20 PageRank iterations on the full cfg4 graph (the device-drawn "
+                                            f"arc list), {dt:.1f} s; oracle/oracle.c or_pagerank, single thread "
+                                            f"pinned to core {core}",
                                   "host": host_cpu()}
     if rank == 0:
         print(json.dumps(result), flush=True)
@@ -487,147 +568,172 @@ def job_name(tag):
     return f"bench_{tag}_{_JOB_TOKEN[0]}"
 
 
-def per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax):
+def frontier_graph(tigr, torch, rec, sym, s):
+    """cfg graph for BFS/SSSP/SSWP (weighted) or CC (symmetrised), drawn on the device, plus the
+    out-degrees of the drawn arc list (input-normalised GTEPS count the arcs of reached nodes)."""
+    src = torch.empty(rec.m, dtype=torch.int32, device="cuda")
+    dst, w = torch.empty_like(src), torch.empty_like(src)
+    tigr.tigr_rmat_coo(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, src, dst, w,
+                       stream=s)
+    deg = torch.bincount(src.long(), minlength=rec.n)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, None if sym else w, symmetrize=sym, stream=s)
+    del src, dst, w
+    torch.cuda.synchronize()
+    return g, deg
+
+
+def input_arcs(algo, out, deg, m):
+    """arcs out of reached nodes (CC: all 2m arcs of the symmetrised graph)."""
+    if algo == "cc":
+        return 2 * m
+    reached = out != (0 if algo == "sswp" else -1)
+    return int(deg[reached].sum().item())
+
+
+def per_algo_multi(tigr, torch, dist, rec, args, s, rank, world, allmax, comm):
+    """N > 1: BFS / SSSP / SSWP / CC on `rec` (cfg4, and BASELINE configs[4] = cfg5) across the
+    ranks.  Every rank holds the whole graph and relaxes its arc-balanced, family-aligned virtual
+    node range (tigr_vgraph_partition); after each relax the replicated values are merged by the
+    communicator: the dense in-place MIN/MAX all-reduce (NCCL ncclAllReduce; BASELINE configs[4]
+    "NCCL min-allreduce"), the sparse exchange of changed nodes, AUTO (per iteration), and --
+    through a node communicator (CUDA IPC) -- the fused exchange.  time = max over ranks of the
+    device time of the run (median of 3); matches_single_gpu_all_ranks: every rank's values equal
+    a one-GPU run of the same graph.  Failures are recorded, not raised, once every rank has
+    reached the same point."""
     import graphgen
-    """N > 1: BFS / SSSP / CC on the scale-24 graph across the ranks with the FUSED exchange
-    (the relax applies each improvement to every peer replica over NVLink; node communicator,
-    CUDA IPC) -- the multi-GPU frontier path.  Every rank holds the whole graph and relaxes its
-    arc-balanced virtual node range; time = max over ranks of the device time of the run;
-    matches_single_gpu: every rank's values equal a one-GPU run of the same graph on its GPU.
-    Failures are recorded, not raised, after every rank has reached the same point."""
+
     n, m = rec.n, rec.m
-    res = {"exchange": "fused", "transport": "node (CUDA IPC + shared memory)"}
-    # probe first, with a short barrier timeout: if shared memory or CUDA IPC is unavailable
-    # here, every rank learns it within seconds and the section is skipped on all of them
-    os.environ["TIGR_GROUP_TIMEOUT"] = "30"
-    comm, err = None, None
-    try:
-        comm = tigr.tigr_comm_init_node(job_name("frontier"), world, rank)
-        small = graphgen.recipe("cfg1")
-        gs = tigr.tigr_graph_rmat(small.n, small.m, small.a, small.b, small.c, small.seed, small.wseed,
-                                  stream=s)
-        vgs = tigr.tigr_virtualize(gs, args.K, args.layout, stream=s)
-        tigr.tigr_vgraph_partition(vgs, world, rank)
-        tigr.tigr_run(vgs, "sssp", 0, comm=comm, exchange="fused", stream=s)
-        tigr.tigr_run(vgs, "sssp", 0, comm=comm, exchange="sparse", stream=s)
-        vgs.free()
-        gs.free()
-    except Exception as e:
-        err = repr(e)
-    if allmax(1.0 if err else 0.0) != 0.0:
-        res["error"] = err or "a peer rank failed the node-communicator probe"
-        return res
-    os.environ["TIGR_GROUP_TIMEOUT"] = "120"
-    for algo in ("bfs", "sssp", "cc"):
+    res = {"config": rec.name, "n": n, "m": m, "partition": "vnode ranges (tigr_vgraph_partition)",
+           "transport": "nccl" if args.transport == "nccl" else "node (CUDA IPC + shared memory)"}
+    # fused needs peer memory: the node communicator (probe first, with a short barrier timeout,
+    # so a box without shared memory / CUDA IPC skips it on every rank within seconds)
+    fcomm = comm if args.transport == "node" else None
+    if fcomm is None:
+        saved = os.environ.get("TIGR_GROUP_TIMEOUT")
+        os.environ["TIGR_GROUP_TIMEOUT"] = "30"
+        err = None
+        try:
+            fcomm = tigr.tigr_comm_init_node(job_name(f"frontier_{rec.name}"), world, rank)
+            small = graphgen.recipe("cfg1")
+            gs = tigr.tigr_graph_rmat(small.n, small.m, small.a, small.b, small.c, small.seed, small.wseed, stream=s)
+            vgs = tigr.tigr_virtualize(gs, args.K, args.layout, stream=s)
+            tigr.tigr_vgraph_partition(vgs, world, rank)
+            tigr.tigr_run(vgs, "sssp", 0, comm=fcomm, exchange="fused", stream=s)
+            vgs.free()
+            gs.free()
+        except Exception as e:  # noqa: BLE001
+            err = repr(e)
+        if allmax(1.0 if err else 0.0) != 0.0:
+            res["fused_error"] = err or "a peer rank failed the node-communicator probe"
+            if fcomm is not None:
+                fcomm.free()
+            fcomm = None
+        if saved is None:
+            os.environ.pop("TIGR_GROUP_TIMEOUT", None)
+        else:
+            os.environ["TIGR_GROUP_TIMEOUT"] = saved
+    modes = [("dense", comm), ("sparse", comm), ("auto", comm)] + ([("fused", fcomm)] if fcomm is not None else [])
+    for algo in ("bfs", "sssp", "sswp", "cc"):
         sym = algo == "cc"
         entry = {}
         try:
-            g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax,
-                                     weighted=not sym, symmetrize=sym, stream=s)
+            g, deg = frontier_graph(tigr, torch, rec, sym, s)
             vg1 = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
             ref = torch.empty(n, dtype=torch.int32, device="cuda")
-            tigr.tigr_run(vg1, algo, 0, out=ref, stream=s)
+            _, st1 = tigr.tigr_run(vg1, algo, rec.source, out=ref, stream=s, return_stats=True)
             vg1.free()
+            entry["ms_single_gpu"] = st1["ms_total"]
+            entry["m_input"] = input_arcs(algo, ref, deg, m)
             vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
             tigr.tigr_vgraph_partition(vg, world, rank)
             out = torch.empty(n, dtype=torch.int32, device="cuda")
-            ts = []
-            for _ in range(3):
-                _, st = tigr.tigr_run(vg, algo, 0, out=out, comm=comm, exchange="fused", stream=s,
-                                      return_stats=True)
-                ts.append(st["ms_total"])
-            torch.cuda.synchronize()
-            entry = {"ms_rank": statistics.median(ts), "iterations": st["iterations"],
-                     "matches_single_gpu": bool(torch.equal(out, ref))}
-            for mode in ("sparse", "dense"):  # the other exchanges, for comparison
-                tm = []
+            ok = True
+            for mode, c in modes:
+                ts = []
                 for _ in range(3):
-                    _, stm = tigr.tigr_run(vg, algo, 0, out=out, comm=comm, exchange=mode, stream=s,
-                                           return_stats=True)
-                    tm.append(stm["ms_total"])
+                    _, st = tigr.tigr_run(vg, algo, rec.source, out=out, comm=c, exchange=mode, stream=s,
+                                          return_stats=True)
+                    ts.append(st["ms_total"])
                 torch.cuda.synchronize()
-                entry[f"ms_rank_{mode}"] = statistics.median(tm)
-                entry["matches_single_gpu"] = entry["matches_single_gpu"] and bool(torch.equal(out, ref))
+                entry[f"ms_rank_{mode}"] = statistics.median(ts)
+                entry[f"iterations_{mode}"] = st["iterations"]
+                ok = ok and bool(torch.equal(out, ref))
+            entry["matches_single_gpu"] = ok
             vg.free()
             g.free()
-        except Exception as e:
+            del deg
+        except Exception as e:  # noqa: BLE001
             entry = {"error": repr(e)}
-        t = allmax(entry.get("ms_rank", float("inf")))
-        for mode in ("sparse", "dense"):
-            if f"ms_rank_{mode}" in entry or "error" in entry:
-                entry[f"ms_{mode}"] = allmax(entry.pop(f"ms_rank_{mode}", float("inf")))
-        ok = allmax(0.0 if entry.get("matches_single_gpu") else 1.0) == 0.0
-        m_arcs = 2 * m if sym else m
-        res[algo] = {"ms": t, "gteps_arcs": m_arcs / (t * 1e-3) / 1e9 if t != float("inf") else None,
-                     "matches_single_gpu_all_ranks": ok, **{k: v for k, v in entry.items() if k != "ms_rank"}}
-    comm.free()
+        row = {"matches_single_gpu_all_ranks": allmax(0.0 if entry.get("matches_single_gpu") else 1.0) == 0.0}
+        m_in = allmax(float(entry.get("m_input", 0)))
+        for mode, _ in modes:
+            t = allmax(entry.get(f"ms_rank_{mode}", float("inf")))
+            row[mode] = {"ms": t, "iterations": entry.get(f"iterations_{mode}"),
+                         "gteps_input": m_in / (t * 1e-3) / 1e9 if t != float("inf") else None}
+        if "ms_single_gpu" in entry:
+            row["ms_single_gpu_rank"] = entry["ms_single_gpu"]
+        if "error" in entry:
+            row["error"] = entry["error"]
+        res[algo] = row
+        torch.cuda.synchronize()
+    if fcomm is not None and fcomm is not comm:
+        fcomm.free()
     return res
 
 
-def frontier_bytes(algo, st, n):
-    """Algorithmic bytes of one frontier run: per processed arc
-    s_e (+4 B weight for SSSP/SSWP) + 4 B target-value read; per successful update 4 B; per
-    active virtual node 4 B; per active node with arcs 12 B (value + row pair); per iteration
-    2 B per node (frontier flags read + cleared)."""
-    s_e = S_E + (4 if algo in ("sssp", "sswp") else 0)
-    return (st["edges_processed"] * (s_e + 4) + st["updates"] * 4 + st["active_vnodes"] * 4
-            + st["active_nodes"] * 12 + st["iterations"] * 2 * n)
-
-
-def per_algo(tigr, torch, rec, args, s, deg, peak):
-    """Algorithm-only GTEPS for BFS/SSSP/CC/SSWP on the same scale-24 graph (weights 1-64;
-    CC on the symmetrised graph), device-timed, on the in-degree-reordered graph
-    (tigr_graph_reorder; its one-off cost is reported as reorder_ms, like the virtual split's
-    transform time) and, for comparison, in canonical numbering (ms_canonical).
-    gteps_input = arcs out of reached vertices (CC: all 2m arcs) / time; gteps_processed =
-    arcs of active virtual nodes (collect_stats) / time; roofline_frac = algorithmic bytes /
-    relax-kernel time (CUDA events per relax launch) / measured HBM peak."""
+def per_algo(tigr, torch, rec, args, s, peak, gceil):
+    """Algorithm-only GTEPS for BFS/SSSP/SSWP/CC on the same scale-24 graph (weights 1-64; CC on
+    the symmetrised graph), device-timed, in canonical numbering (the main numbers) and, beside
+    them, on the in-degree-reordered copy (tigr_graph_reorder; its one-off cost is reorder_ms).
+    gteps_input = arcs out of reached vertices (CC: all 2m arcs) / time; gteps_processed = arcs
+    of active virtual nodes (collect_stats) / time; roofline_frac = the library's algorithmic
+    bytes (tigr_stats.bytes_alg) / relax-kernel time (CUDA events per relax
+    launch) / measured HBM peak; gather_frac_l2 = processed arcs per second of relax time / the
+    measured L2 random-gather ceiling (each processed arc gathers one 4-byte target value)."""
     res = {}
     n, m = rec.n, rec.m
-    g = vg = None
-    for algo in ("bfs", "sssp", "sswp", "cc"):
-        sym = algo == "cc"
-        if g is None or sym:
-            if g is not None:
-                vg.free(); g.free(); vgc.free(); gc.free()
-            gc = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax,
-                                      weighted=not sym, symmetrize=sym, stream=s)
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(s)
-            g = tigr.tigr_graph_reorder(gc, stream=s)
-            e1.record(s)
-            torch.cuda.synchronize()
-            reorder_ms = e0.elapsed_time(e1)
-            vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
-            vgc = tigr.tigr_virtualize(gc, args.K, args.layout, stream=s)
+    ceil_l2 = (gceil or {}).get("l2_64MB_ggather_s")
+
+    def measure(vg, algo, deg):
         out = torch.empty(n, dtype=torch.int32, device="cuda")
         _, st = tigr.tigr_run(vg, algo, 0, out=out, stream=s, collect_stats=1, return_stats=True)
-        times, canon, relax = [], [], []
+        times, relax = [], []
         for _ in range(3):
             _, st2 = tigr.tigr_run(vg, algo, 0, out=out, stream=s, return_stats=True)
             times.append(st2["ms_total"])
-            _, st3 = tigr.tigr_run(vgc, algo, 0, out=out, stream=s, return_stats=True)
-            canon.append(st3["ms_total"])
             _, st4 = tigr.tigr_run(vg, algo, 0, out=out, stream=s, return_stats=True, time_kernels=1)
             relax.append(st4["ms_relax"])
-        t = statistics.median(times)
-        t_relax = statistics.median(relax)
-        if algo == "cc":
-            m_in = 2 * m
-        else:
-            reached = out.cpu().numpy().view(np.uint32)
-            mask = reached != (0 if algo == "sswp" else 0xFFFFFFFF)
-            m_in = int(deg[mask].sum())
-        nbytes = frontier_bytes(algo, st, n)
-        res[algo] = {"ms": t, "ms_relax": t_relax, "ms_canonical": statistics.median(canon), "reorder_ms": reorder_ms,
-                     "iterations": st["iterations"], "queue_iterations": st["queue_iterations"],
-                     "gteps_input": m_in / (t * 1e-3) / 1e9,
-                     "gteps_processed": st["edges_processed"] / (t * 1e-3) / 1e9,
-                     "edges_processed": st["edges_processed"], "updates": st["updates"],
-                     "algorithmic_bytes": nbytes,
-                     "roofline_frac": nbytes / (t_relax * 1e-3) / 1e9 / peak,
-                     "roofline_frac_whole_run": nbytes / (t * 1e-3) / 1e9 / peak}
-    vg.free(); g.free(); vgc.free(); gc.free()
+        t, t_relax = statistics.median(times), statistics.median(relax)
+        m_in = input_arcs(algo, out, deg, m)
+        r = {"ms": t, "ms_relax": t_relax, "iterations": st["iterations"],
+             "queue_iterations": st["queue_iterations"], "gteps_input": m_in / (t * 1e-3) / 1e9,
+             "gteps_processed": st["edges_processed"] / (t * 1e-3) / 1e9,
+             "edges_processed": st["edges_processed"], "updates": st["updates"],
+             "algorithmic_bytes": st["bytes_alg"],
+             "roofline_frac": st["bytes_alg"] / (t_relax * 1e-3) / 1e9 / peak,
+             "roofline_frac_whole_run": st["bytes_alg"] / (t * 1e-3) / 1e9 / peak}
+        if ceil_l2:
+            r["gather_frac_l2"] = st["edges_processed"] / (t_relax * 1e-3) / 1e9 / ceil_l2
+        return r
+
+    for algo in ("bfs", "sssp", "sswp", "cc"):
+        sym = algo == "cc"
+        gc, deg = frontier_graph(tigr, torch, rec, sym, s)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        gr = tigr.tigr_graph_reorder(gc, stream=s)
+        e1.record(s)
+        torch.cuda.synchronize()
+        vgc = tigr.tigr_virtualize(gc, args.K, args.layout, stream=s)
+        vgr = tigr.tigr_virtualize(gr, args.K, args.layout, stream=s)
+        res[algo] = measure(vgc, algo, deg)
+        res[algo]["reordered"] = measure(vgr, algo, deg)
+        res[algo]["reordered"]["reorder_ms"] = e0.elapsed_time(e1)
+        vgc.free()
+        vgr.free()
+        gc.free()
+        gr.free()
+        del deg
     # NEXT-1: pull PageRank on the in-CSR (same graph, 20 iterations), relax timed per launch
     g = tigr.tigr_graph_rmat(n, m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, stream=s)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -711,7 +817,7 @@ def per_config(tigr, torch, s, peak):
             else:
                 reached = out != (0 if algo == "sswp" else -1)
                 m_in = int(deg[reached].sum().item())
-            nbytes = frontier_bytes(algo, st, n)
+            nbytes = st["bytes_alg"]  # the library's byte model (collect_stats run)
             entry[f"{algo}_K{K}"] = {
                 "ms": t, "ms_relax": st3["ms_relax"], "iterations": st["iterations"],
                 "gteps_input": m_in / (t * 1e-3) / 1e9,

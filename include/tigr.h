@@ -115,6 +115,9 @@ typedef struct {
     tigr_comm* comm;      /* NULL = single GPU; else this rank's communicator (see tigr_vgraph_partition) */
     void* stream;         /* cudaStream_t */
     int exchange;         /* tigr_exchange (multi-GPU frontier algorithms; default AUTO) */
+    uint32_t frontier_div;/* FRONTIER_AUTO switch point D: an iteration runs from the queue while its
+                             active nodes own fewer than 1/D of this rank's virtual nodes, else the
+                             dense sweep (0 = default 2) */
 } tigr_run_opts;
 
 typedef struct {
@@ -129,6 +132,10 @@ typedef struct {
     uint32_t queue_iterations;/* iterations whose relax ran from the active-node queue (FRONTIER_AUTO/QUEUE) */
     uint32_t sparse_exchanges;/* multi-GPU: iterations merged by the sparse (changed-node list) exchange */
     uint64_t active_nodes;    /* sum over iterations of active nodes that own virtual nodes (FRONTIER_AUTO/QUEUE) */
+    double ms_kernels;        /* device time of the run outside the multi-GPU exchanges (ms_total - ms_exchange) */
+    uint64_t bytes_alg;       /* algorithmic bytes of the relax launches by the SURVEY.md §8(d) byte model
+                                 (DESIGN.md §5): PR always; BFS/SSSP/CC/SSWP only with collect_stats
+                                 (it needs the processed-arc counts), else 0 */
 } tigr_stats;
 
 /* Fill *opts with the defaults above. */
@@ -138,7 +145,9 @@ void tigr_run_opts_default(tigr_run_opts* opts);
 
 /* Build a device CSR from an arc list (src[e] -> dst[e], weight w[e]); w may be NULL
  * (unweighted graph).  Arcs are grouped by source (Fig. 10a); duplicates
- * and self-loops are kept; the order of arcs within a source is unspecified.
+ * and self-loops are kept; the build is STABLE: the arcs of a source keep their input order
+ * (arc e before arc f iff e < f), so the device CSR is the canonical one (a stable counting sort
+ * by source) and tigr_graph_export_coo returns the arcs in that order.
  * symmetrize=1 appends (dst[e] -> src[e], w[e]) for every arc (weak connectivity, CC).
  * Errors: EINVAL (an id >= n, n == 0), ERANGE (n > 0xFFFFFFFE or too many arcs). */
 tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
@@ -284,9 +293,11 @@ tigr_status tigr_run(tigr_vgraph* vg, tigr_algo algo, uint32_t source, const tig
 /* ------------------------------------------------------------- multi-GPU ---- */
 
 /* NCCL bootstrap: rank 0 creates the 128-byte id and broadcasts it (e.g. over
- * torch.distributed); every rank then calls tigr_comm_init on its own device. */
+ * torch.distributed); every rank then calls tigr_comm_init for its own GPU: `device` is the
+ * CUDA device ordinal the rank runs on (it becomes the calling thread's current device), or
+ * -1 for the current device.  Errors: EINVAL (bad rank / nranks / device), ENCCL. */
 tigr_status tigr_comm_unique_id(uint8_t id[128]);
-tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
+tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], int device, tigr_comm** out);
 void tigr_comm_free(tigr_comm* comm);
 
 /* Thread-group communicator: nranks ranks that are threads of ONE process, each on its own

@@ -49,7 +49,8 @@ class tigr_run_opts(ctypes.Structure):
     _fields_ = [("max_iters", ctypes.c_uint32), ("pr_iters", ctypes.c_uint32), ("pr_damping", ctypes.c_double),
                 ("pr_dangling", ctypes.c_int), ("schedule", ctypes.c_int), ("frontier", ctypes.c_int),
                 ("use_graph", ctypes.c_int), ("collect_stats", ctypes.c_int), ("time_kernels", ctypes.c_int),
-                ("comm", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("exchange", ctypes.c_int)]
+                ("comm", ctypes.c_void_p), ("stream", ctypes.c_void_p), ("exchange", ctypes.c_int),
+                ("frontier_div", ctypes.c_uint32)]
 
 
 class tigr_stats(ctypes.Structure):
@@ -57,7 +58,7 @@ class tigr_stats(ctypes.Structure):
                 ("edges_processed", ctypes.c_uint64), ("updates", ctypes.c_uint64),
                 ("active_vnodes", ctypes.c_uint64), ("ms_total", ctypes.c_double), ("ms_relax", ctypes.c_double),
                 ("ms_exchange", ctypes.c_double), ("queue_iterations", ctypes.c_uint32), ("sparse_exchanges", ctypes.c_uint32),
-                ("active_nodes", ctypes.c_uint64)]
+                ("active_nodes", ctypes.c_uint64), ("ms_kernels", ctypes.c_double), ("bytes_alg", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -91,7 +92,7 @@ _SIGS = {
     "tigr_vgraph_free": (None, [_P]),
     "tigr_run": (_I, [_P, _I, _U32, ctypes.POINTER(tigr_run_opts), _P, _I, ctypes.POINTER(tigr_stats)]),
     "tigr_comm_unique_id": (_I, [_P]),
-    "tigr_comm_init": (_I, [_I, _I, _P, ctypes.POINTER(_P)]),
+    "tigr_comm_init": (_I, [_I, _I, _P, _I, ctypes.POINTER(_P)]),
     "tigr_comm_free": (None, [_P]),
     "tigr_comm_group_create": (_I, [_I, ctypes.POINTER(_P)]),
     "tigr_comm_init_group": (_I, [_P, _I, ctypes.POINTER(_P)]),
@@ -442,10 +443,11 @@ def tigr_comm_unique_id() -> bytes:
     return bytes(buf)
 
 
-def tigr_comm_init(nranks: int, rank: int, uid: bytes) -> Comm:
+def tigr_comm_init(nranks: int, rank: int, uid: bytes, device: int = -1) -> Comm:
+    """NCCL communicator of `rank` on CUDA device `device` (-1: the current device)."""
     buf = (ctypes.c_uint8 * 128).from_buffer_copy(uid)
     out = _P()
-    _check(_lib.tigr_comm_init(nranks, rank, buf, ctypes.byref(out)))
+    _check(_lib.tigr_comm_init(nranks, rank, buf, device, ctypes.byref(out)))
     return Comm(out.value, nranks, rank)
 
 

@@ -38,6 +38,16 @@ void trace(cudaStream_t s, const char* what) {
     last = now;
 }
 
+int dev_knob(const char* name, int dflt) {
+#ifdef TIGR_DEV_KNOBS
+    const char* e = getenv(name);
+    return e ? atoi(e) : dflt;
+#else
+    (void)name;
+    return dflt;
+#endif
+}
+
 tigr_status fail(tigr_status st, const std::string& msg) {
     t_err = msg;
     return st;
@@ -183,7 +193,7 @@ tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, c
                                   const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out);
 tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
                                        const uint32_t* w, int symmetrize, uint32_t src_lo, uint32_t src_hi,
-                                       cudaStream_t s, tigr_graph** out);
+                                       cudaStream_t s, tigr_graph** out, const HostArcs* host);
 tigr_status coo_source_cuts(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, int symmetrize,
                             int nranks, cudaStream_t s, uint32_t* cuts);
 tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col, const uint32_t* w,
@@ -204,7 +214,7 @@ tigr_status assignment_device(const tigr_vgraph* vg, uint32_t* counts, uint32_t*
 tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank);
 void partition_ranges(uint32_t n, const int64_t* rp, const uint32_t* vp, int nranks, uint32_t* lo, uint32_t* hi);
 tigr_status comm_unique_id(uint8_t id[128]);
-tigr_status comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out);
+tigr_status comm_init(int nranks, int rank, const uint8_t id[128], int device, tigr_comm** out);
 void comm_free(tigr_comm* c);
 tigr_status comm_group_create(int nranks, tigr_comm_group** out);
 tigr_status comm_init_node(const char* name, int nranks, int rank, tigr_comm** out);
@@ -252,6 +262,29 @@ void tigr_run_opts_default(tigr_run_opts* o) {
     o->exchange = TIGR_EXCHANGE_AUTO;
 }
 
+}  // extern "C"
+
+namespace tigr {
+namespace {
+// the arc-list builds: device arrays are used in place; host arrays get device buffers that the
+// build fills chunk by chunk, overlapping the PCIe copies with its arc-list scan (sort.cu)
+tigr_status coo_build(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
+                      int is_device_ptr, int symmetrize, uint32_t lo, uint32_t hi, cudaStream_t s, tigr_graph** out) {
+    if (is_device_ptr || m == 0)
+        return graph_from_coo_part_device(n, m, src, dst, w, symmetrize, lo, hi, s, out, nullptr);
+    TmpBuf ts, td, tw;
+    TIGR_TRY(ts.alloc(sizeof(uint32_t) * m, s));
+    TIGR_TRY(td.alloc(sizeof(uint32_t) * m, s));
+    if (w) TIGR_TRY(tw.alloc(sizeof(uint32_t) * m, s));
+    const HostArcs host{src, dst, w};
+    return graph_from_coo_part_device(n, m, ts.as<uint32_t>(), td.as<uint32_t>(), w ? tw.as<uint32_t>() : nullptr,
+                                      symmetrize, lo, hi, s, out, &host);
+}
+}  // namespace
+}  // namespace tigr
+
+extern "C" {
+
 tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
                                 int is_device_ptr, int symmetrize, void* stream, tigr_graph** out) {
     if (!out) return fail(TIGR_EINVAL, "graph_from_coo: out is NULL");
@@ -261,13 +294,7 @@ tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, con
     if (m && (!src || !dst)) return fail(TIGR_EINVAL, "graph_from_coo: src/dst NULL");
     TIGR_TRY(need_device());
     cudaStream_t s = (cudaStream_t)stream;
-    TmpBuf ts, td, tw;
-    const uint32_t *ds = nullptr, *dd = nullptr, *dw = nullptr;
-    TIGR_TRY(stage(src, m, is_device_ptr, s, ts, &ds));
-    TIGR_TRY(stage(dst, m, is_device_ptr, s, td, &dd));
-    TIGR_TRY(stage(w, m, is_device_ptr, s, tw, &dw));
-    trace(s, "coo: stage");
-    TIGR_TRY(graph_from_coo_device(n, m, ds, dd, dw, symmetrize, s, out));
+    TIGR_TRY(coo_build(n, m, src, dst, w, is_device_ptr, symmetrize, 0, 0xFFFFFFFFu, s, out));
     TIGR_CK(cudaStreamSynchronize(s));
     trace(s, "coo: done");
     return TIGR_OK;
@@ -284,12 +311,7 @@ tigr_status tigr_graph_from_coo_part(uint32_t n, uint64_t m, const uint32_t* src
     if (src_lo > src_hi) return fail(TIGR_EINVAL, "graph_from_coo_part: src_lo > src_hi");
     TIGR_TRY(need_device());
     cudaStream_t s = (cudaStream_t)stream;
-    TmpBuf ts, td, tw;
-    const uint32_t *ds = nullptr, *dd = nullptr, *dw = nullptr;
-    TIGR_TRY(stage(src, m, is_device_ptr, s, ts, &ds));
-    TIGR_TRY(stage(dst, m, is_device_ptr, s, td, &dd));
-    TIGR_TRY(stage(w, m, is_device_ptr, s, tw, &dw));
-    TIGR_TRY(graph_from_coo_part_device(n, m, ds, dd, dw, symmetrize, src_lo, src_hi, s, out));
+    TIGR_TRY(coo_build(n, m, src, dst, w, is_device_ptr, symmetrize, src_lo, src_hi, s, out));
     TIGR_CK(cudaStreamSynchronize(s));
     return TIGR_OK;
 }
@@ -521,10 +543,11 @@ tigr_status tigr_comm_unique_id(uint8_t id[128]) {
     return comm_unique_id(id);
 }
 
-tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out) {
+tigr_status tigr_comm_init(int nranks, int rank, const uint8_t id[128], int device, tigr_comm** out) {
     if (!id || !out) return fail(TIGR_EINVAL, "comm_init: NULL");
     *out = nullptr;
-    return comm_init(nranks, rank, id, out);
+    TIGR_TRY(need_device());
+    return comm_init(nranks, rank, id, device, out);
 }
 
 void tigr_comm_free(tigr_comm* c) { comm_free(c); }

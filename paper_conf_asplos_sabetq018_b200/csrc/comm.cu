@@ -293,8 +293,16 @@ tigr_status comm_unique_id(uint8_t id[128]) {
     return TIGR_OK;
 }
 
-tigr_status comm_init(int nranks, int rank, const uint8_t id[128], tigr_comm** out) {
+tigr_status comm_init(int nranks, int rank, const uint8_t id[128], int device, tigr_comm** out) {
     if (nranks < 1 || rank < 0 || rank >= nranks) return fail(TIGR_EINVAL, "comm_init: bad rank/nranks");
+    if (device >= 0) {
+        int count = 0;
+        TIGR_CK(cudaGetDeviceCount(&count));
+        if (device >= count) return fail(TIGR_EINVAL, "comm_init: device ordinal out of range");
+        TIGR_CK(cudaSetDevice(device));
+    } else if (device != -1) {
+        return fail(TIGR_EINVAL, "comm_init: device must be >= 0 or -1 (current)");
+    }
     TIGR_TRY(nccl_ready());
     ncclUniqueId u;
     memcpy(&u, id, 128);

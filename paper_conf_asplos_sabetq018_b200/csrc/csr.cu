@@ -20,7 +20,8 @@ tigr_status rmat_range(uint32_t n, uint64_t e0, uint64_t count, double a, double
                        uint64_t seed, uint64_t wseed, uint32_t wmin, uint32_t wmax, uint32_t* src,
                        uint32_t* dst, uint32_t* w, cudaStream_t s);
 tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
-                             int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi);
+                             int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi,
+                             const HostArcs* host);
 
 namespace {
 
@@ -286,9 +287,11 @@ tigr_status expand_arcs(const tigr_graph* g, uint32_t* src, uint32_t* dst, uint3
 
 // src_lo/src_hi: keep only the arcs whose source lies in [src_lo, src_hi) (multi-GPU partitioned
 // builds); the in-degree sketch and the id validation still cover every arc
+// host (nullable): src / dst / w are device buffers still to be filled from these host arrays
+// (the build copies them in chunks, overlapped with its arc-list scan)
 tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
                                        const uint32_t* w, int symmetrize, uint32_t src_lo, uint32_t src_hi,
-                                       cudaStream_t s, tigr_graph** out) {
+                                       cudaStream_t s, tigr_graph** out, const HostArcs* host) {
     const uint64_t arcs = symmetrize ? 2 * m : m;
     if (arcs >= (1ull << 32) * 3) return fail(TIGR_ERANGE, "graph: too many arcs");
     tigr_graph* g = new tigr_graph();
@@ -296,7 +299,7 @@ tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* s
     g->m = arcs;
     g->weighted = w != nullptr;
     g->symmetric = symmetrize != 0;
-    tigr_status st = csr_build_sorted(n, m, src, dst, w, symmetrize, s, g, src_lo, src_hi);
+    tigr_status st = csr_build_sorted(n, m, src, dst, w, symmetrize, s, g, src_lo, src_hi, host);
     g->part_lo = src_lo;
     g->part_hi = src_hi < n ? src_hi : n;
     if (st == TIGR_OK) {
@@ -313,7 +316,7 @@ tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* s
 
 tigr_status graph_from_coo_device(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
                                   const uint32_t* w, int symmetrize, cudaStream_t s, tigr_graph** out) {
-    return graph_from_coo_part_device(n, m, src, dst, w, symmetrize, 0, 0xFFFFFFFFu, s, out);
+    return graph_from_coo_part_device(n, m, src, dst, w, symmetrize, 0, 0xFFFFFFFFu, s, out, nullptr);
 }
 
 tigr_status graph_from_csr_device(uint32_t n, uint64_t m, const int64_t* rp, const uint32_t* col,

@@ -44,6 +44,18 @@
 // CC uses the same bitmap for one exact case: a label lowered to 0, the smallest id, is
 // final (nothing is better than 0), and on power-law graphs the giant component -- most
 // targets -- carries label 0 after the first iterations.
+// SSSP and SSWP settle by the frontier bound.  At the start of iteration it, every value that
+// has not yet been pushed along all its arcs belongs to a node stamped active for it (the
+// frontier rule: an atomic that may have improved a node stamps it for the next iteration, and
+// a node whose virtual nodes read an older value was stamped again when it was lowered).  So
+// every candidate of iteration it and later derives from the current values of the active
+// nodes: SSSP candidates are >= mu + w >= mu, mu = the minimum over the active nodes (weights
+// >= 0; UDT's dumb arcs weigh 0), and SSWP candidates min(x, w) are <= M, the maximum over them.
+// A value below mu (SSSP) or at least M (SSWP) can never improve again: final.  k_compact
+// computes the bound while it builds the queue, and after iteration it sets the bit of every
+// node beyond iteration it's bound (frontier.cu); the relax only tests bits.  (Setting bits from
+// the relax's own gathers was measured slower: the L1 keeps serving a stale zero word, so every
+// SM re-issued the atomicOr for the same hot targets.)  Bits persist (a final value stays final).
 //
 // This header holds the relax kernel template; frontier_{bfs,sssp,sswp,cc}.cu instantiate it
 // for one algorithm each (parallel compilation), frontier.cu holds the queue build and the
@@ -117,14 +129,27 @@ __device__ __forceinline__ void map_round(const uint32_t* __restrict__ qv, const
 // applied, in the same branch, to every peer's replica with the relax's own atomic (over
 // NVLink when the peer is another GPU) and activates the node there too -- the peers see it
 // like an update from one more SM.  Only improvements travel: bytes ~ updates x (P-1) x 8.
+// Scope: a replica word receives atomics from its owner GPU and from every peer GPU at once, so
+// with peers every atomic on a replica -- the owner's own included (apply8) -- is system-scope
+// (atom.sys): only atomics whose scopes include each other are atomic with respect to each other
+// in the PTX memory model, and a gpu-scope atomic does not include another GPU's threads.  The
+// stamp stores and the plain value gathers are ordered by the end-of-iteration barrier (kernel
+// completion, stream sync, host barrier); a gather that misses a concurrent peer update reads a
+// stale larger (smaller, SSWP) value, which only costs an atomic that cannot lower it -- the same
+// benign staleness as between the SMs of one GPU.
+template <int A>
+__device__ __forceinline__ void atomic_better_sys(uint32_t* p, uint32_t alt) {
+    if (A == TIGR_SSWP) atomicMax_system(p, alt);
+    else atomicMin_system(p, alt);
+}
+
 template <int A>
 __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, uint32_t n, uint32_t it, uint32_t v,
                                            uint32_t alt) {
     const uint64_t slot = (uint64_t)((it + 1) & 1u) * n;
     for (int r = 0; r < pp->P; ++r) {
         if (r == pp->me) continue;
-        if (A == TIGR_SSWP) atomicMax(pp->val[r] + v, alt);
-        else atomicMin(pp->val[r] + v, alt);
+        atomic_better_sys<A>(pp->val[r] + v, alt);
         pp->stamp[r][slot + v] = it + 1;
     }
 }
@@ -133,7 +158,9 @@ __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, ui
 template <int A, int LAYOUT, bool BSP, int B, bool STATS, int MINB, bool PRE>
 __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
-    const bool BITS = (A == TIGR_BFS || A == TIGR_CC) && f.settled != nullptr;  // uniform per launch
+    constexpr uint32_t kFinal = A == TIGR_SSWP ? kInf : 0u;  // a settled target reads as unimprovable
+    const bool BITS = f.settled != nullptr;    // uniform per launch
+    if (!a.ctl->cont) return;  // an iteration enqueued past the fixed point (batched host loop, run.cu)
     const int lane = threadIdx.x & 31;
     const uint32_t it = a.ctl->it;
     const unsigned long long qp = a.ctl->qpack[it & 1u];
@@ -220,20 +247,20 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             kn[r] = k + 2 * step[r];
             if (STATS && act[r]) ++n_vn;
         }
-        // BFS with a settled bitmap (f.settled): the test reads one bit of a 2 MB array instead
-        // of the 4-byte level (see k_relax_fq's header); cur[q] = 1 means "settled, skip"
+        // settled bitmap (f.settled): the test reads one bit of an n/8-byte array instead of the
+        // 4-byte value (see the header); a settled target reads as kFinal (never improvable)
         auto gather8 = [&](const uint32_t* nb, uint32_t* cur) {
-            if (BITS) {  // settled targets read as level 0 (never improved); the rest read the level
+            if (BITS) {
                 uint32_t b[8];
 #pragma unroll
                 for (int q = 0; q < 8; ++q)
                     b[q] = (nb[q] == kPad) ? 1u : (f.settled[nb[q] >> 5] >> (nb[q] & 31u)) & 1u;
 #pragma unroll
-                for (int q = 0; q < 8; ++q) cur[q] = b[q] ? 0u : a.val[nb[q]];
+                for (int q = 0; q < 8; ++q) cur[q] = b[q] ? kFinal : a.val[nb[q]];
                 return;
             }
 #pragma unroll
-            for (int q = 0; q < 8; ++q) cur[q] = (nb[q] == kPad) ? 0u : a.val[nb[q]];
+            for (int q = 0; q < 8; ++q) cur[q] = (nb[q] == kPad) ? kFinal : a.val[nb[q]];
         };
         auto apply8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv, const uint32_t* cur) {
 #pragma unroll
@@ -242,11 +269,16 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                 if (STATS) ++n_edges;
                 const uint32_t alt = combine<A>(xv, W ? ww[q] : 0u);
                 if (better<A>(alt, cur[q])) {
-                    if (A == TIGR_SSWP) atomicMax(a.val + nb[q], alt);
-                    else atomicMin(a.val + nb[q], alt);
-                    if (f.peers) push_peers<A>(f.peers, a.n, it, nb[q], alt);
-                    // the level becomes alt = it, final (see the header): mark it settled
-                    if (BITS && (A == TIGR_BFS || alt == 0u))  // CC: only label 0 is final
+                    if (f.peers) {  // fused exchange: system-scope on every replica (push_peers)
+                        atomic_better_sys<A>(a.val + nb[q], alt);
+                        push_peers<A>(f.peers, a.n, it, nb[q], alt);
+                    } else if (A == TIGR_SSWP) {
+                        atomicMax(a.val + nb[q], alt);
+                    } else {
+                        atomicMin(a.val + nb[q], alt);
+                    }
+                    // BFS: the level becomes alt = it, final (see the header); CC: label 0 is final
+                    if (BITS && (A == TIGR_BFS || (A == TIGR_CC && alt == 0u)))
                         atomicOr(f.settled + (nb[q] >> 5), 1u << (nb[q] & 31u));
                     stamp_next[nb[q]] = it + 1;
                     touched = true;
@@ -332,13 +364,13 @@ FqFn pick_fq(bool bsp, bool stats) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     constexpr int B = W ? 2 : 4;
     constexpr bool PRE = W;
-    if (!bsp && !stats) {  // development knob: alternative shapes (TIGR_FQ_SHAPE)
-        const char* e = getenv("TIGR_FQ_SHAPE");
+    if (!bsp && !stats) {  // TIGR_FQ_SHAPE: alternative shapes in development builds
+
         // BFS and CC with their settled bitmap are latency-bound rather than L1/L2-bound
         // (profiles/README.md): 2 virtual nodes per thread with all gathers issued first,
         // 4 blocks/SM (64 registers, no spills); cfg4 BFS 1.47 -> 1.34 ms, CC 3.44 -> 3.07 ms
         const int dflt = (A == TIGR_BFS || A == TIGR_CC) ? 1 : 0;
-        switch (e ? atoi(e) : dflt) {
+        switch (dev_knob("TIGR_FQ_SHAPE", dflt)) {
             case 1: return &k_relax_fq<A, LAYOUT, false, 2, false, 4, true>;
             default: break;
         }

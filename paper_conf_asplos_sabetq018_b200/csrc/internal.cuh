@@ -48,6 +48,11 @@ inline void count_launch(uint64_t k = 1) { g_launches.fetch_add(k, std::memory_o
 // the stream and prints the host wall time since the previous trace point (stderr).
 void trace(cudaStream_t s, const char* what);
 
+// Development knobs for A/B sweeps (tools/dev/): read from the environment only when the
+// library is built with -DTIGR_DEV_KNOBS (TIGR_DEV_KNOBS=1 python tools/native_build.py); the
+// shipped build always takes the default, so no environment variable changes a kernel.
+int dev_knob(const char* name, int dflt);
+
 inline unsigned grid_for(uint64_t items, int block = kBlock) {
     uint64_t g = (items + block - 1) / block;
     return (unsigned)(g ? g : 1);
@@ -76,6 +81,14 @@ struct TmpBuf {  // cudaMallocAsync / cudaFreeAsync on a stream
     tigr_status alloc(size_t nbytes, cudaStream_t stream);
     ~TmpBuf();
     template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// Host arrays of an arc list (tigr_graph_from_coo with host pointers): the CSR build copies them
+// to its device buffers chunk by chunk, overlapped with the arc-list scan (sort.cu).
+struct HostArcs {
+    const uint32_t* src;
+    const uint32_t* dst;
+    const uint32_t* w;
 };
 
 // ---- scan (scan.cu) ----------------------------------------------------------------------

@@ -219,11 +219,6 @@ unsigned grid_cap(uint64_t items, int per_sm) {
 
 }  // namespace
 
-bool pr_cid_enabled() {
-    const char* e = getenv("TIGR_PR_VARIANT");
-    return !e || atoi(e) == 13;
-}
-
 // once per vgraph: cid order, n_in, col_pr (workspace), all on the device
 tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
     Workspace& ws = vg->ws;
@@ -333,11 +328,10 @@ static void fill_plan(PrCidPlan& p, int layout) {
 // memory: one table per SM instead of two 8192-slot copies), 4 virtual nodes per thread.
 // Measured at cfg4 (relax ms/launch): 256x2 blocks, 8192 slots 1.53; 512x1, 24576 1.15;
 // 768x1, 24576 1.12; 768x1, 28672 1.21; 1024x1 (spills) 1.16.  TIGR_PR_CFG selects the
-// alternatives for experiments.
+// alternatives in development builds (dev_knob).
 PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
     PrCidPlan p;
-    const char* e = getenv("TIGR_PR_CFG");
-    switch (e ? atoi(e) : 5) {
+    switch (dev_knob("TIGR_PR_CFG", 5)) {
         case 0: fill_plan<4, 256, 8192, 2>(p, vg->layout); break;
         case 1: fill_plan<4, 512, 24576, 1>(p, vg->layout); break;
         case 6: fill_plan<4, 768, 28672, 1>(p, vg->layout); break;

@@ -80,6 +80,7 @@ __device__ __forceinline__ void walk(const uint32_t* __restrict__ col, const uin
 template <int A, int LAYOUT, bool VEC, int FRONT, bool BSP, bool STATS>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    if (!a.ctl->cont) return;  // an iteration enqueued past the fixed point (batched host loop, run.cu)
     const uint64_t i = (uint64_t)a.lo + (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
     const uint32_t it = (FRONT == TIGR_FRONTIER_DENSE) ? a.ctl->it : 0;
     bool touched = false;
@@ -145,6 +146,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
 template <int A, int LAYOUT, int FRONT, bool BSP, int B>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    if (!a.ctl->cont) return;  // past the fixed point (batched host loop)
     const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * kRelaxThreads) + threadIdx.x;
     const uint32_t it = (FRONT == TIGR_FRONTIER_DENSE) ? a.ctl->it : 0;
     const uint32_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;   // not written in this launch
@@ -252,16 +254,9 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
     if (__any_sync(0xffffffffu, touched) && (threadIdx.x & 31) == 0) a.ctl->changed = 1;
 }
 
-int fr_variant() {
-    const char* e = getenv("TIGR_FR_VARIANT");
-    return e ? atoi(e) : 2;
-}
-
 template <int A, int LAYOUT>
 static RelaxFn pick_mlp(int front, bool bsp, int B) {
 #define TIGR_MLP(F, BS, BB) if (front == F && bsp == BS && B == BB) return &k_relax_mlp<A, LAYOUT, F, BS, BB>;
-    TIGR_MLP(TIGR_FRONTIER_DENSE, false, 2) TIGR_MLP(TIGR_FRONTIER_DENSE, true, 2)
-    TIGR_MLP(TIGR_FRONTIER_NONE, false, 2) TIGR_MLP(TIGR_FRONTIER_NONE, true, 2)
     TIGR_MLP(TIGR_FRONTIER_DENSE, false, 4) TIGR_MLP(TIGR_FRONTIER_DENSE, true, 4)
     TIGR_MLP(TIGR_FRONTIER_NONE, false, 4) TIGR_MLP(TIGR_FRONTIER_NONE, true, 4)
 #undef TIGR_MLP
@@ -270,9 +265,8 @@ static RelaxFn pick_mlp(int front, bool bsp, int B) {
 
 // multi-vnode frontier kernel, or nullptr (then relax_kernel's one-vnode-per-thread kernel)
 RelaxFn relax_mlp_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats, int* per_thread) {
-    const int var = fr_variant();
-    if (!vec || stats || var == 0 || algo == TIGR_PR) return nullptr;
-    const int B = var == 1 ? 2 : 4;
+    if (!vec || stats || algo == TIGR_PR) return nullptr;
+    constexpr int B = 4;  // 4 virtual nodes per thread (cfg4 sweep; the 2-per-thread shape is slower)
     *per_thread = B;
     const bool st = layout == TIGR_LAYOUT_STRIDED;
     switch (algo) {
@@ -316,96 +310,10 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_pr(RelaxArgs a) {
     }
 }
 
-// PageRank push, B virtual nodes per thread, loads of every stage issued for all B vnodes
-// before the first atomic (memory-level parallelism: the per-vnode chain vn_phys -> node
-// record -> edge chunks is three dependent latencies; B independent chains overlap them).
-// Thread t of block b handles vnodes b*B*T + r*T + t (r < B), so each stage stays coalesced.
-template <int LAYOUT, int B, bool HINT>
-__global__ void __launch_bounds__(kRelaxThreads) k_relax_pr_mlp(RelaxArgs a) {
-    const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * kRelaxThreads) + threadIdx.x;
-    const uint64_t pol = HINT ? policy_evict_last() : 0;
-    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
-    uint32_t v[B];
-#pragma unroll
-    for (int r = 0; r < B; ++r) {
-        const uint64_t i = base + (uint64_t)r * kRelaxThreads;
-        v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
-    }
-    uint4 info[B];
-    double x[B];
-#pragma unroll
-    for (int r = 0; r < B; ++r) {
-        info[r] = make_uint4(0, 0, 0, 1);
-        x[r] = 0.0;
-        if (v[r] != kPad) { info[r] = __ldg(a.vinfo + v[r]); x[r] = __ldg(a.contrib + v[r]); }
-    }
-    uint4 c0[B], c1[B];
-    uint32_t kn[B], kend[B], step[B];
-#pragma unroll
-    for (int r = 0; r < B; ++r) {
-        const uint64_t i = base + (uint64_t)r * kRelaxThreads;
-        const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
-        uint32_t k;
-        if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
-        else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
-        else {
-            const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
-            k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
-            kend[r] = (per >= q - k) ? q : k + per;
-        }
-        const uint4* cb = c4 + info[r].x;
-        c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
-        c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
-        kn[r] = k + 2 * step[r];
-    }
-#pragma unroll
-    for (int r = 0; r < B; ++r) {
-        const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
-#pragma unroll
-        for (int t = 0; t < 8; ++t) {
-            if (nb[t] == kPad) continue;
-            if (HINT) red_add_f64(a.acc + nb[t], x[r], pol);
-            else atomicAdd(a.acc + nb[t], x[r]);
-        }
-    }
-    // chunks beyond the first two (K > 8, or K = no-split): rare, plain loop
-#pragma unroll
-    for (int r = 0; r < B; ++r) {
-        const uint4* cb = c4 + info[r].x;
-        for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
-            const uint4 c = ldg_chunk(cb + k);
-            const uint32_t nb[4] = {c.x, c.y, c.z, c.w};
-#pragma unroll
-            for (int t = 0; t < 4; ++t) {
-                if (nb[t] == kPad) continue;
-                if (HINT) red_add_f64(a.acc + nb[t], x[r], pol);
-                else atomicAdd(a.acc + nb[t], x[r]);
-            }
-        }
-    }
-}
+// sampled in-degree (PageRank accumulator order, pr.cu): every kHotSampleStride-th 16-byte
+// chunk of the arc array
+constexpr int kHotSampleStride = 16;
 
-// ------------------------------------------------------------------------------------------
-// PageRank push with the hottest destinations privatised in shared memory.
-//
-// Power-law in-degrees make the RED traffic collide on a few L2 sectors (cfg4: the top vertex
-// receives 0.14% of all arcs, and the 4 vertices of its 32-byte sector ~0.24%); B200 serialises
-// same-sector reductions, which caps skewed f64 REDs at ~70 G/s versus ~190 G/s spread
-// (tools/micro/red_bench.cu).  Each persistent block keeps an open-addressing table of the
-// hottest destinations (sampled in-degree, chosen on the device) in shared memory, adds their
-// contributions there, and flushes one RED per hot vertex at the end.  All other arcs RED
-// straight to L2.  Same sums, different association order (PR parity is 1e-6).
-// ------------------------------------------------------------------------------------------
-int pr_variant();
-
-constexpr int kHotMaxSlots = 8192;        // largest table (power of two)
-constexpr int kHotMaxIds = kHotMaxSlots / 4;  // load factor <= 1/4: ~1.4 probes for a miss
-constexpr int kHotSampleStride = 16;      // sample every 16th 16-byte chunk of the arc array
-
-template <int LOGS>
-__device__ __forceinline__ uint32_t hot_hash(uint32_t v) { return (v * 0x9E3779B1u) >> (32 - LOGS); }
-
-// sampled in-degree: every kHotSampleStride-th chunk of the arc array
 __global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uint32_t* __restrict__ cnt) {
     for (uint64_t k = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) * kHotSampleStride; k < nchunks;
          k += (uint64_t)gridDim.x * blockDim.x * kHotSampleStride) {
@@ -415,212 +323,6 @@ __global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uin
         if (c.z != kPad) atomicAdd(cnt + c.z, 1u);
         if (c.w != kPad) atomicAdd(cnt + c.w, 1u);
     }
-}
-
-// histogram of floor(log2(count)) (bucket 0 = count 0)
-__global__ void k_hot_loghist(const uint32_t* __restrict__ cnt, uint32_t n, uint32_t* __restrict__ hist) {
-    __shared__ uint32_t h[33];
-    if (threadIdx.x < 33) h[threadIdx.x] = 0;
-    __syncthreads();
-    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        const uint32_t c = cnt[v];
-        if (c) atomicAdd(&h[32 - __clz(c)], 1u);
-    }
-    __syncthreads();
-    if (threadIdx.x < 33 && h[threadIdx.x]) atomicAdd(&hist[threadIdx.x], h[threadIdx.x]);
-}
-
-// hot = sampled count >= 2^(b-1) for the smallest bucket b keeping #hot <= max_ids (and >= 2)
-__global__ void k_hot_compact(const uint32_t* __restrict__ cnt, uint32_t n, const uint32_t* __restrict__ hist,
-                              uint32_t max_ids, uint32_t* __restrict__ hot_ids, uint32_t* __restrict__ n_hot) {
-    __shared__ uint32_t thr;
-    if (threadIdx.x == 0) {
-        uint32_t acc = 0, b = 33;
-        while (b > 2 && acc + hist[b - 1] <= max_ids) { acc += hist[b - 1]; --b; }
-        thr = (b >= 33) ? 0xFFFFFFFFu : (1u << (b - 1));  // bucket b holds counts in [2^(b-1), 2^b)
-    }
-    __syncthreads();
-    const uint32_t t = thr;
-    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
-        if (cnt[v] >= t && cnt[v] >= 2) {
-            const uint32_t h = atomicAdd(n_hot, 1u);
-            if (h < max_ids) hot_ids[h] = v;
-        }
-    }
-}
-
-// LOGS: log2 of the table size (2^LOGS slots, at most 2^LOGS / 4 hot ids); MINB: blocks/SM
-template <int LAYOUT, int B, int LOGS, int MINB, int MASKBITS = 0>
-__global__ void __launch_bounds__(kRelaxThreads, MINB) k_relax_pr_hot(RelaxArgs a, const uint32_t* __restrict__ hot_ids,
-                                                                     const uint32_t* __restrict__ n_hot_p, uint32_t tiles) {
-    constexpr int kSlots = 1 << LOGS;
-    extern __shared__ __align__(16) unsigned char hsm[];
-    double* s_acc = reinterpret_cast<double*>(hsm);
-    uint32_t* s_key = reinterpret_cast<uint32_t*>(hsm + sizeof(double) * kSlots);
-    const int t = threadIdx.x;
-    for (int i = t; i < kSlots; i += kRelaxThreads) { s_key[i] = kPad; s_acc[i] = 0.0; }
-    __syncthreads();
-    const uint32_t n_hot = min(*n_hot_p, (uint32_t)(kSlots / 4));
-    for (uint32_t h = t; h < n_hot; h += kRelaxThreads) {
-        const uint32_t id = hot_ids[h];
-        uint32_t s = hot_hash<LOGS>(id);
-        while (atomicCAS(&s_key[s], kPad, id) != kPad) s = (s + 1) & (kSlots - 1);
-    }
-    __syncthreads();
-    const uint64_t pol = policy_evict_last();
-    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
-    auto push = [&](uint32_t nb, double x) {
-        uint32_t s = hot_hash<LOGS>(nb);
-        for (;;) {
-            const uint32_t k = s_key[s];
-            if (k == nb) { atomicAdd(&s_acc[s], x); return; }
-            if (k == kPad) {  // MASKBITS: timing experiment only (folds targets into 2^MASKBITS slots)
-                red_add_f64(a.acc + (MASKBITS ? (nb & ((1u << MASKBITS) - 1)) : nb), x, pol);
-                return;
-            }
-            s = (s + 1) & (kSlots - 1);
-        }
-    };
-    for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
-        const uint64_t base = (uint64_t)a.lo + (uint64_t)tile * (B * kRelaxThreads) + t;
-        uint32_t v[B];
-#pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
-            v[r] = i < a.hi ? __ldg(a.vn_phys + i) : kPad;
-        }
-        uint4 info[B];
-        double x[B];
-#pragma unroll
-        for (int r = 0; r < B; ++r) {
-            info[r] = make_uint4(0, 0, 0, 1);
-            x[r] = 0.0;
-            if (v[r] != kPad) { info[r] = __ldg(a.vinfo + v[r]); x[r] = __ldg(a.contrib + v[r]); }
-        }
-        uint4 c0[B], c1[B];
-        uint32_t kn[B], kend[B], step[B];
-#pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint64_t i = base + (uint64_t)r * kRelaxThreads;
-            const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
-            uint32_t k;
-            if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
-            else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
-            else {
-                const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
-                k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
-                kend[r] = (per >= q - k) ? q : k + per;
-            }
-            const uint4* cb = c4 + info[r].x;
-            c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
-            c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
-            kn[r] = k + 2 * step[r];
-        }
-#pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
-#pragma unroll
-            for (int q = 0; q < 8; ++q)
-                if (nb[q] != kPad) push(nb[q], x[r]);
-        }
-#pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint4* cb = c4 + info[r].x;
-            for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
-                const uint4 c = ldg_chunk(cb + k);
-                const uint32_t nb[4] = {c.x, c.y, c.z, c.w};
-#pragma unroll
-                for (int q = 0; q < 4; ++q)
-                    if (nb[q] != kPad) push(nb[q], x[r]);
-            }
-        }
-    }
-    __syncthreads();
-    for (int i = t; i < kSlots; i += kRelaxThreads) {
-        const uint32_t k = s_key[i];
-        if (k != kPad && s_acc[i] != 0.0) red_add_f64(a.acc + k, s_acc[i], pol);
-    }
-}
-
-uint32_t pr_hot_max() { return kHotMaxIds; }
-
-// sampled in-degrees -> device list of at most max_ids hottest destinations (no host sync)
-tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uint32_t max_ids, uint32_t* cnt_tmp,
-                          uint32_t* hist_tmp, uint32_t* hot_ids, uint32_t* n_hot, cudaStream_t s) {
-    TIGR_CK(cudaMemsetAsync(cnt_tmp, 0, sizeof(uint32_t) * n, s));
-    TIGR_CK(cudaMemsetAsync(hist_tmp, 0, sizeof(uint32_t) * 33, s));
-    TIGR_CK(cudaMemsetAsync(n_hot, 0, sizeof(uint32_t), s));
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const uint64_t samples = (nchunks + kHotSampleStride - 1) / kHotSampleStride;
-    if (samples) {
-        k_hot_sample<<<grid_for(samples < (uint64_t)sms * 2048 ? samples : (uint64_t)sms * 2048), kBlock, 0, s>>>(
-            reinterpret_cast<const uint4*>(col), nchunks, cnt_tmp);
-        TIGR_CKL("hot sample");
-    }
-    const unsigned g = (unsigned)std::min<uint64_t>(grid_for(n), (uint64_t)sms * 8);
-    k_hot_loghist<<<g, kBlock, 0, s>>>(cnt_tmp, n, hist_tmp);
-    TIGR_CKL("hot loghist");
-    k_hot_compact<<<g, kBlock, 0, s>>>(cnt_tmp, n, hist_tmp, max_ids, hot_ids, n_hot);
-    TIGR_CKL("hot compact");
-    return TIGR_OK;
-}
-
-template <int B, int LOGS, int MINB, int MASKBITS = 0>
-static PrHotConfig make_hot(int layout) {
-    PrHotConfig c;
-    c.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_hot<TIGR_LAYOUT_STRIDED, B, LOGS, MINB, MASKBITS>
-                                         : &k_relax_pr_hot<TIGR_LAYOUT_CONSECUTIVE, B, LOGS, MINB, MASKBITS>;
-    c.vnodes_per_thread = B;
-    c.smem = (sizeof(double) + sizeof(uint32_t)) << LOGS;
-    c.max_ids = (1u << LOGS) / 4;
-    return c;
-}
-
-// variants (TIGR_PR_VARIANT): 6 = 8192 slots, 4 vnodes/thread; 7 = 8192, 2/thread;
-// 8 = 4096 slots, 4/thread; 9 = 2048 slots, 4/thread; 10 = 4096 slots, 2/thread
-PrHotConfig relax_pr_hot_config(int layout, bool vec) {
-    PrHotConfig none;
-    if (!vec) return none;
-    switch (pr_variant()) {
-        case 6: return make_hot<4, 13, 2>(layout);
-        case 7: return make_hot<2, 13, 2>(layout);
-        case 8: return make_hot<4, 12, 3>(layout);
-        case 9: return make_hot<4, 11, 3>(layout);
-        case 10: return make_hot<2, 12, 4>(layout);
-        case 11: return make_hot<4, 13, 2, 23>(layout);   // timing experiment: wrong results
-        case 12: return make_hot<4, 13, 2, 22>(layout);   // timing experiment: wrong results
-        default: return none;
-    }
-}
-
-// kernel variant (development knob, TIGR_PR_VARIANT): 0 = one vnode per thread (k_relax_pr),
-// 1/2/3/4 = 1/2/4/8 vnodes per thread with L2 hints, 5 = 4 per thread without the RED hint
-int pr_variant() {
-    const char* e = getenv("TIGR_PR_VARIANT");
-    return e ? atoi(e) : 6;
-}
-
-int pr_vnodes_per_thread(int layout, bool vec, bool stats) {
-    const int var = pr_variant();
-    if (!vec || stats || var == 0) return 1;
-    return var == 1 ? 1 : (var == 2 ? 2 : (var == 3 ? 4 : (var == 4 ? 8 : (var == 5 ? 4 : 1))));
-}
-
-RelaxFn relax_pr_mlp_kernel(int layout, bool vec, bool stats) {
-    const int var = pr_variant();
-    if (!vec || stats || var == 0) return nullptr;
-    const bool st = layout == TIGR_LAYOUT_STRIDED;
-#define TIGR_PR_PICK(VAR, B, H) \
-    if (var == VAR) return st ? &k_relax_pr_mlp<TIGR_LAYOUT_STRIDED, B, H> : &k_relax_pr_mlp<TIGR_LAYOUT_CONSECUTIVE, B, H>;
-    TIGR_PR_PICK(1, 1, true)
-    TIGR_PR_PICK(2, 2, true)
-    TIGR_PR_PICK(3, 4, true)
-    TIGR_PR_PICK(4, 8, true)
-    TIGR_PR_PICK(5, 4, false)
-#undef TIGR_PR_PICK
-    return nullptr;
 }
 
 // ------------------------------------------------------------------------------------------
@@ -671,7 +373,8 @@ RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool s
 // ------------------------------------------------------------------------------------------
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
                        uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
-                       const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order) {
+                       const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order,
+                       uint32_t* __restrict__ settled) {
     // reordered graphs (tigr_graph_reorder): the source is an original id, CC labels are
     // original ids (the minimum original id of the component)
     const uint32_t src = cid ? cid[source] : source;
@@ -682,6 +385,9 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
         else if (algo == TIGR_SSWP) x = 0;
         if (v == src && algo != TIGR_CC) x = (algo == TIGR_SSWP) ? kInf : 0;
         val[v] = x;
+        // the source's value (BFS/SSSP 0, SSWP infinity) is final from the start: its settled bit
+        // (cleared before this kernel; frontier_kernel.cuh) spares every gather of it
+        if (settled && v == src && algo != TIGR_CC) atomicOr(settled + (v >> 5), 1u << (v & 31u));
         stamp[v] = 0u;                                                // parity 0
         stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == src) ? 1u : 0u;  // parity 1: it = 1
     }
@@ -690,6 +396,8 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
         ctl->xchanged[0] = 0; ctl->xchanged[1] = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
         ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0; ctl->nodes = 0;
+        ctl->bound_id = algo == TIGR_SSWP ? 0u : kInf;  // max / min identity
+        ctl->bound[0] = ctl->bound_id; ctl->bound[1] = ctl->bound_id;
     }
 }
 
@@ -710,9 +418,14 @@ tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* ou
 
 // end of one iteration: decide whether to continue; sets the graph's WHILE condition
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle) {
+    if (!ctl->cont) {  // already stopped: an iteration enqueued past the fixed point (run.cu)
+        if (use_handle) cudaGraphSetConditional(h, 0);
+        return;
+    }
     const uint32_t changed = ctl->changed;
     ctl->nodes += ctl->qpack[ctl->it & 1u] >> 32;
     ctl->qpack[ctl->it & 1u] = 0ull;  // queue slot consumed by this iteration (frontier.cu)
+    ctl->bound[ctl->it & 1u] = ctl->bound_id;  // and its frontier bound
     uint32_t cont = changed ? 1u : 0u;
     if (changed && ctl->it >= ctl->max_iters) { cont = 0; ctl->notconv = 1; }
     ctl->changed = 0;
@@ -724,6 +437,7 @@ __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle
 // multi-GPU: after the all-reduce, activate every node whose replica value moved
 __global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
                        uint32_t* __restrict__ stamp, Ctl* ctl) {
+    if (!ctl->cont) return;  // past the fixed point (batched host loop, run.cu)
     const uint32_t it = ctl->it;
     bool moved = false;
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;

@@ -40,7 +40,7 @@ struct FqArgs {
     const uint32_t* qo;   // uint32[2][n] queue-space first virtual node of each entry
     int mode;             // 0 = per iteration (queue if vnodes * dense_div < span), 1 = queue, 2 = dense
     uint32_t dense_div;
-    uint32_t* settled;    // BFS only: bit v set once v's level is final (nullptr: test the value)
+    uint32_t* settled;    // bit v set once v's value is final (nullptr: always test the value)
     const FusedPeers* peers;  // fused exchange: every improvement is also applied to the peers' replicas
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
@@ -48,24 +48,16 @@ FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);
 unsigned relax_fq_grid(FqFn fn);   // persistent grid: SMs x resident blocks
 int relax_fq_threads();
 struct Ctl;
-tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s);
+// bmode: frontier bound into ctl->bound (0 none, 1 min = SSSP, 2 max = SSWP); bound_all: over
+// every stamped node (replicas), else over the stamped nodes with arcs in this rank's range;
+// settled (nullable): SSSP / SSWP bitmap the compaction settles by the previous bound
+tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s, int bmode, int bound_all,
+                           const uint32_t* settled);
 typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
 
 RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats);
 // frontier relax with *per_thread virtual nodes per thread (nullptr: use relax_kernel's)
 RelaxFn relax_mlp_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats, int* per_thread);
-// PageRank push with several virtual nodes per thread (nullptr: use relax_kernel's); B per thread
-RelaxFn relax_pr_mlp_kernel(int layout, bool vec, bool stats);
-int pr_vnodes_per_thread(int layout, bool vec, bool stats);
-// PageRank push with shared-memory privatisation of the hottest destinations (persistent grid)
-typedef void (*RelaxHotFn)(RelaxArgs, const uint32_t*, const uint32_t*, uint32_t);
-struct PrHotConfig {
-    RelaxHotFn fn = nullptr;
-    int vnodes_per_thread = 1;
-    size_t smem = 0;          // dynamic shared memory per block
-    uint32_t max_ids = 0;     // hot destinations the table holds
-};
-PrHotConfig relax_pr_hot_config(int layout, bool vec);
 // PageRank push with an in-degree-ordered accumulator (pr.cu)
 struct PrFuse {
     int mode = 0;               // 0 read contrib, 1 first iteration (x = x0), 2 from prev
@@ -80,20 +72,17 @@ struct PrCidPlan {
     int threads = 256, per_thread = 4;
     size_t smem = 0;
 };
-bool pr_cid_enabled();
 RelaxFn relax_pr_pull_kernel(int layout, int* per_thread);   // pull PageRank (pr.cu, NEXT-1)
 tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s);
 PrCidPlan pr_cid_plan(tigr_vgraph* vg);
 tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,
                          double* dsum_next, cudaStream_t s, double* acc = nullptr, bool reset = true);
-uint32_t pr_hot_max();        // capacity of the workspace's hot-id list (>= any config's max_ids)
-tigr_status pr_hot_select(const uint32_t* col, uint64_t nchunks, uint32_t n, uint32_t max_ids, uint32_t* cnt_tmp,
-                          uint32_t* hist_tmp, uint32_t* hot_ids, uint32_t* n_hot, cudaStream_t s);
 AssignFn assign_kernel(int layout, bool vec);
 
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
                        uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
-                       const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order);
+                       const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order,
+                       uint32_t* __restrict__ settled);
 // out[v] = val[cid[v]] (results of a reordered graph in original ids)
 tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* out, bool f64, cudaStream_t s);
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle);

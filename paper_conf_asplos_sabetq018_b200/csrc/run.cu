@@ -7,6 +7,7 @@
 // on the device, so there is no host round trip per iteration (the paper copies `finished`
 // back every iteration).  PageRank runs pr_iters x (relax -> [all-reduce] -> apply).
 #include <algorithm>
+#include <mutex>
 #include <vector>
 
 #include "internal.cuh"
@@ -17,7 +18,36 @@ namespace tigr {
 
 tigr_status comm_allreduce(tigr_comm* c, void* buf, size_t count, int algo, cudaStream_t s);
 
+// Pinned host mirrors of the control block, one per workspace (a vgraph may be run from any
+// thread, and two vgraphs may run at once on different threads, so the mirror is never shared).
+// cudaMallocHost synchronises the device, and the bench rebuilds its vgraph every step, so
+// mirrors come from a process-wide free list that grows in slabs and never shrinks.
+namespace {
+std::mutex g_ctl_mu;
+std::vector<Ctl*> g_ctl_free;
+}  // namespace
+
+Ctl* pinned_ctl_acquire() {
+    std::lock_guard<std::mutex> lk(g_ctl_mu);
+    if (g_ctl_free.empty()) {
+        constexpr int kSlab = 64;
+        Ctl* slab = nullptr;
+        if (cudaMallocHost(&slab, sizeof(Ctl) * kSlab) != cudaSuccess) return nullptr;
+        for (int i = kSlab - 1; i >= 0; --i) g_ctl_free.push_back(slab + i);
+    }
+    Ctl* c = g_ctl_free.back();
+    g_ctl_free.pop_back();
+    return c;
+}
+
+void pinned_ctl_release(Ctl* c) {
+    if (!c) return;
+    std::lock_guard<std::mutex> lk(g_ctl_mu);
+    g_ctl_free.push_back(c);
+}
+
 Workspace::~Workspace() {
+    pinned_ctl_release(ctl_host);
     for (auto& kv : graphs) {
         if (kv.second.exec) cudaGraphExecDestroy(kv.second.exec);
         if (kv.second.stream) cudaStreamDestroy(kv.second.stream);
@@ -34,11 +64,8 @@ tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
     const size_t n = vg->g->n ? vg->g->n : 1;
     if (!ws.ctl.p) {
         TIGR_TRY(ws.ctl.alloc(sizeof(Ctl), s));
-        // pinned control-block mirror: one per host thread for the process lifetime (a
-        // cudaMallocHost per vgraph would synchronise the device on every graph rebuild)
-        static thread_local Ctl* t_ctl = nullptr;
-        if (!t_ctl) TIGR_CK(cudaMallocHost(&t_ctl, sizeof(Ctl)));
-        ws.ctl_host = t_ctl;
+        ws.ctl_host = pinned_ctl_acquire();
+        if (!ws.ctl_host) return fail(TIGR_ENOMEM, "cudaMallocHost of the control-block mirror failed");
         for (auto& e : ws.ev) TIGR_CK(cudaEventCreate(&e));
     }
     if (pr) {
@@ -46,7 +73,6 @@ tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
             TIGR_TRY(ws.x.alloc(sizeof(double) * n, s));
             TIGR_TRY(ws.contrib.alloc(sizeof(double) * n, s));
             TIGR_TRY(ws.acc.alloc(sizeof(double) * n, s));
-            TIGR_TRY(ws.hot.alloc(sizeof(uint32_t) * (n + 34 + pr_hot_max()), s));
         }
     } else if (!ws.val.p) {
         TIGR_TRY(ws.val.alloc(sizeof(uint32_t) * n, s));
@@ -90,6 +116,7 @@ struct FrontierPlan {
     unsigned grid;
     bool bsp, comm;
     bool fused = false;    // TIGR_EXCHANGE_FUSED: the relax updates the peers' replicas itself
+    int bmode = 0;         // frontier bound for the settled test (frontier.cu k_compact): 1 SSSP, 2 SSWP
     int algo;
     tigr_comm* c;
     uint32_t n;
@@ -98,7 +125,7 @@ struct FrontierPlan {
 // enqueue one iteration body; returns number of kernels it launches
 tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditionalHandle h, int use_handle,
                          int* kernels, cudaEvent_t ev_a = nullptr, cudaEvent_t ev_b = nullptr,
-                         uint32_t* sparse_count = nullptr) {
+                         uint32_t* sparse_count = nullptr, cudaEvent_t ev_c = nullptr) {
     int k = 0;
     if (p.bsp && (!p.comm || p.fused))
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * p.n, cudaMemcpyDeviceToDevice, s));
@@ -121,8 +148,9 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
         TIGR_TRY(exchange_frontier(p.xa, s, &sparse));  // its kernels count their own launches
         if (sparse && sparse_count) ++*sparse_count;
     }
+    if (ev_c) TIGR_CK(cudaEventRecord(ev_c, s));
     if (p.fq) {  // next iteration's queue from the stamps just written
-        TIGR_TRY(compact_launch(p.vg, p.args.ctl, 1, s));
+        TIGR_TRY(compact_launch(p.vg, p.args.ctl, 1, s, p.bmode, p.comm ? 1 : 0, p.fa.settled));
         ++k;
     }
     k_control<<<1, 1, 0, s>>>(p.args.ctl, h, use_handle);
@@ -144,16 +172,15 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         p.fa.qv = ws.qv.as<uint32_t>();
         p.fa.qo = ws.qo.as<uint32_t>();
         p.fa.mode = front == TIGR_FRONTIER_QUEUE ? 1 : 0;
-        const char* e = getenv("TIGR_FQ_MODE");   // development knob: force 1 = queue, 2 = dense
-        if (e && front == TIGR_FRONTIER_AUTO) p.fa.mode = atoi(e);
-        const char* d = getenv("TIGR_FQ_DIV");
-        p.fa.dense_div = d ? (uint32_t)atoi(d) : 2u;
+        if (front == TIGR_FRONTIER_AUTO) p.fa.mode = dev_knob("TIGR_FQ_MODE", 0);  // 1 queue, 2 dense
+        p.fa.dense_div = o.frontier_div ? o.frontier_div : 2u;
         p.fa.settled = nullptr;
         p.fa.peers = nullptr;
-        const char* bb = getenv("TIGR_BFS_BITS");  // development knob: 0 = test the values instead
-        if ((algo == TIGR_BFS || algo == TIGR_CC) && !(bb && atoi(bb) == 0)) {
+        // settled bitmap (frontier_kernel.cuh): a target whose value is final is never gathered
+        if (dev_knob("TIGR_SETTLED_BITS", 1)) {
             if (!ws.settled.p) TIGR_TRY(ws.settled.alloc(sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
             p.fa.settled = ws.settled.as<uint32_t>();
+            p.bmode = algo == TIGR_SSSP ? 1 : (algo == TIGR_SSWP ? 2 : 0);
         }
     } else if (front == TIGR_FRONTIER_QUEUE) {
         return fail(TIGR_EUNSUPPORTED, "frontier QUEUE needs the 16-byte-chunk layout (4 | K)");
@@ -196,19 +223,20 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     cudaEvent_t t0 = ws.ev[0], t1 = ws.ev[1];
     TIGR_CK(cudaEventRecord(t0, s));
     const tigr_graph* gg = vg->g;
+    if (p.fq && p.fa.settled) TIGR_CK(cudaMemsetAsync(p.fa.settled, 0, sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
     k_init<<<grid_for(n), kBlock, 0, s>>>(algo, n, source, p.args.val, p.args.stamp, p.args.ctl, max_iters,
                                           gg->reordered ? gg->perm_cid.as<uint32_t>() : nullptr,
-                                          gg->reordered ? gg->perm_order.as<uint32_t>() : nullptr);
+                                          gg->reordered ? gg->perm_order.as<uint32_t>() : nullptr,
+                                          p.fq ? p.fa.settled : nullptr);
     TIGR_CKL("init");
-    if (p.fq && p.fa.settled) TIGR_CK(cudaMemsetAsync(p.fa.settled, 0, sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
     if (p.bsp || p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
-    if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s));  // iteration 1's queue
+    if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s, p.bmode, p.comm ? 1 : 0, p.fa.settled));  // iteration 1's queue
     if (p.fused) TIGR_TRY(fused_barrier(p.c, s));  // every replica initialised before any remote update
 
     int kpi = 0;
     uint32_t launches = 0, sparse_exchanges = 0;
-    double ms_relax = 0.0;
+    double ms_relax = 0.0, ms_ex = 0.0;
     // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
     const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
     if (use_graph) {
@@ -251,18 +279,32 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         TIGR_CK(cudaEventRecord(ws.ev[3], cg.stream));
         TIGR_CK(cudaStreamWaitEvent(s, ws.ev[3], 0));
     } else {
+        // Host loop (multi-GPU, time_kernels, use_graph = 0).  Iterations are enqueued in batches
+        // and the control block is read back once per batch: every kernel of an iteration body
+        // returns at once when ctl->cont is already 0, so the iterations enqueued past the fixed
+        // point are no-ops (a dense exchange's all-reduce then merges identical replicas).  The
+        // dense exchange decides nothing on the host, so it batches 4 iterations per round trip;
+        // the sparse and fused exchanges and per-launch timing need the host every iteration.
+        const bool dense_x = p.comm && !p.fused && o.exchange == TIGR_EXCHANGE_DENSE;
+        const int batch = (dense_x && !o.time_kernels) ? 4 : 1;
         for (;;) {
-            int k = 0;
-            TIGR_TRY(enqueue_body(p, s, 0, 0, &k, o.time_kernels ? ws.ev[2] : nullptr,
-                                  o.time_kernels ? ws.ev[3] : nullptr, &sparse_exchanges));
-            count_launch(k);
-            launches += p.grid ? 1 : 0;
+            for (int b = 0; b < batch; ++b) {
+                int k = 0;
+                TIGR_TRY(enqueue_body(p, s, 0, 0, &k, o.time_kernels ? ws.ev[2] : nullptr,
+                                      o.time_kernels ? ws.ev[3] : nullptr, &sparse_exchanges,
+                                      o.time_kernels && p.comm ? ws.ev[4] : nullptr));
+                count_launch(k);
+            }
             TIGR_CK(cudaMemcpyAsync(ws.ctl_host, p.args.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
             TIGR_CK(cudaStreamSynchronize(s));
             if (o.time_kernels && p.grid) {
                 float ms = 0.f;
                 TIGR_CK(cudaEventElapsedTime(&ms, ws.ev[2], ws.ev[3]));
                 ms_relax += ms;
+                if (p.comm) {
+                    TIGR_CK(cudaEventElapsedTime(&ms, ws.ev[3], ws.ev[4]));
+                    ms_ex += ms;
+                }
             }
             if (!ws.ctl_host->cont) break;
         }
@@ -271,9 +313,9 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     TIGR_CK(cudaMemcpyAsync(ws.ctl_host, p.args.ctl, sizeof(Ctl), cudaMemcpyDeviceToHost, s));
     TIGR_CK(cudaStreamSynchronize(s));
     const Ctl& c = *ws.ctl_host;
+    launches = p.grid ? c.it : 0;  // one relax launch per executed iteration
     if (use_graph) {
         count_launch((uint64_t)c.it * kpi);
-        launches = p.grid ? c.it : 0;
     }
     if (st) {
         float ms = 0.f;
@@ -288,6 +330,16 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         st->queue_iterations = c.queue_iters;
         st->active_nodes = c.nodes;
         st->sparse_exchanges = sparse_exchanges;
+        st->ms_exchange = ms_ex;
+        st->ms_kernels = ms - ms_ex;
+        // SURVEY §8(d) byte model: per processed arc s_e (+4 weight) + 4 (target
+        // value), per update 4, per active virtual node 4 (vn_phys), per active node with arcs
+        // 12 (value + row pair), per iteration 2 B per node (frontier flags read + cleared)
+        if (o.collect_stats) {
+            const uint64_t s_e = (algo == TIGR_SSSP || algo == TIGR_SSWP) ? 8 : 4;
+            st->bytes_alg = c.edges * (s_e + 4) + c.updates * 4 + c.vnodes * 4 + c.nodes * 12 +
+                            (uint64_t)c.it * 2 * n;
+        }
     }
     if (c.notconv) return fail(TIGR_ENOTCONV, "max_iters reached before the fixed point");
     return TIGR_OK;
@@ -297,14 +349,15 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     Workspace& ws = vg->ws;
     const uint32_t n = vg->g->n;
     RelaxArgs a = make_args(vg);
-    // preferred: in-degree-ordered accumulator (pr.cu); else the hashed hot-destination kernel
-    // a transposed graph runs pull-based PageRank (pr.cu, NEXT-1); divide by the original
-    // graph's out-degrees, which the transpose carries
+    // preferred: the in-degree-ordered accumulator (pr.cu k_relax_pr_cid); a transposed graph
+    // runs pull-based PageRank (pr.cu, NEXT-1) and divides by the original graph's
+    // out-degrees, which the transpose carries; 4 ∤ K layouts and stats runs use the plain
+    // one-vnode-per-thread push (relax.cu k_relax_pr)
     const bool pull = vg->g->transposed;
     if (o.pr_dangling && (vg->g->part_lo != 0 || vg->g->part_hi < n))
         return fail(TIGR_EUNSUPPORTED, "pr_dangling = 1 needs every out-degree: not on a partitioned graph");
     const uint32_t* out_deg = pull ? vg->g->src_deg.as<uint32_t>() : vg->g->deg.as<uint32_t>();
-    const bool use_cid = !pull && !o.collect_stats && vg->vec && pr_cid_enabled();
+    const bool use_cid = !pull && !o.collect_stats && vg->vec;
     PrCidPlan cp;
     if (use_cid) {
         TIGR_TRY(pr_cid_prepare(vg, s));
@@ -312,37 +365,15 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
     }
     // fused apply (pr.cu PrFuse): the relax derives contributions from the previous accumulator;
     // two accumulators alternate; dangling-mass redistribution keeps the separate apply
-    const char* fe = getenv("TIGR_PR_FUSE");
-    const bool fuse = use_cid && !o.pr_dangling && !(fe && atoi(fe) == 0) && o.pr_iters > 0;
+    const bool fuse = use_cid && !o.pr_dangling && o.pr_iters > 0;
     if (fuse && !ws.acc2.p) TIGR_TRY(ws.acc2.alloc(sizeof(double) * (n ? n : 1), s));
-    // pull: sources in out-degree order (pr.cu pr_pull_prepare); TIGR_PR_PULL_OID=0 disables
-    const char* po = getenv("TIGR_PR_PULL_OID");
-    const bool pull_oid = pull && vg->vec && !(po && atoi(po) == 0);
+    // pull: sources in out-degree order (pr.cu pr_pull_prepare)
+    const bool pull_oid = pull && vg->vec;
     const uint32_t* oid = nullptr;
     if (pull_oid) {
         TIGR_TRY(pr_pull_prepare(vg, s));
         oid = ws.cid.as<uint32_t>();
         a.col = ws.col_pr.as<uint32_t>();
-    }
-    const PrHotConfig hc =
-        (pull || o.collect_stats || use_cid) ? PrHotConfig() : relax_pr_hot_config(vg->layout, vg->vec);
-    const RelaxHotFn hot = hc.fn;
-    uint32_t* hot_cnt = ws.hot.as<uint32_t>();
-    uint32_t* hot_hist = hot_cnt + n;
-    uint32_t* hot_n = hot_hist + 33;
-    uint32_t* hot_ids = hot_n + 1;
-    unsigned hot_grid = 0, hot_tiles = 0;
-    if (hot) {
-        TIGR_CK(cudaFuncSetAttribute(hot, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hc.smem));
-        int per_sm = 0, dev = 0, sms = 148;
-        TIGR_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, hot, kRelaxThreads, hc.smem));
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        const uint64_t per_tile = (uint64_t)kRelaxThreads * hc.vnodes_per_thread;
-        hot_tiles = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_tile - 1) / per_tile);
-        hot_grid = (unsigned)std::min<uint64_t>(hot_tiles, (uint64_t)sms * (per_sm > 0 ? per_sm : 1));
-        TIGR_TRY(pr_hot_select(vg->g->col.as<uint32_t>(), vg->g->nchunks, n, hc.max_ids, hot_cnt, hot_hist, hot_ids,
-                               hot_n, s));
     }
     RelaxFn relax = nullptr;
     uint64_t per_block = kRelaxThreads;
@@ -353,9 +384,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         relax = relax_pr_pull_kernel(vg->layout, &per);
         per_block *= per;
     } else {
-        relax = relax_pr_mlp_kernel(vg->layout, vg->vec, o.collect_stats != 0);
-        if (relax) per_block *= pr_vnodes_per_thread(vg->layout, vg->vec, o.collect_stats != 0);
-        else relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
+        relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
     }
     const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
     const bool comm = o.comm != nullptr;
@@ -395,10 +424,6 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         if (use_cid && cp.tiles) {
             cp.fn<<<cp.grid, cp.threads, cp.smem, s>>>(a, ws.col_pr.as<uint32_t>(), cp.tiles, fz);
             TIGR_CKL("pr relax (cid)");
-            ++launches;
-        } else if (hot && hot_tiles) {
-            hot<<<hot_grid, kRelaxThreads, hc.smem, s>>>(a, hot_ids, hot_n, hot_tiles);
-            TIGR_CKL("pr relax (hot)");
             ++launches;
         } else if (grid) {
             relax<<<grid, kRelaxThreads, 0, s>>>(a);
@@ -449,6 +474,12 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         st->ms_total = ms;
         st->ms_relax = ms_relax;
         st->ms_exchange = ms_ex;
+        st->ms_kernels = ms - ms_ex;
+        // SURVEY §8(d) byte model per relax launch: per arc 4 (target) + 16 (RED = read + write
+        // of the f64 accumulator), per virtual node 4, per node with arcs its source value: 20
+        // with the apply fused in (previous accumulator 8 + cid 4 + row pair 8), else 16
+        // (contrib 8 + row pair 8)
+        st->bytes_alg = (uint64_t)launches * (vg->g->m * 20 + (uint64_t)(vg->hi - vg->lo) * 4 + vg->n_out * (fuse ? 20 : 16));
     }
     return TIGR_OK;
 }
@@ -535,6 +566,17 @@ void partition_ranges(uint32_t n, const int64_t* rp, const uint32_t* vp, int nra
 
 // the same rule on the device: one thread per cut, binary search over row_ptr (no D2H of the
 // node arrays; only the 2 range bounds come back)
+// nodes with out-arcs among [cuts[0], cuts[1]) (cuts on the device, from k_partition)
+__global__ void k_count_out(const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cuts,
+                            unsigned long long* __restrict__ cnt) {
+    const uint32_t lo = cuts[0], hi = cuts[1];
+    uint32_t c = 0;
+    for (uint32_t v = lo + blockIdx.x * blockDim.x + threadIdx.x; v < hi; v += gridDim.x * blockDim.x) c += deg[v] != 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(cnt, (unsigned long long)c);
+}
+
 __global__ void k_partition(const int64_t* __restrict__ rp, const uint32_t* __restrict__ vp, uint32_t n,
                             int nranks, int rank, uint32_t* out) {
     const int c = threadIdx.x;  // 0: cut(rank), 1: cut(rank + 1)
@@ -554,23 +596,39 @@ __global__ void k_partition(const int64_t* __restrict__ rp, const uint32_t* __re
         cut = lo;
     }
     out[c] = vp[cut];
+    out[2 + c] = cut;
 }
 
 tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank) {
     if (nranks < 1 || rank < 0 || rank >= nranks) return fail(TIGR_EINVAL, "partition: bad rank/nranks");
     const tigr_graph* g = vg->g;
-    if (nranks == 1 || g->n == 0) { vg->lo = 0; vg->hi = (uint32_t)vg->nv; return TIGR_OK; }
     cudaStream_t s = vg->vnode_ptr.s;
     TmpBuf out;
-    TIGR_TRY(out.alloc(2 * sizeof(uint32_t), s));
-    k_partition<<<1, 32, 0, s>>>(g->row_ptr.as<int64_t>(), vg->vnode_ptr.as<uint32_t>(), g->n, nranks, rank,
-                                 out.as<uint32_t>());
-    TIGR_CKL("partition");
-    uint32_t h[2] = {0, 0};
+    TIGR_TRY(out.alloc(4 * sizeof(uint32_t) + sizeof(unsigned long long), s));
+    unsigned long long* cnt = reinterpret_cast<unsigned long long*>(out.as<char>() + 16);
+    if (nranks == 1 || g->n == 0) {
+        vg->lo = 0;
+        vg->hi = (uint32_t)vg->nv;
+        const uint32_t full[4] = {0, (uint32_t)vg->nv, 0, g->n};
+        TIGR_CK(cudaMemcpyAsync(out.p, full, sizeof(full), cudaMemcpyHostToDevice, s));
+    } else {
+        k_partition<<<1, 32, 0, s>>>(g->row_ptr.as<int64_t>(), vg->vnode_ptr.as<uint32_t>(), g->n, nranks, rank,
+                                     out.as<uint32_t>());
+        TIGR_CKL("partition");
+    }
+    TIGR_CK(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long), s));
+    if (g->n) {
+        k_count_out<<<grid_for(g->n / 8 + 1), kBlock, 0, s>>>(g->deg.as<uint32_t>(), out.as<uint32_t>() + 2, cnt);
+        TIGR_CKL("partition count");
+    }
+    uint32_t h[4] = {0, 0, 0, 0};
+    unsigned long long hn = 0;
     TIGR_CK(cudaMemcpyAsync(h, out.p, sizeof(h), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaMemcpyAsync(&hn, cnt, sizeof(hn), cudaMemcpyDeviceToHost, s));
     TIGR_CK(cudaStreamSynchronize(s));
     vg->lo = h[0];
     vg->hi = h[1];
+    vg->n_out = hn;
     return TIGR_OK;
 }
 

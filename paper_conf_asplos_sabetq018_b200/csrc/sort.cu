@@ -13,6 +13,8 @@
 // padded segment of its source.
 #include <algorithm>
 #include <cstdlib>
+#include <map>
+#include <mutex>
 #include <utility>
 #include <vector>
 
@@ -50,30 +52,33 @@ __device__ __forceinline__ void coo_item(const uint32_t* __restrict__ src, const
 // (validation: checked on the host before any id is used as an index), and optionally the
 // in-degree sketch the PageRank accumulator order uses (pr.cu): a has-in-arcs flag per node
 // (tested before set, so hub targets do not serialise stores) and an in-degree count sampled
-// on every 16th arc.  Arc e of the (optionally symmetrised) list: key = source, t = target.
+// on every 16th item.  Covers the input arcs f in [f0, f1) -- the host-input build scans each
+// chunk as its copy lands (api.cu) -- and, when symmetrising (sym), their reversed items
+// m + f too.  Item e: key = source, t = target.
 __global__ void k_coo_scan(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
-                           uint64_t M, int passes, int bits, unsigned long long* __restrict__ hist,
-                           uint32_t* __restrict__ maxid, uint32_t n, uint8_t* __restrict__ in_flag,
-                           uint32_t* __restrict__ in_sample, uint32_t klo, uint32_t khi,
-                           unsigned long long* __restrict__ n_local) {
+                           uint64_t f0, uint64_t f1, int sym, int passes, int bits,
+                           unsigned long long* __restrict__ hist, uint32_t* __restrict__ maxid, uint32_t n,
+                           uint8_t* __restrict__ in_flag, uint32_t* __restrict__ in_sample, uint32_t klo,
+                           uint32_t khi, unsigned long long* __restrict__ n_local) {
     __shared__ uint32_t h[4][kMaxRadix];
     for (int i = threadIdx.x; i < 4 * kMaxRadix; i += blockDim.x) (&h[0][0])[i] = 0;
     __syncthreads();
     const uint32_t mask = (1u << bits) - 1;
     uint32_t mx = 0, local = 0;
-    for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < M; e += (uint64_t)gridDim.x * blockDim.x) {
-        const bool rev = e >= m;
-        const uint64_t f = rev ? e - m : e;
+    for (uint64_t f = f0 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; f < f1; f += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t s = src[f], d = dst[f];
-        const uint32_t k = rev ? d : s, t = rev ? s : d;
         mx = max(mx, max(s, d));
-        if (k < n && k >= klo && k < khi) {  // this build's source range (partitioned graphs)
-            ++local;
-            for (int p = 0; p < passes; ++p) atomicAdd(&h[p][(k >> (p * bits)) & mask], 1u);
-        }
-        if (in_flag && t < n) {
-            if (!in_flag[t]) in_flag[t] = 1;
-            if ((e & 15) == 0) atomicAdd(in_sample + t, 1u);
+        for (int dir = 0; dir <= sym; ++dir) {
+            const uint64_t e = dir ? m + f : f;
+            const uint32_t k = dir ? d : s, t = dir ? s : d;
+            if (k < n && k >= klo && k < khi) {  // this build's source range (partitioned graphs)
+                ++local;
+                for (int p = 0; p < passes; ++p) atomicAdd(&h[p][(k >> (p * bits)) & mask], 1u);
+            }
+            if (in_flag && t < n) {
+                if (!in_flag[t]) in_flag[t] = 1;
+                if ((e & 15) == 0) atomicAdd(in_sample + t, 1u);
+            }
         }
     }
 #pragma unroll
@@ -366,18 +371,40 @@ unsigned sort_grid(uint64_t items) {
     return (unsigned)(want == 0 ? 1 : (want < cap ? want : cap));
 }
 
+// Host-input builds (api.cu tigr_graph_from_coo with host pointers): the arc list reaches the
+// device in chunks on a copy stream, and each chunk is scanned on the build stream as soon as
+// it lands, so the PCIe transfer and the scan overlap; the sort passes need the whole list.
+constexpr uint64_t kCopyChunk = 1ull << 24;  // arcs per chunk (64 MB per array)
+
+cudaStream_t copy_stream() {
+    static std::mutex mu;
+    static std::map<int, cudaStream_t> streams;  // one per device, for the process lifetime
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = streams.find(dev);
+    if (it != streams.end()) return it->second;
+    cudaStream_t cs = nullptr;
+    if (cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) != cudaSuccess) return nullptr;
+    streams[dev] = cs;
+    return cs;
+}
+
 template <bool W>
 tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* w, uint64_t m, uint64_t M,
                       uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out, bool validate,
                       uint8_t* in_flag = nullptr, uint32_t* in_sample = nullptr, uint32_t klo = 0,
-                      uint32_t khi = 0xFFFFFFFFu, uint64_t* M_out = nullptr) {
+                      uint32_t khi = 0xFFFFFFFFu, uint64_t* M_out = nullptr, const HostArcs* host = nullptr) {
     typedef typename ValT<W>::T VT;
     int key_bits = 0;
     while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
     const int passes = key_bits == 0 ? 1 : (key_bits + 7) / 8;
     const int bits = key_bits == 0 ? 1 : (key_bits + passes - 1) / passes;
-    const char* si_env = getenv("TIGR_SORT_SI");
-    const int SI = si_env ? atoi(si_env) : 16;
+    // items per thread: 16 (development builds may sweep 12/20/24 with TIGR_SORT_SI; the
+    // source-range-filtered first pass exists for 16 only, so filtered builds always use 16)
+    const bool filtered = klo != 0 || khi < n;
+    int SI = filtered ? 16 : dev_knob("TIGR_SORT_SI", 16);
+    if (SI != 12 && SI != 20 && SI != 24) SI = 16;
     const uint64_t tile_items = (uint64_t)kST * SI;
     const uint64_t tiles = (M + tile_items - 1) / tile_items;
 
@@ -399,10 +426,35 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     TIGR_CK(cudaMemsetAsync(maxid.p, 0, sizeof(uint32_t), s));
     TIGR_TRY(nloc.alloc(sizeof(unsigned long long), s));
     TIGR_CK(cudaMemsetAsync(nloc.p, 0, sizeof(unsigned long long), s));
-    const bool filtered = klo != 0 || khi < n;
     trace(s, "sort: alloc+memset");
-    if (M) {
-        k_coo_scan<<<sort_grid(M), kBlock, 0, s>>>(src, dst, m, M, passes, bits, hist.as<unsigned long long>(),
+    const int sym = M > m ? 1 : 0;
+    if (M && host) {  // src / dst / w are the device destinations of the host arrays
+        cudaStream_t cs = copy_stream();
+        if (!cs) return fail(TIGR_ECUDA, "graph_from_coo: copy stream creation failed");
+        cudaEvent_t ready;
+        TIGR_CK(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
+        TIGR_CK(cudaEventRecord(ready, s));  // the destinations (fresh allocations) are free on s
+        TIGR_CK(cudaStreamWaitEvent(cs, ready, 0));
+        cudaEventDestroy(ready);
+        for (uint64_t f0 = 0; f0 < m; f0 += kCopyChunk) {
+            const uint64_t f1 = std::min<uint64_t>(m, f0 + kCopyChunk);
+            const size_t bytes = sizeof(uint32_t) * (f1 - f0);
+            TIGR_CK(cudaMemcpyAsync(const_cast<uint32_t*>(src) + f0, host->src + f0, bytes, cudaMemcpyHostToDevice, cs));
+            TIGR_CK(cudaMemcpyAsync(const_cast<uint32_t*>(dst) + f0, host->dst + f0, bytes, cudaMemcpyHostToDevice, cs));
+            if (W) TIGR_CK(cudaMemcpyAsync(const_cast<uint32_t*>(w) + f0, host->w + f0, bytes, cudaMemcpyHostToDevice, cs));
+            cudaEvent_t landed;
+            TIGR_CK(cudaEventCreateWithFlags(&landed, cudaEventDisableTiming));
+            TIGR_CK(cudaEventRecord(landed, cs));
+            TIGR_CK(cudaStreamWaitEvent(s, landed, 0));
+            cudaEventDestroy(landed);  // released once it has completed
+            k_coo_scan<<<sort_grid(f1 - f0), kBlock, 0, s>>>(src, dst, m, f0, f1, sym, passes, bits,
+                                                              hist.as<unsigned long long>(), maxid.as<uint32_t>(), n,
+                                                              in_flag, in_sample, klo, khi,
+                                                              nloc.as<unsigned long long>());
+            TIGR_CKL("coo scan (chunk)");
+        }
+    } else if (M) {
+        k_coo_scan<<<sort_grid(m), kBlock, 0, s>>>(src, dst, m, 0, m, sym, passes, bits, hist.as<unsigned long long>(),
                                                     maxid.as<uint32_t>(), n, in_flag, in_sample, klo, khi,
                                                     nloc.as<unsigned long long>());
         TIGR_CKL("coo scan");
@@ -457,7 +509,8 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
 
 template <bool W>
 tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
-                         int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi) {
+                         int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi,
+                         const HostArcs* host) {
     typedef typename ValT<W>::T VT;
     const uint64_t Mall = symmetrize ? 2 * m : m;
     uint64_t M = Mall;
@@ -468,7 +521,7 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     TIGR_CK(cudaMemsetAsync(g->in_flag.p, 0, n, s));
     TIGR_CK(cudaMemsetAsync(g->in_sample.p, 0, sizeof(uint32_t) * n, s));
     TIGR_TRY(sort_arcs<W>(src, dst, w, m, Mall, n, s, keys, vals, true, g->in_flag.as<uint8_t>(),
-                          g->in_sample.as<uint32_t>(), klo, khi, &M));
+                          g->in_sample.as<uint32_t>(), klo, khi, &M, host));
     g->has_in_sketch = true;
     g->m = M;  // arcs of this build's source range (all arcs unless partitioned)
     // degrees from runs
@@ -570,9 +623,10 @@ tigr_status sort_pairs_u32(const uint32_t* keys, const uint32_t* vals, uint64_t 
 
 // Stable device CSR build from an arc list (device pointers).  Caller validated ids < n.
 tigr_status csr_build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
-                             int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi) {
-    if (w) return build_sorted<true>(n, m, src, dst, w, symmetrize, s, g, klo, khi);
-    return build_sorted<false>(n, m, src, dst, w, symmetrize, s, g, klo, khi);
+                             int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi,
+                             const HostArcs* host) {
+    if (w) return build_sorted<true>(n, m, src, dst, w, symmetrize, s, g, klo, khi, host);
+    return build_sorted<false>(n, m, src, dst, w, symmetrize, s, g, klo, khi, host);
 }
 
 }  // namespace tigr

@@ -25,6 +25,12 @@ struct Ctl {
     uint32_t queue_iters;  // iterations the queue-driven (dynamic-mapping) path ran
     uint32_t xcount;       // multi-GPU sparse exchange: records this rank packed (exchange.cu)
     unsigned long long nodes;  // sum over iterations of active nodes with arcs (queue entries)
+    // frontier bound of the iteration of parity s (frontier.cu k_compact): SSSP the minimum, SSWP
+    // the maximum value over the active nodes; every node whose value is below (SSSP) / at or
+    // above (SSWP) it is final.  bound_id = the identity (reset value, k_init / k_control)
+    uint32_t bound[2];
+    uint32_t bound_id;
+    uint32_t pad2;
 };
 
 struct GraphKey {
@@ -51,7 +57,6 @@ struct Workspace {
     DevBuf contrib;  // double[n] PR x/deg
     DevBuf acc;      // double[n] PR accumulator
     DevBuf acc2;     // double[n] second accumulator (fused apply alternates the two; pr.cu)
-    DevBuf hot;      // uint32: PR hot-destination selection {count[n], hist[33], n_hot, ids[max]}
     DevBuf cid;      // uint32[n]: PR accumulator id (in-degree order; pr.cu)
     DevBuf col_pr;   // uint32[4 * nchunks]: arc targets as accumulator ids (PR only)
     uint32_t n_in = 0;       // nodes with in-arcs (= accumulator entries ever written)
@@ -59,11 +64,11 @@ struct Workspace {
     DevBuf qv;       // uint32[2][n]: active-node queue (node ids), one slot per iteration parity
     DevBuf qo;       // uint32[2][n]: first queue-space virtual node of each entry (exclusive prefix)
     DevBuf settled;  // uint32[n/32+1]: BFS settled bitmap (frontier.cu)
-    DevBuf xlist;
-    DevBuf peers;    // FusedPeers (fused multi-GPU exchange, exchange.cu)    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
+    DevBuf xlist;    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
+    DevBuf peers;    // FusedPeers (fused multi-GPU exchange, exchange.cu)
     DevBuf ctl;      // Ctl
-    Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (thread-local, not owned)
-    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    Ctl* ctl_host = nullptr;  // pinned mirror for the host loop (owned: pinned_ctl_acquire, run.cu)
+    cudaEvent_t ev[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
     std::vector<cudaEvent_t> tev;  // per-relax-launch timing events (time_kernels)
     std::map<GraphKey, CachedGraph> graphs;
     ~Workspace();
@@ -81,6 +86,7 @@ struct tigr_vgraph {
     tigr::DevBuf vn_phys;        // uint32[nv]
     tigr::DevBuf vinfo;          // uint4[n] = {chunk base, degree, first vnode, family size}
     uint32_t lo = 0, hi = 0;     // this rank's vnode range
+    uint64_t n_out = 0;          // nodes with out-arcs whose virtual nodes lie in [lo, hi)
     double ms_build = 0.0;
     tigr::Workspace ws;
 };

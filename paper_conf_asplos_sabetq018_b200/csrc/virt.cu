@@ -35,12 +35,20 @@ __global__ void k_emit(const uint32_t* __restrict__ vptr, uint32_t n, uint32_t* 
     }
 }
 
+// also counts the nodes with out-arcs (the byte model's "active physical vertex with d > 0")
 __global__ void k_vinfo(const uint32_t* __restrict__ cptr, const uint32_t* __restrict__ deg,
-                        const uint32_t* __restrict__ vptr, uint32_t n, uint4* __restrict__ vinfo) {
+                        const uint32_t* __restrict__ vptr, uint32_t n, uint4* __restrict__ vinfo,
+                        unsigned long long* __restrict__ n_out) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
-    if (v >= n) return;
-    const uint32_t b = vptr[v];
-    vinfo[v] = make_uint4(cptr[v], deg[v], b, vptr[v + 1] - b);
+    bool out = false;
+    if (v < n) {
+        const uint32_t b = vptr[v];
+        const uint32_t d = deg[v];
+        vinfo[v] = make_uint4(cptr[v], d, b, vptr[v + 1] - b);
+        out = d != 0;
+    }
+    const int c = __syncthreads_count(out);
+    if (threadIdx.x == 0 && c) atomicAdd(n_out, (unsigned long long)c);
 }
 
 }  // namespace
@@ -75,12 +83,19 @@ tigr_status virtualize_device(const tigr_graph* g, uint32_t K, tigr_layout layou
     if ((st = vg->vinfo.alloc(sizeof(uint4) * (g->n ? g->n : 1), s))) return bail(st);
     k_emit<<<grid_for(g->n), kBlock, 0, s>>>(vg->vnode_ptr.as<uint32_t>(), g->n, vg->vn_phys.as<uint32_t>());
     count_launch();
+    TmpBuf cnt;
+    if ((st = cnt.alloc(sizeof(unsigned long long), s))) return bail(st);
+    cudaMemsetAsync(cnt.p, 0, sizeof(unsigned long long), s);
     k_vinfo<<<grid_for(g->n), kBlock, 0, s>>>(g->cptr.as<uint32_t>(), g->deg.as<uint32_t>(),
-                                               vg->vnode_ptr.as<uint32_t>(), g->n, vg->vinfo.as<uint4>());
+                                               vg->vnode_ptr.as<uint32_t>(), g->n, vg->vinfo.as<uint4>(),
+                                               cnt.as<unsigned long long>());
     count_launch();
+    unsigned long long n_out = 0;
+    cudaMemcpyAsync(&n_out, cnt.p, sizeof(n_out), cudaMemcpyDeviceToHost, s);
     cudaEventRecord(e1, s);
     cudaError_t e = cudaEventSynchronize(e1);
     if (e != cudaSuccess) return bail(cuda_fail(e, "virtualize", __FILE__, __LINE__));
+    vg->n_out = n_out;
     float ms = 0.f;
     cudaEventElapsedTime(&ms, e0, e1);
     cudaEventDestroy(e0);

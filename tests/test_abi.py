@@ -78,12 +78,14 @@ def test_opts_default_and_version():
     exe = os.path.join(ROOT, "build", "abi_sizes")
     with open(src, "w") as f:
         f.write('#include <stdio.h>\n#include <stddef.h>\n#include "tigr.h"\n'
-                'int main(void){printf("%zu %zu %zu %zu\\n", sizeof(tigr_run_opts), sizeof(tigr_stats),'
-                ' offsetof(tigr_run_opts, exchange), offsetof(tigr_stats, sparse_exchanges));return 0;}\n')
+                'int main(void){printf("%zu %zu %zu %zu %zu %zu\\n", sizeof(tigr_run_opts), sizeof(tigr_stats),'
+                ' offsetof(tigr_run_opts, exchange), offsetof(tigr_stats, sparse_exchanges),'
+                ' offsetof(tigr_run_opts, frontier_div), offsetof(tigr_stats, bytes_alg));return 0;}\n')
     subprocess.run(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), src, "-o", exe], check=True)
     sizes = [int(x) for x in subprocess.run([exe], check=True, capture_output=True, text=True).stdout.split()]
     assert sizes == [ctypes.sizeof(tigr.tigr_run_opts), ctypes.sizeof(tigr.tigr_stats),
-                     tigr.tigr_run_opts.exchange.offset, tigr.tigr_stats.sparse_exchanges.offset]
+                     tigr.tigr_run_opts.exchange.offset, tigr.tigr_stats.sparse_exchanges.offset,
+                     tigr.tigr_run_opts.frontier_div.offset, tigr.tigr_stats.bytes_alg.offset]
 
 
 def _build_c_example():

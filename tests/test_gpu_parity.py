@@ -256,24 +256,23 @@ def test_edge_cases_queue(tigr, name, K, schedule):
 
 
 @pytest.mark.parametrize("layout", ["consecutive", "strided"])
-@pytest.mark.parametrize("div", ["1", "2", "1000000"])
-def test_hybrid_frontier_switch(tigr, layout, div, monkeypatch):
+@pytest.mark.parametrize("div", [1, 2, 1000000])
+def test_hybrid_frontier_switch(tigr, layout, div):
     """FRONTIER_AUTO switches between the queue and the dense sweep per iteration on the device
-    (TIGR_FQ_DIV = D: queue while the queued vnodes are < 1/D of all, so D = 1 is almost always
+    (frontier_div = D: queue while the queued vnodes are < 1/D of all, so D = 1 is almost always
     the queue and D = 1e6 almost always the dense sweep): every switch point gives the oracle's
     values and BSP iteration counts."""
-    monkeypatch.setenv("TIGR_FQ_DIV", div)
     rec = graphgen.recipe("cfg1")
     src, dst, w = graphgen.generate(rec)
     want = _oracle_all(rec.n, src, dst, w)
     for K in (4, 8, 32):
-        _assert_parity(_run_all(tigr, rec.n, src, dst, w, K, layout), want)
+        _assert_parity(_run_all(tigr, rec.n, src, dst, w, K, layout, frontier_div=div), want)
     o = oracle.csr_build(rec.n, src, dst, w)
     g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
     vg = tigr.tigr_virtualize(g, 8, layout)
     for algo, code in (("bfs", oracle.BFS), ("sssp", oracle.SSSP), ("sswp", oracle.SSWP)):
         _, want_it, _ = oracle.push_virtual(o, oracle.Virtual(o, 8), code, 0, schedule=1, worklist=1)
-        vals, st = tigr.tigr_run(vg, algo, 0, schedule=1, return_stats=True)
+        vals, st = tigr.tigr_run(vg, algo, 0, schedule=1, return_stats=True, frontier_div=div)
         assert np.array_equal(vals, want[algo]) and st["iterations"] == want_it, (algo, st["iterations"], want_it)
 
 
@@ -317,22 +316,22 @@ def test_pr_dangling_redistribute(tigr):
     assert abs(got.sum() - 1.0) < 1e-9  # redistribute conserves mass
 
 
-@pytest.mark.parametrize("fuse", ["0", "1"])
-def test_pr_iteration_counts_and_fused_apply(tigr, fuse, monkeypatch):
+@pytest.mark.parametrize("dangling", [0, 1])
+def test_pr_iteration_counts_and_fused_apply(tigr, dangling):
     """PageRank after 0, 1, 2, 3 and 20 iterations, with the apply fused into the relax
-    (default) and separate (TIGR_PR_FUSE=0): the two accumulators alternate correctly and x is
-    materialised after the last iteration; damping 0.5 and 1.0 exercise the constants."""
-    monkeypatch.setenv("TIGR_PR_FUSE", fuse)
+    (pr_dangling = 0, the default) and as a separate pass (pr_dangling = 1 needs it): the two
+    accumulators alternate correctly and x is materialised after the last iteration; damping
+    0.5 and 1.0 exercise the constants."""
     rec = graphgen.recipe("cfg1")
     src, dst, _ = graphgen.generate(rec)
     o = oracle.csr_build(rec.n, src, dst)
     vg = tigr.tigr_virtualize(tigr.tigr_graph_from_coo(rec.n, src, dst, None), 8)
     for iters in (0, 1, 2, 3, 20):
-        got = tigr.tigr_run(vg, "pr", pr_iters=iters)
-        assert np.abs(got - oracle.pagerank(o, iters)).max() <= 1e-15, iters
+        got = tigr.tigr_run(vg, "pr", pr_iters=iters, pr_dangling=dangling)
+        assert np.abs(got - oracle.pagerank(o, iters, 0.85, dangling)).max() <= 1e-15, iters
     for d in (0.5, 1.0):
-        got = tigr.tigr_run(vg, "pr", pr_iters=7, pr_damping=d)
-        assert np.abs(got - oracle.pagerank(o, 7, d)).max() <= 1e-15, d
+        got = tigr.tigr_run(vg, "pr", pr_iters=7, pr_damping=d, pr_dangling=dangling)
+        assert np.abs(got - oracle.pagerank(o, 7, d, dangling)).max() <= 1e-15, d
 
 
 def test_errors(tigr):

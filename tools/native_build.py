@@ -44,14 +44,17 @@ def _nccl_include() -> list[str]:
     return []
 
 
-def build_tigr(force: bool = False, verbose: bool = False) -> str:
-    """nvcc -gencode arch=compute_100a,code=sm_100a every csrc/*.cu -> libtigr.so (in-tree)."""
+def build_tigr(force: bool = False, verbose: bool = False, dev: bool = False) -> str:
+    """nvcc -gencode arch=compute_100a,code=sm_100a every csrc/*.cu -> libtigr.so (in-tree).
+
+    dev=True builds build/libtigr_dev.so with -DTIGR_DEV_KNOBS (the TIGR_* development knobs of
+    DESIGN.md §10c read from the environment; load it with TIGR_LIB for A/B sweeps)."""
     from concurrent.futures import ThreadPoolExecutor
 
     pkg = os.path.join(ROOT, "paper_conf_asplos_sabetq018_b200")
     csrc = os.path.join(pkg, "csrc")
-    target = os.path.join(pkg, "libtigr.so")
-    objdir = os.path.join(ROOT, "build", "obj")
+    target = os.path.join(ROOT, "build", "libtigr_dev.so") if dev else os.path.join(pkg, "libtigr.so")
+    objdir = os.path.join(ROOT, "build", "obj_dev" if dev else "obj")
     os.makedirs(objdir, exist_ok=True)
     sources = sorted(os.path.join(csrc, f) for f in os.listdir(csrc) if f.endswith(".cu"))
     headers = sorted(os.path.join(csrc, f) for f in os.listdir(csrc) if f.endswith((".cuh", ".h")))
@@ -59,6 +62,8 @@ def build_tigr(force: bool = False, verbose: bool = False) -> str:
     flags = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-Wall",
              "--expt-relaxed-constexpr", "--extended-lambda", *ARCH, "-I", os.path.join(ROOT, "include"),
              *_nccl_include()]
+    if dev:
+        flags += ["-DTIGR_DEV_KNOBS"]
     if os.environ.get("TIGR_PTXAS_VERBOSE"):
         flags += ["-Xptxas", "-v"]
 
@@ -80,8 +85,23 @@ def build_tigr(force: bool = False, verbose: bool = False) -> str:
     return target
 
 
+def build_micro(force: bool = False) -> str:
+    """tools/micro/gather_ceiling.cu -> build/libmicro.so (measurement helper bench.py loads;
+    not part of the product library)."""
+    src = os.path.join(ROOT, "tools", "micro", "gather_ceiling.cu")
+    target = os.path.join(ROOT, "build", "libmicro.so")
+    os.makedirs(os.path.dirname(target), exist_ok=True)
+    if force or _stale(target, [src]):
+        subprocess.run([NVCC, "-O3", "-lineinfo", *ARCH, "-Xcompiler", "-fPIC", "-shared", src, "-o", target + ".tmp"],
+                       check=True)
+        os.replace(target + ".tmp", target)
+    return target
+
+
 if __name__ == "__main__":
     sys.path.insert(0, ROOT)
     import __graft_entry__  # noqa: E402
 
     __graft_entry__.build()
+    if "--dev" in sys.argv:
+        build_tigr(dev=True)
