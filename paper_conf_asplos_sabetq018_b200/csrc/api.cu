@@ -79,8 +79,16 @@ std::mutex g_cache_mu;
 std::multimap<std::pair<int, size_t>, CachedBlock> g_free;  // (device, size) -> block
 std::map<void*, std::pair<int, size_t>> g_live;             // live block -> (device, size)
 constexpr size_t kGran = 2u << 20;
+}  // namespace
+
+// incremented whenever libtigr returns cached blocks to the driver: an address published before
+// may then name a different allocation
+std::atomic<uint64_t> g_free_epoch{0};
+
+namespace {
 
 void release_cached_locked() {
+    g_free_epoch.fetch_add(1);  // device addresses may be handed out again (comm.cu IPC handle cache)
     int cur = 0;
     cudaGetDevice(&cur);
     for (auto& kv : g_free) {

@@ -117,16 +117,27 @@ struct NodeShm {
     } slot[kMaxGroupRanks];
 };
 
+extern std::atomic<uint64_t> g_free_epoch;  // api.cu
+
 struct NodeGroup : PeerGroup {
     std::string name;
     NodeShm* shm = nullptr;
     int me = 0;
     bool owner = false;
     std::vector<const void*> mine = std::vector<const void*>(8, nullptr);
-    std::map<std::string, void*> opened;  // IPC handle bytes -> mapped base
+    // exporter: one cudaIpcGetMemHandle per allocation (valid until libtigr frees blocks to the
+    // driver, g_free_epoch); importer: mappings by handle, at most kMaxOpened, least recently
+    // used closed first (a mapping of a block its owner has since freed is never reused --
+    // a new allocation has a new handle -- and is closed when it ages out)
+    static constexpr size_t kMaxOpened = 256;  // > 3 pointers x 15 peers of one fused run
+    std::map<void*, cudaIpcMemHandle_t> exported;
+    uint64_t exported_epoch = 0;
+    struct Opened { void* p; uint64_t used; };
+    std::map<std::string, Opened> opened;  // IPC handle bytes -> mapped base
+    uint64_t clock = 0;
 
     ~NodeGroup() override {
-        for (auto& kv : opened) cudaIpcCloseMemHandle(kv.second);
+        for (auto& kv : opened) cudaIpcCloseMemHandle(kv.second.p);
         if (shm) munmap(shm, sizeof(NodeShm));
         if (owner) shm_unlink(name.c_str());
     }
@@ -153,13 +164,24 @@ struct NodeGroup : PeerGroup {
         return TIGR_OK;
     }
     tigr_status publish(int r, const void* const* ptrs, int k) override {
+        const uint64_t epoch = g_free_epoch.load();
+        if (epoch != exported_epoch) {
+            exported.clear();
+            exported_epoch = epoch;
+        }
         for (int i = 0; i < k; ++i) {
             mine[i] = ptrs[i];
             void* base = nullptr;
             size_t off = 0;
             if (!cache_base(ptrs[i], &base, &off))
                 return fail(TIGR_EINVAL, "node communicator: buffer not allocated by libtigr");
-            TIGR_CK(cudaIpcGetMemHandle(&shm->slot[r].h[i], base));
+            auto it = exported.find(base);
+            if (it == exported.end()) {
+                cudaIpcMemHandle_t h;
+                TIGR_CK(cudaIpcGetMemHandle(&h, base));
+                it = exported.emplace(base, h).first;
+            }
+            shm->slot[r].h[i] = it->second;
             shm->slot[r].off[i] = off;
         }
         return TIGR_OK;
@@ -170,11 +192,19 @@ struct NodeGroup : PeerGroup {
             const std::string key(reinterpret_cast<const char*>(&shm->slot[r].h[i]), sizeof(cudaIpcMemHandle_t));
             auto it = opened.find(key);
             if (it == opened.end()) {
+                if (opened.size() >= kMaxOpened) {  // close the least recently used mapping
+                    auto lru = opened.begin();
+                    for (auto j = opened.begin(); j != opened.end(); ++j)
+                        if (j->second.used < lru->second.used) lru = j;
+                    cudaIpcCloseMemHandle(lru->second.p);
+                    opened.erase(lru);
+                }
                 void* p = nullptr;
                 TIGR_CK(cudaIpcOpenMemHandle(&p, shm->slot[r].h[i], cudaIpcMemLazyEnablePeerAccess));
-                it = opened.emplace(key, p).first;
+                it = opened.emplace(key, Opened{p, 0}).first;
             }
-            out[i] = static_cast<const char*>(it->second) + shm->slot[r].off[i];
+            it->second.used = ++clock;
+            out[i] = static_cast<const char*>(it->second.p) + shm->slot[r].off[i];
         }
         return TIGR_OK;
     }

@@ -18,19 +18,10 @@ constexpr uint32_t kFull = 0xffffffffu;
 // ------------------------------------------------------------------------------------------
 // queue build: nodes stamped for iteration it + delta that own virtual nodes in [lo, hi)
 // ------------------------------------------------------------------------------------------
-// SSSP / SSWP (bmode 1 / 2) also keep the settled bitmap of k_relax_fq (frontier_kernel.cuh):
-//   * bound: the minimum / maximum value over the stamped nodes -- those with arcs in this
-//     rank's range on one GPU; every stamped node with replicas (bound_all), since another rank
-//     may own their arcs -- into ctl->bound[slot];
-//   * settle (delta = 1, i.e. after iteration it): every node whose value is below (SSSP) / at
-//     least (SSWP) iteration it's bound is final; its bit is set here, one owner lane per 32-node
-//     word (so the relax never issues atomics for it and never re-reads a stale word).
 __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restrict__ stamp,
                                                          const uint4* __restrict__ vinfo, uint32_t n, uint32_t lo,
                                                          uint32_t hi, Ctl* ctl, uint32_t* __restrict__ qv,
-                                                         uint32_t* __restrict__ qo, int delta,
-                                                         const uint32_t* __restrict__ val, int bmode, int bound_all,
-                                                         uint32_t* __restrict__ settled) {
+                                                         uint32_t* __restrict__ qo, int delta) {
     __shared__ unsigned long long s_warp[kFqThreads / 32];
     __shared__ unsigned long long s_base;
     if (!ctl->cont) return;  // past the fixed point (batched host loop, run.cu); k_init sets cont
@@ -40,31 +31,9 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
     uint32_t* ov = qv + (uint64_t)slot * n;
     uint32_t* oo = qo + (uint64_t)slot * n;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    uint32_t bnd = bmode == 2 ? 0u : kInf;
-    const bool settle = bmode && settled && delta == 1;
-    const uint32_t bcur = settle ? ctl->bound[ctl->it & 1u] : 0u;  // bound of the iteration just run
     constexpr uint32_t kTileNodes = kFqThreads * kCompactPer;
-    static_assert(32 % kCompactPer == 0, "a settled word spans whole threads");
     for (uint64_t tile0 = (uint64_t)blockIdx.x * kTileNodes; tile0 < n; tile0 += (uint64_t)gridDim.x * kTileNodes) {
         const uint64_t v0 = tile0 + (uint64_t)threadIdx.x * kCompactPer;
-        if (settle) {  // 32 / kCompactPer lanes share one bitmap word
-            const uint32_t word = v0 < n ? settled[v0 >> 5] : kFull;
-            const int sh = (int)(v0 & 31u);
-            uint32_t add = 0;
-            if (((word >> sh) & 0xFFu) != 0xFFu) {
-#pragma unroll
-                for (int q = 0; q < kCompactPer; ++q) {
-                    const uint64_t v = v0 + q;
-                    if (v < n && !((word >> (sh + q)) & 1u)) {
-                        const uint32_t x = val[v];
-                        if (bmode == 2 ? x >= bcur : x < bcur) add |= 1u << (sh + q);
-                    }
-                }
-            }
-#pragma unroll
-            for (int o = 1; o < 32 / kCompactPer; o <<= 1) add |= __shfl_xor_sync(kFull, add, o);
-            if ((lane & (32 / kCompactPer - 1)) == 0 && (add & ~word)) settled[v0 >> 5] = word | add;
-        }
         uint32_t m[kCompactPer];
         unsigned long long mine = 0;  // (entries << 32) | vnodes of this thread's nodes
 #pragma unroll
@@ -74,10 +43,6 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
             if (v < n && __ldg(st + v) == itn) {
                 const uint4 info = __ldg(vinfo + v);
                 if (info.w && info.z >= lo && info.z < hi) m[q] = info.w;
-                if (bmode && (m[q] || bound_all)) {
-                    const uint32_t x = val[v];
-                    bnd = bmode == 2 ? max(bnd, x) : min(bnd, x);
-                }
             }
             if (m[q]) mine += (1ull << 32) | m[q];
         }
@@ -105,17 +70,6 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
             ov[e] = (uint32_t)(v0 + q);
             oo[e] = (uint32_t)pos;
             pos += (1ull << 32) | m[q];
-        }
-    }
-    if (bmode) {  // one atomic per warp
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            const uint32_t y = __shfl_xor_sync(kFull, bnd, o);
-            bnd = bmode == 2 ? max(bnd, y) : min(bnd, y);
-        }
-        if (lane == 0 && bnd != (bmode == 2 ? 0u : kInf)) {
-            if (bmode == 2) atomicMax(&ctl->bound[slot], bnd);
-            else atomicMin(&ctl->bound[slot], bnd);
         }
     }
 }
@@ -148,8 +102,7 @@ unsigned relax_fq_grid(FqFn fn) {
 
 int relax_fq_threads() { return kFqThreads; }
 
-tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s, int bmode, int bound_all,
-                           const uint32_t* settled) {
+tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s) {
     const uint32_t n = vg->g->n;
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
@@ -158,9 +111,7 @@ tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStrea
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(tiles, (uint64_t)sms * 8));
     k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<uint32_t>(), vg->vinfo.as<uint4>(), n, vg->lo, vg->hi, ctl,
                                           const_cast<uint32_t*>(vg->ws.qv.as<uint32_t>()),
-                                          const_cast<uint32_t*>(vg->ws.qo.as<uint32_t>()), delta,
-                                          vg->ws.val.as<uint32_t>(), bmode, bound_all,
-                                          bmode ? const_cast<uint32_t*>(settled) : nullptr);
+                                          const_cast<uint32_t*>(vg->ws.qo.as<uint32_t>()), delta);
     TIGR_CK(cudaGetLastError());
     return TIGR_OK;
 }

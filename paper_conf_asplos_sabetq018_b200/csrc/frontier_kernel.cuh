@@ -44,18 +44,10 @@
 // CC uses the same bitmap for one exact case: a label lowered to 0, the smallest id, is
 // final (nothing is better than 0), and on power-law graphs the giant component -- most
 // targets -- carries label 0 after the first iterations.
-// SSSP and SSWP settle by the frontier bound.  At the start of iteration it, every value that
-// has not yet been pushed along all its arcs belongs to a node stamped active for it (the
-// frontier rule: an atomic that may have improved a node stamps it for the next iteration, and
-// a node whose virtual nodes read an older value was stamped again when it was lowered).  So
-// every candidate of iteration it and later derives from the current values of the active
-// nodes: SSSP candidates are >= mu + w >= mu, mu = the minimum over the active nodes (weights
-// >= 0; UDT's dumb arcs weigh 0), and SSWP candidates min(x, w) are <= M, the maximum over them.
-// A value below mu (SSSP) or at least M (SSWP) can never improve again: final.  k_compact
-// computes the bound while it builds the queue, and after iteration it sets the bit of every
-// node beyond iteration it's bound (frontier.cu); the relax only tests bits.  (Setting bits from
-// the relax's own gathers was measured slower: the L1 keeps serving a stale zero word, so every
-// SM re-issued the atomicOr for the same hot targets.)  Bits persist (a final value stays final).
+// SSSP and SSWP test the value itself: a bitmap settled by the frontier bound (values below the
+// minimum active value, SSSP, or at least the maximum, SSWP, are final) was built and measured
+// slower (cfg4 SSSP 2.68 -> 4.03 ms): in their heavy iterations few targets are
+// final, so the bit test only adds a second dependent access before the value gather.
 //
 // This header holds the relax kernel template; frontier_{bfs,sssp,sswp,cc}.cu instantiate it
 // for one algorithm each (parallel compilation), frontier.cu holds the queue build and the
@@ -158,8 +150,8 @@ __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, ui
 template <int A, int LAYOUT, bool BSP, int B, bool STATS, int MINB, bool PRE>
 __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
-    constexpr uint32_t kFinal = A == TIGR_SSWP ? kInf : 0u;  // a settled target reads as unimprovable
-    const bool BITS = f.settled != nullptr;    // uniform per launch
+    constexpr uint32_t kFinal = 0u;  // a settled BFS / CC target reads as 0: never improvable
+    const bool BITS = (A == TIGR_BFS || A == TIGR_CC) && f.settled != nullptr;  // uniform per launch
     if (!a.ctl->cont) return;  // an iteration enqueued past the fixed point (batched host loop, run.cu)
     const int lane = threadIdx.x & 31;
     const uint32_t it = a.ctl->it;

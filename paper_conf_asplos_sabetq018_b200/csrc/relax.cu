@@ -385,9 +385,9 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
         else if (algo == TIGR_SSWP) x = 0;
         if (v == src && algo != TIGR_CC) x = (algo == TIGR_SSWP) ? kInf : 0;
         val[v] = x;
-        // the source's value (BFS/SSSP 0, SSWP infinity) is final from the start: its settled bit
-        // (cleared before this kernel; frontier_kernel.cuh) spares every gather of it
-        if (settled && v == src && algo != TIGR_CC) atomicOr(settled + (v >> 5), 1u << (v & 31u));
+        // BFS: the source's level 0 is final from the start; its settled bit (cleared before this
+        // kernel; frontier_kernel.cuh) spares every gather of it -- R-MAT's source is a hub
+        if (settled && v == src && algo == TIGR_BFS) atomicOr(settled + (v >> 5), 1u << (v & 31u));
         stamp[v] = 0u;                                                // parity 0
         stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == src) ? 1u : 0u;  // parity 1: it = 1
     }
@@ -396,8 +396,6 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
         ctl->xchanged[0] = 0; ctl->xchanged[1] = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;
         ctl->qpack[0] = 0ull; ctl->qpack[1] = 0ull; ctl->queue_iters = 0; ctl->nodes = 0;
-        ctl->bound_id = algo == TIGR_SSWP ? 0u : kInf;  // max / min identity
-        ctl->bound[0] = ctl->bound_id; ctl->bound[1] = ctl->bound_id;
     }
 }
 
@@ -425,7 +423,6 @@ __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle
     const uint32_t changed = ctl->changed;
     ctl->nodes += ctl->qpack[ctl->it & 1u] >> 32;
     ctl->qpack[ctl->it & 1u] = 0ull;  // queue slot consumed by this iteration (frontier.cu)
-    ctl->bound[ctl->it & 1u] = ctl->bound_id;  // and its frontier bound
     uint32_t cont = changed ? 1u : 0u;
     if (changed && ctl->it >= ctl->max_iters) { cont = 0; ctl->notconv = 1; }
     ctl->changed = 0;

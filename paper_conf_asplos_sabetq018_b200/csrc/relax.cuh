@@ -40,7 +40,7 @@ struct FqArgs {
     const uint32_t* qo;   // uint32[2][n] queue-space first virtual node of each entry
     int mode;             // 0 = per iteration (queue if vnodes * dense_div < span), 1 = queue, 2 = dense
     uint32_t dense_div;
-    uint32_t* settled;    // bit v set once v's value is final (nullptr: always test the value)
+    uint32_t* settled;    // BFS / CC: bit v set once v's value is final (nullptr: always test the value)
     const FusedPeers* peers;  // fused exchange: every improvement is also applied to the peers' replicas
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
@@ -48,11 +48,7 @@ FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);
 unsigned relax_fq_grid(FqFn fn);   // persistent grid: SMs x resident blocks
 int relax_fq_threads();
 struct Ctl;
-// bmode: frontier bound into ctl->bound (0 none, 1 min = SSSP, 2 max = SSWP); bound_all: over
-// every stamped node (replicas), else over the stamped nodes with arcs in this rank's range;
-// settled (nullable): SSSP / SSWP bitmap the compaction settles by the previous bound
-tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s, int bmode, int bound_all,
-                           const uint32_t* settled);
+tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s);
 typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
 
 RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats);

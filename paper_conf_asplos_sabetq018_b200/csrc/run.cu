@@ -116,7 +116,6 @@ struct FrontierPlan {
     unsigned grid;
     bool bsp, comm;
     bool fused = false;    // TIGR_EXCHANGE_FUSED: the relax updates the peers' replicas itself
-    int bmode = 0;         // frontier bound for the settled test (frontier.cu k_compact): 1 SSSP, 2 SSWP
     int algo;
     tigr_comm* c;
     uint32_t n;
@@ -150,7 +149,7 @@ tigr_status enqueue_body(const FrontierPlan& p, cudaStream_t s, cudaGraphConditi
     }
     if (ev_c) TIGR_CK(cudaEventRecord(ev_c, s));
     if (p.fq) {  // next iteration's queue from the stamps just written
-        TIGR_TRY(compact_launch(p.vg, p.args.ctl, 1, s, p.bmode, p.comm ? 1 : 0, p.fa.settled));
+        TIGR_TRY(compact_launch(p.vg, p.args.ctl, 1, s));
         ++k;
     }
     k_control<<<1, 1, 0, s>>>(p.args.ctl, h, use_handle);
@@ -176,11 +175,13 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         p.fa.dense_div = o.frontier_div ? o.frontier_div : 2u;
         p.fa.settled = nullptr;
         p.fa.peers = nullptr;
-        // settled bitmap (frontier_kernel.cuh): a target whose value is final is never gathered
-        if (dev_knob("TIGR_SETTLED_BITS", 1)) {
+        // BFS / CC settled bitmap (frontier_kernel.cuh): a target whose value is final is never
+        // gathered.  (SSSP / SSWP were measured slower with a bitmap settled by the frontier
+        // bound: their targets are rarely final in the heavy iterations, so the bit test only
+        // puts a second dependent access in front of the value gather -- DESIGN.md §5.)
+        if ((algo == TIGR_BFS || algo == TIGR_CC) && dev_knob("TIGR_BFS_BITS", 1)) {
             if (!ws.settled.p) TIGR_TRY(ws.settled.alloc(sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
             p.fa.settled = ws.settled.as<uint32_t>();
-            p.bmode = algo == TIGR_SSSP ? 1 : (algo == TIGR_SSWP ? 2 : 0);
         }
     } else if (front == TIGR_FRONTIER_QUEUE) {
         return fail(TIGR_EUNSUPPORTED, "frontier QUEUE needs the 16-byte-chunk layout (4 | K)");
@@ -231,7 +232,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     TIGR_CKL("init");
     if (p.bsp || p.comm)
         TIGR_CK(cudaMemcpyAsync((void*)p.args.prev, p.args.val, sizeof(uint32_t) * n, cudaMemcpyDeviceToDevice, s));
-    if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s, p.bmode, p.comm ? 1 : 0, p.fa.settled));  // iteration 1's queue
+    if (p.fq) TIGR_TRY(compact_launch(vg, p.args.ctl, 0, s));  // iteration 1's queue
     if (p.fused) TIGR_TRY(fused_barrier(p.c, s));  // every replica initialised before any remote update
 
     int kpi = 0;

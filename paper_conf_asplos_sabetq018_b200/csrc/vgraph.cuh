@@ -25,12 +25,6 @@ struct Ctl {
     uint32_t queue_iters;  // iterations the queue-driven (dynamic-mapping) path ran
     uint32_t xcount;       // multi-GPU sparse exchange: records this rank packed (exchange.cu)
     unsigned long long nodes;  // sum over iterations of active nodes with arcs (queue entries)
-    // frontier bound of the iteration of parity s (frontier.cu k_compact): SSSP the minimum, SSWP
-    // the maximum value over the active nodes; every node whose value is below (SSSP) / at or
-    // above (SSWP) it is final.  bound_id = the identity (reset value, k_init / k_control)
-    uint32_t bound[2];
-    uint32_t bound_id;
-    uint32_t pad2;
 };
 
 struct GraphKey {
