@@ -60,9 +60,11 @@ typedef enum {
 
 /* Edge assignment of the virtual nodes of one family. */
 typedef enum {
-    TIGR_LAYOUT_CONSECUTIVE = 0, /* Fig. 10 / Alg. 2: vnode j owns segment positions [jK, (j+1)K) */
+    TIGR_LAYOUT_CONSECUTIVE = 0, /* Fig. 10 / Alg. 2: vnode j owns segment positions [jK, (j+1)K)
+                                    (whole units: the same unit rule as STRIDED) */
     TIGR_LAYOUT_STRIDED = 1      /* Fig. 12 / Alg. 3: vnode j owns units j, j+m_v, j+2m_v, ...
-                                    (unit = one 16-byte chunk of 4 edges when 4 | K, else 1 edge) */
+                                    (unit = one 32-byte span of 8 edges when 8 | K, one 16-byte
+                                    chunk of 4 edges when 4 | K, else 1 edge) */
 } tigr_layout;
 
 /* Worklist policy (§5; Table 8). */

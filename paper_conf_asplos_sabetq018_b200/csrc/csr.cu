@@ -2,9 +2,10 @@
 //
 // CSR = node array (exclusive scan of out-degrees) + edge array grouped by source
 // (Fig. 10a; "we reorder the edges during the construction of CSR",
-// L1131-1132).  B200 layout: every node's segment starts on a 16-byte boundary and is
-// padded to a multiple of 4 slots (pads = 0xFFFFFFFF), so the relax kernels can move
-// edges (and, in a separate array, weights) as 128-bit chunks; cptr[v] is the first chunk.
+// L1131-1132).  B200 layout: every node's segment starts on a 32-byte boundary and is
+// padded to a multiple of 8 slots (pads = 0xFFFFFFFF), so the relax kernels can move
+// edges (and, in a separate array, weights) as 256-bit spans or 128-bit chunks; cptr[v] is
+// the first span.
 // From an arc list the CSR is built by a stable radix sort on the source (sort.cu), so the
 // arcs of a source keep their input order: the canonical CSR, element-identical to a stable
 // counting sort.
@@ -31,9 +32,9 @@ __global__ void k_pad(const uint32_t* __restrict__ deg, const uint32_t* __restri
                       uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
     if (v >= n) return;
-    const uint64_t base = (uint64_t)cptr[v] * kChunk;
+    const uint64_t base = (uint64_t)cptr[v] * kSpan;
     const uint32_t d = deg[v];
-    const uint64_t end = (uint64_t)cptr[v + 1] * kChunk;
+    const uint64_t end = (uint64_t)cptr[v + 1] * kSpan;
     for (uint64_t s = base + d; s < end; ++s) {
         col[s] = kPad;
         if (wt) wt[s] = 0;
@@ -67,7 +68,7 @@ __global__ void k_csr_to_padded(const int64_t* __restrict__ rp, uint32_t n, uint
     for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m;
          e += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t v = owner_of(rp, n, e);
-        const uint64_t slot = (uint64_t)cptr[v] * kChunk + (e - rp[v]);
+        const uint64_t slot = (uint64_t)cptr[v] * kSpan + (e - rp[v]);
         const uint32_t c = cin[e];
         if (c >= n) *bad = 1;
         col[slot] = c;
@@ -82,7 +83,7 @@ __global__ void k_padded_to_csr(const int64_t* __restrict__ rp, uint32_t n, uint
     for (uint64_t e = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; e < m;
          e += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t v = owner_of(rp, n, e);
-        const uint64_t slot = (uint64_t)cptr[v] * kChunk + (e - rp[v]);
+        const uint64_t slot = (uint64_t)cptr[v] * kSpan + (e - rp[v]);
         if (cout) cout[e] = col[slot];
         if (wout) wout[e] = wt[slot];
     }
@@ -137,7 +138,7 @@ __global__ void __launch_bounds__(256) k_expand_arcs(const int64_t* __restrict__
                 v = owner_of(rp, v0, v1, p);
                 beg = rp[v];
             }
-            const uint64_t c = (uint64_t)cptr[v] * kChunk + (p - (uint64_t)beg);
+            const uint64_t c = (uint64_t)cptr[v] * kSpan + (p - (uint64_t)beg);
             src[p] = v;
             dst[p] = col[c];
             if (w) w[p] = wt[c];
@@ -168,7 +169,7 @@ __global__ void k_udt_arcs(const int64_t* __restrict__ rp, const uint32_t* __res
     uint64_t beg = 0, cb = 0;
     uint32_t d = 0, tb = 0, t = 0;
     if (v < n) {
-        beg = (uint64_t)rp[v]; d = (uint32_t)(rp[v + 1] - rp[v]); cb = (uint64_t)cptr[v] * kChunk;
+        beg = (uint64_t)rp[v]; d = (uint32_t)(rp[v + 1] - rp[v]); cb = (uint64_t)cptr[v] * kSpan;
         tb = tptr[v]; t = tptr[v + 1] - tb;
     }
     auto parent = [&](uint32_t vv, uint64_t p, uint32_t tt, uint32_t tbb) -> uint32_t {
@@ -224,9 +225,10 @@ tigr_status layout_from_degrees(tigr_graph* g, cudaStream_t s) {
                                 reinterpret_cast<uint64_t*>(g->row_ptr.p), s));
     TIGR_TRY(g->cptr.alloc(sizeof(uint32_t) * ((size_t)g->n + 1), s));
     uint64_t nch = 0;
-    TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), g->n, SCAN_CEIL_DIV, kChunk, g->cptr.as<uint32_t>(),
+    TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), g->n, SCAN_CEIL_DIV, kSpan, g->cptr.as<uint32_t>(),
                                 s, &nch));
-    if (nch >= (1ull << 32)) return fail(TIGR_ERANGE, "graph: padded edge chunks exceed 2^32");
+    if (nch >= (1ull << 31)) return fail(TIGR_ERANGE, "graph: padded edge spans exceed 2^31");
+    nch *= 2;  // 16-byte chunks
     g->nchunks = nch;
     TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));
     if (g->weighted) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));

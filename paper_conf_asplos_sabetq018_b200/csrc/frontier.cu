@@ -78,17 +78,17 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
 // dispatch
 // ------------------------------------------------------------------------------------------
 
-FqFn relax_fq_kernel_bfs(int layout, bool bsp, bool stats);
-FqFn relax_fq_kernel_sssp(int layout, bool bsp, bool stats);
-FqFn relax_fq_kernel_sswp(int layout, bool bsp, bool stats);
-FqFn relax_fq_kernel_cc(int layout, bool bsp, bool stats);
+FqFn relax_fq_kernel_bfs(int layout, int unit, bool bsp, bool stats);
+FqFn relax_fq_kernel_sssp(int layout, int unit, bool bsp, bool stats);
+FqFn relax_fq_kernel_sswp(int layout, int unit, bool bsp, bool stats);
+FqFn relax_fq_kernel_cc(int layout, int unit, bool bsp, bool stats);
 
-FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats) {
+FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats) {
     switch (algo) {
-        case TIGR_BFS: return relax_fq_kernel_bfs(layout, bsp, stats);
-        case TIGR_SSSP: return relax_fq_kernel_sssp(layout, bsp, stats);
-        case TIGR_CC: return relax_fq_kernel_cc(layout, bsp, stats);
-        case TIGR_SSWP: return relax_fq_kernel_sswp(layout, bsp, stats);
+        case TIGR_BFS: return relax_fq_kernel_bfs(layout, unit, bsp, stats);
+        case TIGR_SSSP: return relax_fq_kernel_sssp(layout, unit, bsp, stats);
+        case TIGR_CC: return relax_fq_kernel_cc(layout, unit, bsp, stats);
+        case TIGR_SSWP: return relax_fq_kernel_sswp(layout, unit, bsp, stats);
     }
     return nullptr;
 }

@@ -3,9 +3,8 @@
 
 namespace tigr {
 
-FqFn relax_fq_kernel_bfs(int layout, bool bsp, bool stats) {
-    return layout == TIGR_LAYOUT_STRIDED ? pick_fq<TIGR_BFS, TIGR_LAYOUT_STRIDED>(bsp, stats)
-                                         : pick_fq<TIGR_BFS, TIGR_LAYOUT_CONSECUTIVE>(bsp, stats);
+FqFn relax_fq_kernel_bfs(int layout, int unit, bool bsp, bool stats) {
+    return pick_fq<TIGR_BFS>(layout, unit, bsp, stats);
 }
 
 }  // namespace tigr

@@ -147,7 +147,7 @@ __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, ui
 }
 
 
-template <int A, int LAYOUT, bool BSP, int B, bool STATS, int MINB, bool PRE>
+template <int A, int LAYOUT, int U, bool BSP, int B, bool STATS, int MINB, bool PRE>
 __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     constexpr uint32_t kFinal = 0u;  // a settled BFS / CC target reads as 0: never improvable
@@ -218,25 +218,13 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
         uint32_t kn[B], kend[B], step[B];
 #pragma unroll
         for (int r = 0; r < B; ++r) {
-            const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
             const uint32_t jj = queue ? j[r] : j[r] - info[r].z;  // offset within the family
             uint32_t k;
             if (!act[r]) { k = 0; step[r] = 1; kend[r] = 0; }
-            else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = jj; step[r] = info[r].w; kend[r] = q; }
-            else {
-                const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
-                k = jj * per; step[r] = 1;
-                kend[r] = (per >= q - k) ? q : k + per;
-            }
-            const uint4 pad4 = make_uint4(kPad, kPad, kPad, kPad);
-            const bool h0 = k < kend[r], h1 = k + step[r] < kend[r];
-            c0[r] = h0 ? ldg_chunk(c4 + info[r].x + k) : pad4;
-            c1[r] = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : pad4;
-            if (W) {
-                w0[r] = h0 ? ldg_chunk(w4 + info[r].x + k) : make_uint4(0, 0, 0, 0);
-                w1[r] = h1 ? ldg_chunk(w4 + info[r].x + k + step[r]) : make_uint4(0, 0, 0, 0);
-            }
-            kn[r] = k + 2 * step[r];
+            else unit_range<U, LAYOUT>(info[r].y, jj, info[r].w, a.K, k, step[r], kend[r]);
+            // the first 8 slots: one span (U = 8) or two chunks (U = 4)
+            kn[r] = load8<U>(c4, info[r].x, k, step[r], kend[r], c0[r], c1[r], make_uint4(kPad, kPad, kPad, kPad));
+            if (W) load8<U>(w4, info[r].x, k, step[r], kend[r], w0[r], w1[r], make_uint4(0, 0, 0, 0));
             if (STATS && act[r]) ++n_vn;
         }
         // settled bitmap (f.settled): the test reads one bit of an n/8-byte array instead of the
@@ -309,13 +297,12 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             }
         }
 #pragma unroll
-        for (int r = 0; r < B; ++r) {  // chunks beyond the first two (K > 8 or no split)
-            for (uint32_t k = kn[r]; k < kend[r]; k += 2 * step[r]) {
-                const bool h1 = k + step[r] < kend[r];
-                const uint4 a0 = ldg_chunk(c4 + info[r].x + k);
-                const uint4 a1 = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
-                uint4 b0 = make_uint4(0, 0, 0, 0), b1 = b0;
-                if (W) { b0 = ldg_chunk(w4 + info[r].x + k); if (h1) b1 = ldg_chunk(w4 + info[r].x + k + step[r]); }
+        for (int r = 0; r < B; ++r) {  // units beyond the first 8 slots (K > 8 or no split)
+            for (uint32_t k = kn[r]; k < kend[r];) {
+                uint4 a0, a1, b0 = make_uint4(0, 0, 0, 0), b1 = b0;
+                const uint32_t next = load8<U>(c4, info[r].x, k, step[r], kend[r], a0, a1, make_uint4(kPad, kPad, kPad, kPad));
+                if (W) load8<U>(w4, info[r].x, k, step[r], kend[r], b0, b1, make_uint4(0, 0, 0, 0));
+                k = next;
                 const uint32_t nb[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
                 const uint32_t ww[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
                 relax8(nb, ww, x[r]);
@@ -351,24 +338,31 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
 // occupancy matters more than per-thread depth.  BFS and CC (settled bitmap): see pick_fq;
 // BSP / stats variants: 4 vnodes per thread, 80 registers, 3 blocks/SM.  Weighted (SSSP, SSWP; one more 16-byte load per chunk): 2 vnodes
 // per thread with all target gathers of both issued before the first atomic, 3 blocks/SM.
-template <int A, int LAYOUT>
-FqFn pick_fq(bool bsp, bool stats) {
+template <int A, int LAYOUT, int U>
+FqFn pick_fq_u(bool bsp, bool stats) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     constexpr int B = W ? 2 : 4;
     constexpr bool PRE = W;
     if (!bsp && !stats) {  // TIGR_FQ_SHAPE: alternative shapes in development builds
-
         // BFS and CC with their settled bitmap are latency-bound rather than L1/L2-bound
         // (profiles/README.md): 2 virtual nodes per thread with all gathers issued first,
         // 4 blocks/SM (64 registers, no spills); cfg4 BFS 1.47 -> 1.34 ms, CC 3.44 -> 3.07 ms
         const int dflt = (A == TIGR_BFS || A == TIGR_CC) ? 1 : 0;
         switch (dev_knob("TIGR_FQ_SHAPE", dflt)) {
-            case 1: return &k_relax_fq<A, LAYOUT, false, 2, false, 4, true>;
+            case 1: return &k_relax_fq<A, LAYOUT, U, false, 2, false, 4, true>;
             default: break;
         }
     }
-    if (bsp) return stats ? &k_relax_fq<A, LAYOUT, true, B, true, 3, PRE> : &k_relax_fq<A, LAYOUT, true, B, false, 3, PRE>;
-    return stats ? &k_relax_fq<A, LAYOUT, false, B, true, 3, PRE> : &k_relax_fq<A, LAYOUT, false, B, false, 3, PRE>;
+    if (bsp) return stats ? &k_relax_fq<A, LAYOUT, U, true, B, true, 3, PRE> : &k_relax_fq<A, LAYOUT, U, true, B, false, 3, PRE>;
+    return stats ? &k_relax_fq<A, LAYOUT, U, false, B, true, 3, PRE> : &k_relax_fq<A, LAYOUT, U, false, B, false, 3, PRE>;
+}
+
+template <int A>
+FqFn pick_fq(int layout, int unit, bool bsp, bool stats) {
+    if (layout == TIGR_LAYOUT_STRIDED)
+        return unit == 8 ? pick_fq_u<A, TIGR_LAYOUT_STRIDED, 8>(bsp, stats) : pick_fq_u<A, TIGR_LAYOUT_STRIDED, 4>(bsp, stats);
+    return unit == 8 ? pick_fq_u<A, TIGR_LAYOUT_CONSECUTIVE, 8>(bsp, stats)
+                     : pick_fq_u<A, TIGR_LAYOUT_CONSECUTIVE, 4>(bsp, stats);
 }
 
 }  // namespace

@@ -3,9 +3,8 @@
 
 namespace tigr {
 
-FqFn relax_fq_kernel_sssp(int layout, bool bsp, bool stats) {
-    return layout == TIGR_LAYOUT_STRIDED ? pick_fq<TIGR_SSSP, TIGR_LAYOUT_STRIDED>(bsp, stats)
-                                         : pick_fq<TIGR_SSSP, TIGR_LAYOUT_CONSECUTIVE>(bsp, stats);
+FqFn relax_fq_kernel_sssp(int layout, int unit, bool bsp, bool stats) {
+    return pick_fq<TIGR_SSSP>(layout, unit, bsp, stats);
 }
 
 }  // namespace tigr

@@ -14,6 +14,8 @@ namespace tigr {
 
 constexpr uint32_t kInf = 0xFFFFFFFFu;
 constexpr uint32_t kChunk = 4;          // edges per 16-byte chunk (col and weight arrays)
+constexpr uint32_t kSpan = 8;           // edges per 32-byte span: every node's segment starts on a
+                                        // span and is padded to whole spans (cptr counts spans)
 constexpr uint32_t kPad = 0xFFFFFFFFu;  // column value of padding slots
 constexpr int kBlock = 256;
 
@@ -108,12 +110,12 @@ tigr_status exclusive_scan_u32(const uint32_t* in, uint64_t count, ScanKind kind
 struct tigr_graph {
     uint32_t n = 0;
     uint64_t m = 0;          // arcs (after symmetrisation)
-    uint64_t nchunks = 0;    // 16-byte chunks per edge array (padded segments)
+    uint64_t nchunks = 0;    // 16-byte chunks per edge array (padded segments; even: 2 per span)
     bool weighted = false;
     bool symmetric = false;
     tigr::DevBuf row_ptr;    // int64[n+1], canonical offsets
     tigr::DevBuf deg;        // uint32[n]
-    tigr::DevBuf cptr;       // uint32[n+1], first chunk of each node's segment
+    tigr::DevBuf cptr;       // uint32[n+1], first 32-byte span of each node's segment
     tigr::DevBuf col;        // uint32[4 * nchunks], padded segments, pads = 0xFFFFFFFF
     tigr::DevBuf wt;         // uint32[4 * nchunks] or empty
     // in-degree sketch from the arc-list scan (PageRank accumulator order, pr.cu)

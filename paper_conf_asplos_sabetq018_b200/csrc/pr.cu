@@ -87,7 +87,7 @@ __global__ void k_build_col_pr(const uint4* __restrict__ c4, uint64_t nchunks, c
 // x/deg_v, the apply's exact arithmetic (no FMA) -- so the separate apply pass disappears;
 // x is materialised once, after the last iteration.  mode 0: read contrib[v] (unfused);
 // 1: first iteration, x = x0; 2: from acc_prev.
-template <int LAYOUT, int B, int T, int SLOTS, int MINB>
+template <int LAYOUT, int U, int B, int T, int SLOTS, int MINB>
 __global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uint32_t* __restrict__ col_pr,
                                                                    uint32_t tiles, PrFuse fz) {
     extern __shared__ __align__(16) double s_acc[];  // SLOTS entries (dynamic: 64 KB)
@@ -139,19 +139,10 @@ __global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uin
 #pragma unroll
         for (int r = 0; r < B; ++r) {
             const uint64_t i = base + (uint64_t)r * T;
-            const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
             uint32_t k;
             if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
-            else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
-            else {
-                const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
-                k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
-                kend[r] = (per >= q - k) ? q : k + per;
-            }
-            const uint4* cb = c4 + info[r].x;
-            c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
-            c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
-            kn[r] = k + 2 * step[r];
+            else unit_range<U, LAYOUT>(info[r].y, (uint32_t)(i - info[r].z), info[r].w, a.K, k, step[r], kend[r]);
+            kn[r] = load8<U>(c4, info[r].x, k, step[r], kend[r], c0[r], c1[r], make_uint4(kPad, kPad, kPad, kPad));
         }
 #pragma unroll
         for (int r = 0; r < B; ++r) {
@@ -161,13 +152,13 @@ __global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uin
                 if (nb[q] != kPad) push(nb[q], x[r]);
         }
 #pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint4* cb = c4 + info[r].x;
-            for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
-                const uint4 c = ldg_chunk(cb + k);
-                const uint32_t nb[4] = {c.x, c.y, c.z, c.w};
+        for (int r = 0; r < B; ++r) {  // units beyond the first 8 slots (K > 8 or no split)
+            for (uint32_t k = kn[r]; k < kend[r];) {
+                uint4 c, d;
+                k = load8<U>(c4, info[r].x, k, step[r], kend[r], c, d, make_uint4(kPad, kPad, kPad, kPad));
+                const uint32_t nb[8] = {c.x, c.y, c.z, c.w, d.x, d.y, d.z, d.w};
 #pragma unroll
-                for (int q = 0; q < 4; ++q)
+                for (int q = 0; q < 8; ++q)
                     if (nb[q] != kPad) push(nb[q], x[r]);
             }
         }
@@ -315,10 +306,14 @@ tigr_status pr_pull_prepare(tigr_vgraph* vg, cudaStream_t s) {
 }
 
 template <int B, int T, int SLOTS, int MINB>
-static void fill_plan(PrCidPlan& p, int layout) {
+static void fill_plan(PrCidPlan& p, int layout, int unit) {
     static_assert(B >= 1, "");
-    p.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, B, T, SLOTS, MINB>
-                                         : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, B, T, SLOTS, MINB>;
+    if (unit == 8)
+        p.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, 8, B, T, SLOTS, MINB>
+                                             : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, 8, B, T, SLOTS, MINB>;
+    else
+        p.fn = layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_cid<TIGR_LAYOUT_STRIDED, 4, B, T, SLOTS, MINB>
+                                             : &k_relax_pr_cid<TIGR_LAYOUT_CONSECUTIVE, 4, B, T, SLOTS, MINB>;
     p.threads = T;
     p.per_thread = B;
     p.smem = sizeof(double) * SLOTS;
@@ -332,10 +327,10 @@ static void fill_plan(PrCidPlan& p, int layout) {
 PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
     PrCidPlan p;
     switch (dev_knob("TIGR_PR_CFG", 5)) {
-        case 0: fill_plan<4, 256, 8192, 2>(p, vg->layout); break;
-        case 1: fill_plan<4, 512, 24576, 1>(p, vg->layout); break;
-        case 6: fill_plan<4, 768, 28672, 1>(p, vg->layout); break;
-        default: fill_plan<4, 768, 24576, 1>(p, vg->layout); break;
+        case 0: fill_plan<4, 256, 8192, 2>(p, vg->layout, (int)vg->unit); break;
+        case 1: fill_plan<4, 512, 24576, 1>(p, vg->layout, (int)vg->unit); break;
+        case 6: fill_plan<4, 768, 28672, 1>(p, vg->layout, (int)vg->unit); break;
+        default: fill_plan<4, 768, 24576, 1>(p, vg->layout, (int)vg->unit); break;
     }
     cudaFuncSetAttribute(p.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
     int per_sm = 0, dev = 0, sms = 148;
@@ -376,7 +371,7 @@ tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangl
 namespace tigr {
 namespace {
 
-template <int LAYOUT, int B>
+template <int LAYOUT, int U, int B>
 __global__ void __launch_bounds__(256) k_relax_pr_pull(RelaxArgs a) {
     const int lane = threadIdx.x & 31;
     const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * 256) + threadIdx.x;
@@ -395,19 +390,10 @@ __global__ void __launch_bounds__(256) k_relax_pr_pull(RelaxArgs a) {
 #pragma unroll
     for (int r = 0; r < B; ++r) {
         const uint64_t i = base + (uint64_t)r * 256;
-        const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
         uint32_t k;
         if (v[r] == kPad) { k = 0; step[r] = 1; kend[r] = 0; }
-        else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
-        else {
-            const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
-            k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
-            kend[r] = (per >= q - k) ? q : k + per;
-        }
-        const uint4* cb = c4 + info[r].x;
-        c0[r] = k < kend[r] ? ldg_chunk(cb + k) : make_uint4(kPad, kPad, kPad, kPad);
-        c1[r] = k + step[r] < kend[r] ? ldg_chunk(cb + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
-        kn[r] = k + 2 * step[r];
+        else unit_range<U, LAYOUT>(info[r].y, (uint32_t)(i - info[r].z), info[r].w, a.K, k, step[r], kend[r]);
+        kn[r] = load8<U>(c4, info[r].x, k, step[r], kend[r], c0[r], c1[r], make_uint4(kPad, kPad, kPad, kPad));
     }
     double part[B];
 #pragma unroll
@@ -419,11 +405,12 @@ __global__ void __launch_bounds__(256) k_relax_pr_pull(RelaxArgs a) {
         double s = 0.0;
 #pragma unroll
         for (int q = 0; q < 8; ++q) s += g[q];
-        const uint4* cb = c4 + info[r].x;
-        for (uint32_t k = kn[r]; k < kend[r]; k += step[r]) {
-            const uint4 c = ldg_chunk(cb + k);
-            s += (c.x != kPad ? __ldg(a.contrib + c.x) : 0.0) + (c.y != kPad ? __ldg(a.contrib + c.y) : 0.0) +
-                 (c.z != kPad ? __ldg(a.contrib + c.z) : 0.0) + (c.w != kPad ? __ldg(a.contrib + c.w) : 0.0);
+        for (uint32_t k = kn[r]; k < kend[r];) {  // units beyond the first 8 slots
+            uint4 c, d;
+            k = load8<U>(c4, info[r].x, k, step[r], kend[r], c, d, make_uint4(kPad, kPad, kPad, kPad));
+            const uint32_t nb2[8] = {c.x, c.y, c.z, c.w, d.x, d.y, d.z, d.w};
+#pragma unroll
+            for (int q = 0; q < 8; ++q) s += nb2[q] != kPad ? __ldg(a.contrib + nb2[q]) : 0.0;
         }
         part[r] = s;
     }
@@ -453,10 +440,13 @@ __global__ void __launch_bounds__(256) k_relax_pr_pull(RelaxArgs a) {
 
 }  // namespace
 
-RelaxFn relax_pr_pull_kernel(int layout, int* per_thread) {
+RelaxFn relax_pr_pull_kernel(int layout, int unit, int* per_thread) {
     *per_thread = 4;
-    return layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_pull<TIGR_LAYOUT_STRIDED, 4>
-                                         : &k_relax_pr_pull<TIGR_LAYOUT_CONSECUTIVE, 4>;
+    if (unit == 8)
+        return layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_pull<TIGR_LAYOUT_STRIDED, 8, 4>
+                                             : &k_relax_pr_pull<TIGR_LAYOUT_CONSECUTIVE, 8, 4>;
+    return layout == TIGR_LAYOUT_STRIDED ? &k_relax_pr_pull<TIGR_LAYOUT_STRIDED, 4, 4>
+                                         : &k_relax_pr_pull<TIGR_LAYOUT_CONSECUTIVE, 4, 4>;
 }
 
 }  // namespace tigr

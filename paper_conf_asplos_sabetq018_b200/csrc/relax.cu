@@ -26,28 +26,22 @@ namespace tigr {
 // ------------------------------------------------------------------------------------------
 // edge walk: the set of (nbr, w) slots a virtual node owns, in the layout's order
 // ------------------------------------------------------------------------------------------
-// Calls f(nbr[8], w[8]) on batches of up to 8 slots (pads/absent = kPad).
-template <int LAYOUT, bool VEC, bool W, class F>
+// Calls f(nbr[8], w[8]) on batches of up to 8 slots (pads/absent = kPad).  U: arcs per
+// assignment unit -- 8 (32-byte span), 4 (16-byte chunk) or 1 (one arc; 4 does not divide K).
+template <int LAYOUT, int U, bool W, class F>
 __device__ __forceinline__ void walk(const uint32_t* __restrict__ col, const uint32_t* __restrict__ wt,
                                      uint32_t cbase, uint32_t d, uint32_t j, uint32_t mv, uint32_t K, F&& f) {
     uint32_t nb[8], ww[8];
-    if (VEC) {
-        const uint4* c4 = reinterpret_cast<const uint4*>(col) + cbase;
-        const uint4* w4 = reinterpret_cast<const uint4*>(wt) + cbase;
-        const uint32_t q = (d + kChunk - 1) / kChunk;  // chunks of this node
+    if (U > 1) {
+        const uint4* c4 = reinterpret_cast<const uint4*>(col);
+        const uint4* w4 = reinterpret_cast<const uint4*>(wt);
         uint32_t k, step, kend;
-        if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = j; step = mv; kend = q; }
-        else {
-            const uint32_t per = (K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : K / kChunk;
-            k = j * per; step = 1;
-            kend = (per >= q - k) ? q : k + per;
-        }
-        for (; k < kend; k += 2 * step) {
-            const bool has2 = k + step < kend;
-            const uint4 a = ldg_chunk(c4 + k);
-            const uint4 b = has2 ? ldg_chunk(c4 + k + step) : make_uint4(kPad, kPad, kPad, kPad);
-            uint4 wa = make_uint4(0, 0, 0, 0), wb = wa;
-            if (W) { wa = ldg_chunk(w4 + k); if (has2) wb = ldg_chunk(w4 + k + step); }
+        unit_range<(U > 1 ? U : 4), LAYOUT>(d, j, mv, K, k, step, kend);
+        while (k < kend) {
+            uint4 a, b, wa = make_uint4(0, 0, 0, 0), wb = wa;
+            const uint32_t next = load8<(U > 1 ? U : 4)>(c4, cbase, k, step, kend, a, b, make_uint4(kPad, kPad, kPad, kPad));
+            if (W) load8<(U > 1 ? U : 4)>(w4, cbase, k, step, kend, wa, wb, make_uint4(0, 0, 0, 0));
+            k = next;
             nb[0] = a.x; nb[1] = a.y; nb[2] = a.z; nb[3] = a.w;
             nb[4] = b.x; nb[5] = b.y; nb[6] = b.z; nb[7] = b.w;
             ww[0] = wa.x; ww[1] = wa.y; ww[2] = wa.z; ww[3] = wa.w;
@@ -77,7 +71,7 @@ __device__ __forceinline__ void walk(const uint32_t* __restrict__ col, const uin
 // ------------------------------------------------------------------------------------------
 // relax kernel
 // ------------------------------------------------------------------------------------------
-template <int A, int LAYOUT, bool VEC, int FRONT, bool BSP, bool STATS>
+template <int A, int LAYOUT, int U, int FRONT, bool BSP, bool STATS>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     if (!a.ctl->cont) return;  // an iteration enqueued past the fixed point (batched host loop, run.cu)
@@ -101,7 +95,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
             const uint4 info = a.vinfo[v];  // {chunk base, degree, first vnode, family size}
             const uint32_t j = (uint32_t)(i - info.z);
             if (STATS) n_vn = 1;
-            walk<LAYOUT, VEC, W>(a.col, a.wt, info.x, info.y, j, info.w, a.K,
+            walk<LAYOUT, U, W>(a.col, a.wt, info.x, info.y, j, info.w, a.K,
                                  [&](const uint32_t* nb, const uint32_t* ww) {
                 uint32_t cur[8];
 #pragma unroll
@@ -143,7 +137,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
 // stage -- vnode -> node id, activity stamp, node record + value, the first two edge (and
 // weight) chunks, the target-value gathers -- is issued for all B vnodes before the first
 // use, so a warp keeps ~8B independent loads in flight instead of one dependent chain.
-template <int A, int LAYOUT, int FRONT, bool BSP, int B>
+template <int A, int LAYOUT, int U, int FRONT, bool BSP, int B>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     if (!a.ctl->cont) return;  // past the fixed point (batched host loop)
@@ -195,24 +189,11 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
 #pragma unroll
     for (int r = 0; r < B; ++r) {
         const uint64_t i = base + (uint64_t)r * kRelaxThreads;
-        const uint32_t q = (info[r].y + kChunk - 1) / kChunk;
         uint32_t k;
         if (!act[r]) { k = 0; step[r] = 1; kend[r] = 0; }
-        else if (LAYOUT == TIGR_LAYOUT_STRIDED) { k = (uint32_t)(i - info[r].z); step[r] = info[r].w; kend[r] = q; }
-        else {
-            const uint32_t per = (a.K == 0xFFFFFFFFu) ? 0xFFFFFFFFu : a.K / kChunk;
-            k = (uint32_t)(i - info[r].z) * per; step[r] = 1;
-            kend[r] = (per >= q - k) ? q : k + per;
-        }
-        const uint4 pad4 = make_uint4(kPad, kPad, kPad, kPad);
-        const bool h0 = k < kend[r], h1 = k + step[r] < kend[r];
-        c0[r] = h0 ? ldg_chunk(c4 + info[r].x + k) : pad4;
-        c1[r] = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : pad4;
-        if (W) {
-            w0[r] = h0 ? ldg_chunk(w4 + info[r].x + k) : make_uint4(0, 0, 0, 0);
-            w1[r] = h1 ? ldg_chunk(w4 + info[r].x + k + step[r]) : make_uint4(0, 0, 0, 0);
-        }
-        kn[r] = k + 2 * step[r];
+        else unit_range<U, LAYOUT>(info[r].y, (uint32_t)(i - info[r].z), info[r].w, a.K, k, step[r], kend[r]);
+        kn[r] = load8<U>(c4, info[r].x, k, step[r], kend[r], c0[r], c1[r], make_uint4(kPad, kPad, kPad, kPad));
+        if (W) load8<U>(w4, info[r].x, k, step[r], kend[r], w0[r], w1[r], make_uint4(0, 0, 0, 0));
     }
     auto relax8 = [&](const uint32_t* nb, const uint32_t* ww, uint32_t xv) {
         uint32_t cur[8];
@@ -239,13 +220,12 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
         relax8(nb, ww, x[r]);
     }
 #pragma unroll
-    for (int r = 0; r < B; ++r) {  // chunks beyond the first two (K > 8 or no split)
-        for (uint32_t k = kn[r]; k < kend[r]; k += 2 * step[r]) {
-            const bool h1 = k + step[r] < kend[r];
-            const uint4 a0 = ldg_chunk(c4 + info[r].x + k);
-            const uint4 a1 = h1 ? ldg_chunk(c4 + info[r].x + k + step[r]) : make_uint4(kPad, kPad, kPad, kPad);
-            uint4 b0 = make_uint4(0, 0, 0, 0), b1 = b0;
-            if (W) { b0 = ldg_chunk(w4 + info[r].x + k); if (h1) b1 = ldg_chunk(w4 + info[r].x + k + step[r]); }
+    for (int r = 0; r < B; ++r) {  // units beyond the first 8 slots (K > 8 or no split)
+        for (uint32_t k = kn[r]; k < kend[r];) {
+            uint4 a0, a1, b0 = make_uint4(0, 0, 0, 0), b1 = b0;
+            const uint32_t next = load8<U>(c4, info[r].x, k, step[r], kend[r], a0, a1, make_uint4(kPad, kPad, kPad, kPad));
+            if (W) load8<U>(w4, info[r].x, k, step[r], kend[r], b0, b1, make_uint4(0, 0, 0, 0));
+            k = next;
             const uint32_t nb[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
             const uint32_t ww[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
             relax8(nb, ww, x[r]);
@@ -254,35 +234,38 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
     if (__any_sync(0xffffffffu, touched) && (threadIdx.x & 31) == 0) a.ctl->changed = 1;
 }
 
-template <int A, int LAYOUT>
-static RelaxFn pick_mlp(int front, bool bsp, int B) {
-#define TIGR_MLP(F, BS, BB) if (front == F && bsp == BS && B == BB) return &k_relax_mlp<A, LAYOUT, F, BS, BB>;
-    TIGR_MLP(TIGR_FRONTIER_DENSE, false, 4) TIGR_MLP(TIGR_FRONTIER_DENSE, true, 4)
-    TIGR_MLP(TIGR_FRONTIER_NONE, false, 4) TIGR_MLP(TIGR_FRONTIER_NONE, true, 4)
+template <int A, int LAYOUT, int U>
+static RelaxFn pick_mlp(int front, bool bsp) {
+#define TIGR_MLP(F, BS) if (front == F && bsp == BS) return &k_relax_mlp<A, LAYOUT, U, F, BS, 4>;
+    TIGR_MLP(TIGR_FRONTIER_DENSE, false) TIGR_MLP(TIGR_FRONTIER_DENSE, true)
+    TIGR_MLP(TIGR_FRONTIER_NONE, false) TIGR_MLP(TIGR_FRONTIER_NONE, true)
 #undef TIGR_MLP
     return nullptr;
 }
 
-// multi-vnode frontier kernel, or nullptr (then relax_kernel's one-vnode-per-thread kernel)
-RelaxFn relax_mlp_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats, int* per_thread) {
-    if (!vec || stats || algo == TIGR_PR) return nullptr;
-    constexpr int B = 4;  // 4 virtual nodes per thread (cfg4 sweep; the 2-per-thread shape is slower)
-    *per_thread = B;
-    const bool st = layout == TIGR_LAYOUT_STRIDED;
+template <int A>
+static RelaxFn pick_mlp_lu(int layout, int unit, int front, bool bsp) {
+    if (layout == TIGR_LAYOUT_STRIDED)
+        return unit == 8 ? pick_mlp<A, TIGR_LAYOUT_STRIDED, 8>(front, bsp) : pick_mlp<A, TIGR_LAYOUT_STRIDED, 4>(front, bsp);
+    return unit == 8 ? pick_mlp<A, TIGR_LAYOUT_CONSECUTIVE, 8>(front, bsp)
+                     : pick_mlp<A, TIGR_LAYOUT_CONSECUTIVE, 4>(front, bsp);
+}
+
+// multi-vnode frontier kernel (4 virtual nodes per thread; the 2-per-thread shape measured
+// slower), or nullptr (then relax_kernel's one-vnode-per-thread kernel)
+RelaxFn relax_mlp_kernel(int algo, int layout, int unit, int front, bool bsp, bool stats, int* per_thread) {
+    if (unit < 4 || stats || algo == TIGR_PR) return nullptr;
+    *per_thread = 4;
     switch (algo) {
-        case TIGR_BFS: return st ? pick_mlp<TIGR_BFS, TIGR_LAYOUT_STRIDED>(front, bsp, B)
-                                 : pick_mlp<TIGR_BFS, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
-        case TIGR_SSSP: return st ? pick_mlp<TIGR_SSSP, TIGR_LAYOUT_STRIDED>(front, bsp, B)
-                                  : pick_mlp<TIGR_SSSP, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
-        case TIGR_CC: return st ? pick_mlp<TIGR_CC, TIGR_LAYOUT_STRIDED>(front, bsp, B)
-                                : pick_mlp<TIGR_CC, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
-        case TIGR_SSWP: return st ? pick_mlp<TIGR_SSWP, TIGR_LAYOUT_STRIDED>(front, bsp, B)
-                                  : pick_mlp<TIGR_SSWP, TIGR_LAYOUT_CONSECUTIVE>(front, bsp, B);
+        case TIGR_BFS: return pick_mlp_lu<TIGR_BFS>(layout, unit, front, bsp);
+        case TIGR_SSSP: return pick_mlp_lu<TIGR_SSSP>(layout, unit, front, bsp);
+        case TIGR_CC: return pick_mlp_lu<TIGR_CC>(layout, unit, front, bsp);
+        case TIGR_SSWP: return pick_mlp_lu<TIGR_SSWP>(layout, unit, front, bsp);
     }
     return nullptr;
 }
 
-template <int LAYOUT, bool VEC, bool STATS>
+template <int LAYOUT, int U, bool STATS>
 __global__ void __launch_bounds__(kRelaxThreads) k_relax_pr(RelaxArgs a) {
     const uint64_t i = (uint64_t)a.lo + (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
     uint32_t n_edges = 0;
@@ -291,7 +274,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_pr(RelaxArgs a) {
         const double x = a.contrib[v];
         const uint4 info = a.vinfo[v];
         const uint32_t j = (uint32_t)(i - info.z);
-        walk<LAYOUT, VEC, false>(a.col, a.wt, info.x, info.y, j, info.w, a.K,
+        walk<LAYOUT, U, false>(a.col, a.wt, info.x, info.y, j, info.w, a.K,
                                  [&](const uint32_t* nb, const uint32_t*) {
 #pragma unroll
             for (int t = 0; t < 8; ++t) {
@@ -328,9 +311,9 @@ __global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uin
 // ------------------------------------------------------------------------------------------
 // dispatch
 // ------------------------------------------------------------------------------------------
-template <int A, int LAYOUT, bool VEC>
+template <int A, int LAYOUT, int U>
 static RelaxFn pick_front(int front, bool bsp, bool stats) {
-#define TIGR_PICK(F, B, S) if (front == F && bsp == B && stats == S) return &k_relax<A, LAYOUT, VEC, F, B, S>;
+#define TIGR_PICK(F, B, S) if (front == F && bsp == B && stats == S) return &k_relax<A, LAYOUT, U, F, B, S>;
     TIGR_PICK(TIGR_FRONTIER_DENSE, false, false)
     TIGR_PICK(TIGR_FRONTIER_DENSE, false, true)
     TIGR_PICK(TIGR_FRONTIER_DENSE, true, false)
@@ -343,27 +326,35 @@ static RelaxFn pick_front(int front, bool bsp, bool stats) {
     return nullptr;
 }
 
-template <int A>
-static RelaxFn pick_layout(int layout, bool vec, int front, bool bsp, bool stats) {
-    if (layout == TIGR_LAYOUT_STRIDED)
-        return vec ? pick_front<A, TIGR_LAYOUT_STRIDED, true>(front, bsp, stats)
-                   : pick_front<A, TIGR_LAYOUT_STRIDED, false>(front, bsp, stats);
-    return vec ? pick_front<A, TIGR_LAYOUT_CONSECUTIVE, true>(front, bsp, stats)
-               : pick_front<A, TIGR_LAYOUT_CONSECUTIVE, false>(front, bsp, stats);
+template <int A, int LAYOUT>
+static RelaxFn pick_unit(int unit, int front, bool bsp, bool stats) {
+    if (unit == 8) return pick_front<A, LAYOUT, 8>(front, bsp, stats);
+    if (unit == 4) return pick_front<A, LAYOUT, 4>(front, bsp, stats);
+    return pick_front<A, LAYOUT, 1>(front, bsp, stats);
 }
 
-RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats) {
+template <int A>
+static RelaxFn pick_layout(int layout, int unit, int front, bool bsp, bool stats) {
+    if (layout == TIGR_LAYOUT_STRIDED) return pick_unit<A, TIGR_LAYOUT_STRIDED>(unit, front, bsp, stats);
+    return pick_unit<A, TIGR_LAYOUT_CONSECUTIVE>(unit, front, bsp, stats);
+}
+
+template <int LAYOUT>
+static RelaxFn pick_pr(int unit, bool stats) {
+    if (unit == 8) return stats ? &k_relax_pr<LAYOUT, 8, true> : &k_relax_pr<LAYOUT, 8, false>;
+    if (unit == 4) return stats ? &k_relax_pr<LAYOUT, 4, true> : &k_relax_pr<LAYOUT, 4, false>;
+    return stats ? &k_relax_pr<LAYOUT, 1, true> : &k_relax_pr<LAYOUT, 1, false>;
+}
+
+RelaxFn relax_kernel(int algo, int layout, int unit, int front, bool bsp, bool stats) {
     switch (algo) {
-        case TIGR_BFS: return pick_layout<TIGR_BFS>(layout, vec, front, bsp, stats);
-        case TIGR_SSSP: return pick_layout<TIGR_SSSP>(layout, vec, front, bsp, stats);
-        case TIGR_CC: return pick_layout<TIGR_CC>(layout, vec, front, bsp, stats);
-        case TIGR_SSWP: return pick_layout<TIGR_SSWP>(layout, vec, front, bsp, stats);
+        case TIGR_BFS: return pick_layout<TIGR_BFS>(layout, unit, front, bsp, stats);
+        case TIGR_SSSP: return pick_layout<TIGR_SSSP>(layout, unit, front, bsp, stats);
+        case TIGR_CC: return pick_layout<TIGR_CC>(layout, unit, front, bsp, stats);
+        case TIGR_SSWP: return pick_layout<TIGR_SSWP>(layout, unit, front, bsp, stats);
         case TIGR_PR:
-            if (layout == TIGR_LAYOUT_STRIDED)
-                return vec ? (stats ? &k_relax_pr<TIGR_LAYOUT_STRIDED, true, true> : &k_relax_pr<TIGR_LAYOUT_STRIDED, true, false>)
-                           : (stats ? &k_relax_pr<TIGR_LAYOUT_STRIDED, false, true> : &k_relax_pr<TIGR_LAYOUT_STRIDED, false, false>);
-            return vec ? (stats ? &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, true, true> : &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, true, false>)
-                       : (stats ? &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, false, true> : &k_relax_pr<TIGR_LAYOUT_CONSECUTIVE, false, false>);
+            return layout == TIGR_LAYOUT_STRIDED ? pick_pr<TIGR_LAYOUT_STRIDED>(unit, stats)
+                                                 : pick_pr<TIGR_LAYOUT_CONSECUTIVE>(unit, stats);
     }
     return nullptr;
 }
@@ -496,7 +487,7 @@ __global__ void k_pr_apply(uint32_t n, const uint32_t* __restrict__ deg, double 
 }
 
 // per-vnode edge lists, walked with the relax kernels' own arithmetic (layout parity tests)
-template <int LAYOUT, bool VEC>
+template <int LAYOUT, int U>
 __global__ void k_assign(RelaxArgs a, const uint32_t* __restrict__ offs, uint32_t* __restrict__ counts,
                          uint32_t* __restrict__ nbr, uint32_t* __restrict__ wout, int weighted, int pass) {
     const uint64_t i = (uint64_t)blockIdx.x * kRelaxThreads + threadIdx.x;
@@ -507,7 +498,7 @@ __global__ void k_assign(RelaxArgs a, const uint32_t* __restrict__ offs, uint32_
     uint32_t c = 0;
     const uint32_t base = pass ? offs[i] : 0;
     const uint32_t* wt = weighted ? a.wt : a.col;
-    walk<LAYOUT, VEC, true>(a.col, wt, info.x, info.y, j, info.w, a.K,
+    walk<LAYOUT, U, true>(a.col, wt, info.x, info.y, j, info.w, a.K,
                             [&](const uint32_t* nb, const uint32_t* ww) {
         for (int t = 0; t < 8; ++t) {
             if (nb[t] == kPad) continue;
@@ -521,9 +512,12 @@ __global__ void k_assign(RelaxArgs a, const uint32_t* __restrict__ offs, uint32_
     if (!pass) counts[i] = c;
 }
 
-AssignFn assign_kernel(int layout, bool vec) {
-    if (layout == TIGR_LAYOUT_STRIDED) return vec ? &k_assign<TIGR_LAYOUT_STRIDED, true> : &k_assign<TIGR_LAYOUT_STRIDED, false>;
-    return vec ? &k_assign<TIGR_LAYOUT_CONSECUTIVE, true> : &k_assign<TIGR_LAYOUT_CONSECUTIVE, false>;
+AssignFn assign_kernel(int layout, int unit) {
+    if (layout == TIGR_LAYOUT_STRIDED)
+        return unit == 8 ? &k_assign<TIGR_LAYOUT_STRIDED, 8>
+                         : (unit == 4 ? &k_assign<TIGR_LAYOUT_STRIDED, 4> : &k_assign<TIGR_LAYOUT_STRIDED, 1>);
+    return unit == 8 ? &k_assign<TIGR_LAYOUT_CONSECUTIVE, 8>
+                     : (unit == 4 ? &k_assign<TIGR_LAYOUT_CONSECUTIVE, 4> : &k_assign<TIGR_LAYOUT_CONSECUTIVE, 1>);
 }
 
 }  // namespace tigr

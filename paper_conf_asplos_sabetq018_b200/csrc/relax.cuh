@@ -44,16 +44,16 @@ struct FqArgs {
     const FusedPeers* peers;  // fused exchange: every improvement is also applied to the peers' replicas
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
-FqFn relax_fq_kernel(int algo, int layout, bool bsp, bool stats);
+FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats);  // unit 4 or 8 (vgraph.cuh)
 unsigned relax_fq_grid(FqFn fn);   // persistent grid: SMs x resident blocks
 int relax_fq_threads();
 struct Ctl;
 tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s);
 typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
 
-RelaxFn relax_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats);
+RelaxFn relax_kernel(int algo, int layout, int unit, int front, bool bsp, bool stats);
 // frontier relax with *per_thread virtual nodes per thread (nullptr: use relax_kernel's)
-RelaxFn relax_mlp_kernel(int algo, int layout, bool vec, int front, bool bsp, bool stats, int* per_thread);
+RelaxFn relax_mlp_kernel(int algo, int layout, int unit, int front, bool bsp, bool stats, int* per_thread);
 // PageRank push with an in-degree-ordered accumulator (pr.cu)
 struct PrFuse {
     int mode = 0;               // 0 read contrib, 1 first iteration (x = x0), 2 from prev
@@ -68,12 +68,12 @@ struct PrCidPlan {
     int threads = 256, per_thread = 4;
     size_t smem = 0;
 };
-RelaxFn relax_pr_pull_kernel(int layout, int* per_thread);   // pull PageRank (pr.cu, NEXT-1)
+RelaxFn relax_pr_pull_kernel(int layout, int unit, int* per_thread);   // pull PageRank (pr.cu, NEXT-1)
 tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s);
 PrCidPlan pr_cid_plan(tigr_vgraph* vg);
 tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,
                          double* dsum_next, cudaStream_t s, double* acc = nullptr, bool reset = true);
-AssignFn assign_kernel(int layout, bool vec);
+AssignFn assign_kernel(int layout, int unit);
 
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
                        uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,

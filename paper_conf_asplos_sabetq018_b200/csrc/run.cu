@@ -167,7 +167,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     FrontierPlan p;
     p.vg = vg;
     if ((front == TIGR_FRONTIER_AUTO || front == TIGR_FRONTIER_QUEUE) && vg->vec) {
-        p.fq = relax_fq_kernel(algo, vg->layout, o.schedule == 1, o.collect_stats != 0);
+        p.fq = relax_fq_kernel(algo, vg->layout, (int)vg->unit, o.schedule == 1, o.collect_stats != 0);
         p.fa.qv = ws.qv.as<uint32_t>();
         p.fa.qo = ws.qo.as<uint32_t>();
         p.fa.mode = front == TIGR_FRONTIER_QUEUE ? 1 : 0;
@@ -192,7 +192,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     p.c = o.comm;
     p.algo = algo;
     p.n = n;
-    p.relax = relax_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0);
+    p.relax = relax_kernel(algo, vg->layout, (int)vg->unit, front, p.bsp, o.collect_stats != 0);
     if (!p.relax) return fail(TIGR_EUNSUPPORTED, "no relax kernel for this option combination");
     p.args = make_args(vg);
     if (p.comm) {
@@ -212,7 +212,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
                             ws.xlist.as<uint2>(), p.args.ctl};
     }
     int per_thread = 1;
-    if (RelaxFn mlp = relax_mlp_kernel(algo, vg->layout, vg->vec, front, p.bsp, o.collect_stats != 0, &per_thread))
+    if (RelaxFn mlp = relax_mlp_kernel(algo, vg->layout, (int)vg->unit, front, p.bsp, o.collect_stats != 0, &per_thread))
         p.relax = mlp;
     else
         per_thread = 1;
@@ -241,7 +241,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     // NCCL inside a conditional body graph is not relied on: multi-GPU runs use the host loop
     const bool use_graph = o.use_graph && !o.time_kernels && !p.comm;
     if (use_graph) {
-        GraphKey key{algo, vg->layout * 2 + (vg->vec ? 1 : 0),
+        GraphKey key{algo, vg->layout * 16 + (int)vg->unit,
                      p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div * 16 + (p.fa.settled ? 1 << 30 : 0) : front,
                      p.bsp ? 1 : 0, o.collect_stats ? 1 : 0, p.comm ? 1 : 0, vg->lo, vg->hi};
         auto itg = ws.graphs.find(key);
@@ -382,10 +382,10 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         if (!vg->vec || o.collect_stats)
             return fail(TIGR_EUNSUPPORTED, "pull PageRank needs 4 | K and collect_stats = 0");
         int per = 1;
-        relax = relax_pr_pull_kernel(vg->layout, &per);
+        relax = relax_pr_pull_kernel(vg->layout, (int)vg->unit, &per);
         per_block *= per;
     } else {
-        relax = relax_kernel(TIGR_PR, vg->layout, vg->vec, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
+        relax = relax_kernel(TIGR_PR, vg->layout, (int)vg->unit, TIGR_FRONTIER_NONE, false, o.collect_stats != 0);
     }
     const unsigned grid = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_block - 1) / per_block);
     const bool comm = o.comm != nullptr;
@@ -537,7 +537,7 @@ tigr_status assignment_device(const tigr_vgraph* vgc, uint32_t* counts, uint32_t
     RelaxArgs a = make_args(vg);
     a.lo = 0;
     a.hi = (uint32_t)vg->nv;
-    AssignFn f = assign_kernel(vg->layout, vg->vec);
+    AssignFn f = assign_kernel(vg->layout, (int)vg->unit);
     const unsigned grid = (unsigned)((vg->nv + kRelaxThreads - 1) / kRelaxThreads);
     TmpBuf offs;
     TIGR_TRY(offs.alloc(sizeof(uint32_t) * (vg->nv + 1), s));

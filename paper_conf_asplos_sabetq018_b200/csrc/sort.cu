@@ -9,7 +9,7 @@
 // the preceding tiles, and the tile is written back grouped by digit (coalesced runs).
 // No global atomics on the keys themselves, so the heavy skew of power-law sources (the
 // hottest vertex owns 0.14% of all arcs at scale 24) costs nothing.  Degrees come from the
-// run boundaries of the sorted keys; a final kernel places each arc into the 16-byte-aligned,
+// run boundaries of the sorted keys; a final kernel places each arc into the 32-byte-aligned,
 // padded segment of its source.
 #include <algorithm>
 #include <cstdlib>
@@ -327,7 +327,7 @@ __global__ void k_deg_from_runs(const uint32_t* __restrict__ start, const uint32
     if (v < n) deg[v] = end[v] - start[v];
 }
 
-// sorted arcs -> padded, 16-byte-aligned segments
+// sorted arcs -> padded, 32-byte-aligned segments
 template <bool W>
 __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>::T* __restrict__ val, uint64_t M,
                         const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ cptr,
@@ -343,7 +343,7 @@ __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
             x[q] = val[4 * g + q];
-            base[q] = (uint64_t)cptr[v[q]] * kChunk - (uint64_t)row_ptr[v[q]];
+            base[q] = (uint64_t)cptr[v[q]] * kSpan - (uint64_t)row_ptr[v[q]];
         }
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
@@ -355,7 +355,7 @@ __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>
     for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
          i += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t v = key[i];
-        const uint64_t pos = (uint64_t)cptr[v] * kChunk + (i - (uint64_t)row_ptr[v]);
+        const uint64_t pos = (uint64_t)cptr[v] * kSpan + (i - (uint64_t)row_ptr[v]);
         const VT x = val[i];
         col[pos] = (uint32_t)x;
         if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
@@ -543,8 +543,9 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     TIGR_TRY(exclusive_scan_u64(g->deg.as<uint32_t>(), n, SCAN_U32, 1, reinterpret_cast<uint64_t*>(g->row_ptr.p), s));
     TIGR_TRY(g->cptr.alloc(sizeof(uint32_t) * ((size_t)n + 1), s));
     uint64_t nch = 0;
-    TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), n, SCAN_CEIL_DIV, kChunk, g->cptr.as<uint32_t>(), s, &nch));
-    if (nch >= (1ull << 32)) return fail(TIGR_ERANGE, "graph: padded edge chunks exceed 2^32");
+    TIGR_TRY(exclusive_scan_u32(g->deg.as<uint32_t>(), n, SCAN_CEIL_DIV, kSpan, g->cptr.as<uint32_t>(), s, &nch));
+    if (nch >= (1ull << 31)) return fail(TIGR_ERANGE, "graph: padded edge spans exceed 2^31");
+    nch *= 2;  // 16-byte chunks
     g->nchunks = nch;
     trace(s, "csr: deg+scans");
     TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (nch ? nch : 1), s));

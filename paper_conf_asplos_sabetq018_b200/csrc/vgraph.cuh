@@ -74,11 +74,13 @@ struct tigr_vgraph {
     const tigr_graph* g = nullptr;
     uint32_t K = 8;
     tigr_layout layout = TIGR_LAYOUT_STRIDED;
-    bool vec = true;             // 16-byte chunk units (4 | K)
+    uint32_t unit = 8;           // arcs per assignment unit: 8 (32-byte span, 8 | K), 4 (16-byte chunk,
+                                 // 4 | K) or 1 (virt.cu)
+    bool vec = true;             // unit > 1: the chunked kernels (one vector load per unit)
     uint64_t nv = 0;
     tigr::DevBuf vnode_ptr;      // uint32[n+1]
     tigr::DevBuf vn_phys;        // uint32[nv]
-    tigr::DevBuf vinfo;          // uint4[n] = {chunk base, degree, first vnode, family size}
+    tigr::DevBuf vinfo;          // uint4[n] = {first 16-byte chunk, degree, first vnode, family size}
     uint32_t lo = 0, hi = 0;     // this rank's vnode range
     uint64_t n_out = 0;          // nodes with out-arcs whose virtual nodes lie in [lo, hi)
     double ms_build = 0.0;

@@ -6,7 +6,8 @@
 //                                                              (Fig. 10b physicalNodeId row, L931)
 //  a5 layout        per-node record vinfo[v] = {chunk base, d_v, vnode_ptr[v], m_v}: with it a
 //                   virtual node derives its offset j and stride m_v (Alg. 3 lines 3-4, L1163-1165)
-//                   over the 16-byte-chunked segment built by csr.cu.
+//                   over the span-aligned segment built by csr.cu; the stride unit is a 32-byte
+//                   span (8 | K), a 16-byte chunk (4 | K) or one arc.
 // The paper builds the virtual node array serially on the CPU (§6.4, Table 7,
 // L1471-1474); here it is three kernels plus the scan.
 #include "internal.cuh"
@@ -44,7 +45,7 @@ __global__ void k_vinfo(const uint32_t* __restrict__ cptr, const uint32_t* __res
     if (v < n) {
         const uint32_t b = vptr[v];
         const uint32_t d = deg[v];
-        vinfo[v] = make_uint4(cptr[v], d, b, vptr[v + 1] - b);
+        vinfo[v] = make_uint4(2 * cptr[v], d, b, vptr[v + 1] - b);  // .x: first 16-byte chunk
         out = d != 0;
     }
     const int c = __syncthreads_count(out);
@@ -63,8 +64,10 @@ tigr_status virtualize_device(const tigr_graph* g, uint32_t K, tigr_layout layou
     vg->g = g;
     vg->K = K;
     vg->layout = layout;
-    // 16-byte units need the unit to divide K so that no vnode exceeds K edges
-    vg->vec = (K % kChunk == 0) || (K == 0xFFFFFFFFu);
+    // The assignment unit: a 32-byte span of 8 arcs when 8 | K, a 16-byte chunk of
+    // 4 when 4 | K, else one arc -- the unit must divide K so that no vnode exceeds K edges
+    vg->unit = (K == 0xFFFFFFFFu || K % kSpan == 0) ? kSpan : (K % kChunk == 0 ? kChunk : 1u);
+    vg->vec = vg->unit > 1;
     cudaEvent_t e0, e1;
     cudaEventCreate(&e0);
     cudaEventCreate(&e1);

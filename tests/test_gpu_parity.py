@@ -110,7 +110,7 @@ def test_csr_from_csr_roundtrip(tigr):
 
 
 # ------------------------------------------------------------------------------------ a2-a5
-@pytest.mark.parametrize("K", [1, 3, 4, 8, 32, 0xFFFFFFFF])
+@pytest.mark.parametrize("K", [1, 3, 4, 8, 12, 32, 0xFFFFFFFF])
 @pytest.mark.parametrize("layout", ["consecutive", "strided"])
 def test_virtual_split_and_assignment(tigr, K, layout):
     rec = graphgen.recipe("cfg1")
@@ -123,8 +123,9 @@ def test_virtual_split_and_assignment(tigr, K, layout):
     ov = oracle.Virtual(o, K)
     assert np.array_equal(vp, ov.vnode_ptr.astype(np.uint32)) and np.array_equal(ph, ov.vn_phys)
     counts, nbr, ww = tigr.tigr_vgraph_assignment(vg)
-    # the unit of the layout: 16-byte chunks (4 edges) when 4 | K
-    chunk = 4 if (K % 4 == 0 or K == 0xFFFFFFFF) else 1
+    # the unit of the layout: 32-byte spans (8 edges) when 8 | K, 16-byte chunks
+    # (4 edges) when 4 | K, else one edge
+    chunk = 8 if (K % 8 == 0 or K == 0xFFFFFFFF) else (4 if K % 4 == 0 else 1)
     lay = 0 if layout == "consecutive" else 1
     want = np.array([len(ov.edges(i, lay, chunk)) for i in range(ov.nv)], dtype=np.uint32)
     assert np.array_equal(counts, want)
@@ -169,7 +170,7 @@ def _assert_parity(got, want):
     assert err <= 1e-6, err
 
 
-@pytest.mark.parametrize("K", [1, 4, 8, 32, 0xFFFFFFFF])
+@pytest.mark.parametrize("K", [1, 4, 8, 12, 32, 0xFFFFFFFF])
 @pytest.mark.parametrize("layout", ["consecutive", "strided"])
 def test_cfg1_all_algorithms(tigr, K, layout):
     rec = graphgen.recipe("cfg1")

@@ -128,7 +128,7 @@ def test_virtual_split_invariants(K):
         assert vg.nv == g.m
     if K >= deg.max():
         assert vg.nv == int((deg > 0).sum())
-    for layout, chunk in [(0, 1), (1, 1), (1, 2), (1, 4)]:
+    for layout, chunk in [(0, 1), (1, 1), (1, 2), (1, 4), (1, 8)]:
         seen = np.zeros(g.m, dtype=np.int64)
         for v in np.flatnonzero(deg):
             counts = []
@@ -146,7 +146,7 @@ def test_virtual_split_invariants(K):
 
 
 @pytest.mark.parametrize("K", [1, 2, 4, 8, 12, 32])
-@pytest.mark.parametrize("chunk", [1, 2, 4])
+@pytest.mark.parametrize("chunk", [1, 2, 4, 8])
 def test_strided_chunk_closed_form(K, chunk):
     """Strided layout with c-arc units (Fig. 12 L1141-1159 with c = 1):
     vnode j of a family of m_v owns units j, j + m_v, j + 2 m_v, ... of its segment, i.e. its
@@ -186,7 +186,7 @@ def test_thm2_virtual_push_equals_textbook(seed):
         iters = set()
         for K in (1, 3, 8, 1 << 40):
             vg = oracle.Virtual(gg, K)
-            for layout, chunk in [(0, 1), (1, 1), (1, 4)]:
+            for layout, chunk in [(0, 1), (1, 1), (1, 4), (1, 8)]:
                 for schedule in (0, 1):
                     vals, it, conv = oracle.push_virtual(gg, vg, algo, 0, layout, chunk, schedule, 1)
                     assert conv and np.array_equal(vals, ref), (algo, K, layout, schedule)
