@@ -173,12 +173,25 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     bool touched = false;
     uint32_t n_edges = 0, n_upd = 0, n_vn = 0;
-    for (uint64_t tile = warp0; tile < tiles; tile += nwarps) {
-        const uint64_t t0 = tile * kTile;
+    // Tiles go to warps in runs of kRun consecutive tiles, the runs interleaved across warps:
+    // within a run the queue entry index carries over from one tile to the next (map_round
+    // leaves it at an entry that starts at or before the next round), so the 32-ary search --
+    // a chain of dependent loads -- runs once per run, while the interleaving keeps all warps
+    // sweeping the queue front to back together.  Measured at cfg4 (profiles/r02_frontier_tiles.txt,
+    // reordered graph, ms): runs of 1 / 2 / 4 / 8 tiles: BFS 1.32 / 1.27 / 1.27 / 1.37, SSSP 2.20 /
+    // 2.15 / 2.18 / 2.27, CC 2.96 / 2.92 / 2.90 / 2.95.  One contiguous range per warp saved the
+    // most searches but raised the asynchronous schedule's redundant work (SSSP +10 % time).
+    const uint32_t kRun = f.run;  // tiles per run (2; FqArgs)
+    const uint32_t nruns = (uint32_t)((tiles + kRun - 1) / kRun);  // tiles < 2^32 / 32
+    uint32_t kq = 0;
+    for (uint32_t run = (uint32_t)warp0; run < nruns; run += (uint32_t)nwarps)
+    for (uint32_t tile = run * kRun; tile < min(run * kRun + kRun, (uint32_t)tiles); ++tile) {
+        const uint64_t t0 = (uint64_t)tile * kTile;
         uint32_t v[B], j[B];
         bool act[B];
         if (queue) {
-            uint32_t k = warp_search(qo, qn, (uint32_t)t0, lane);
+            if (tile == run * kRun) kq = warp_search(qo, qn, (uint32_t)t0, lane);
+            uint32_t k = kq;
 #pragma unroll
             for (int r = 0; r < B; ++r) {
                 const uint32_t tr = (uint32_t)t0 + 32u * r;
@@ -190,6 +203,7 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                 }
                 if (!act[r]) v[r] = kPad;
             }
+            kq = k;
         } else {
 #pragma unroll
             for (int r = 0; r < B; ++r) {

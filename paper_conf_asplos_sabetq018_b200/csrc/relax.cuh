@@ -42,6 +42,7 @@ struct FqArgs {
     uint32_t dense_div;
     uint32_t* settled;    // BFS / CC: bit v set once v's value is final (nullptr: always test the value)
     const FusedPeers* peers;  // fused exchange: every improvement is also applied to the peers' replicas
+    uint32_t run;         // queue tiles per warp run (frontier_kernel.cuh): the search runs once per run
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
 FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats);  // unit 4 or 8 (vgraph.cuh)

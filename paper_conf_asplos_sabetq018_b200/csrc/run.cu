@@ -175,6 +175,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
         p.fa.dense_div = o.frontier_div ? o.frontier_div : 2u;
         p.fa.settled = nullptr;
         p.fa.peers = nullptr;
+        p.fa.run = (uint32_t)std::max(1, dev_knob("TIGR_FQ_RUN", 2));
         // BFS / CC settled bitmap (frontier_kernel.cuh): a target whose value is final is never
         // gathered.  (SSSP / SSWP were measured slower with a bitmap settled by the frontier
         // bound: their targets are rarely final in the heavy iterations, so the bit test only

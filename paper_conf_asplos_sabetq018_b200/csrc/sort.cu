@@ -15,6 +15,7 @@
 #include <cstdlib>
 #include <map>
 #include <mutex>
+#include <type_traits>
 #include <utility>
 #include <vector>
 
@@ -60,6 +61,9 @@ __global__ void k_coo_scan(const uint32_t* __restrict__ src, const uint32_t* __r
                            unsigned long long* __restrict__ hist, uint32_t* __restrict__ maxid, uint32_t n,
                            uint8_t* __restrict__ in_flag, uint32_t* __restrict__ in_sample, uint32_t klo,
                            uint32_t khi, unsigned long long* __restrict__ n_local) {
+    // one arc per thread and step: measured faster (1.40 ms at cfg4) than 8 arcs per step with
+    // 16-byte loads (1.59 ms; 40 registers, occupancy 97 -> 65 %): the scan is bound by the
+    // shared-memory histogram atomics and the random in-flag reads, not by load latency
     __shared__ uint32_t h[4][kMaxRadix];
     for (int i = threadIdx.x; i < 4 * kMaxRadix; i += blockDim.x) (&h[0][0])[i] = 0;
     __syncthreads();
@@ -109,6 +113,18 @@ __global__ void k_digit_base(const unsigned long long* __restrict__ hist, int pa
         base[p * kMaxRadix + threadIdx.x] = tmp[threadIdx.x];
         __syncthreads();
     }
+}
+
+// look-back status words: relaxed, device-scope (the word itself carries epoch, flag and value,
+// so no other data needs ordering; volatile compiled to system-scope strong loads)
+__device__ __forceinline__ uint64_t status_load(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void status_store(uint64_t* p, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
 
 __device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
@@ -221,7 +237,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         }
         tile_cnt = s;
         const uint64_t word = (epoch << 48) | (tile == 0 ? kFlagInc : kFlagAgg) | (uint64_t)s;
-        *reinterpret_cast<volatile uint64_t*>(&status[(uint64_t)tile * kMaxRadix + t]) = word;
+        status_store(&status[(uint64_t)tile * kMaxRadix + t], word);
     }
     // tile-local digit starts: exclusive scan of tile_cnt over the digits (t < 256)
     {
@@ -252,23 +268,36 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
             s_val[lp] = s_vin[li];
         }
     }
-    // decoupled look-back for this digit (a short sleep between polls keeps the spinning
-    // blocks from flooding L2 while the predecessor tiles finish)
+    // decoupled look-back for this digit, kLook predecessor tiles per step: their status words
+    // are loaded together (independent loads in flight) and consumed newest first until an
+    // inclusive prefix is met; a predecessor that has published nothing yet is re-polled after
+    // a short sleep (keeps the spinning blocks from flooding L2).  ncu showed the one-at-a-time
+    // walk -- ~9 dependent L2 round trips per tile -- as a quarter of the pass.
     if (t < radix) {
+        constexpr int kLook = 4;
         uint64_t excl = 0;
         if (tile > 0) {
-            for (int64_t p = (int64_t)tile - 1; p >= 0; --p) {
-                const volatile uint64_t* sp = reinterpret_cast<const volatile uint64_t*>(&status[(uint64_t)p * kMaxRadix + t]);
-                uint64_t st = *sp;
-                while ((st >> 48) != epoch || (st & (3ull << 46)) == 0) {
-                    __nanosleep(64);
-                    st = *sp;
+            int64_t p = (int64_t)tile - 1;
+            bool done = false;
+            while (!done && p >= 0) {
+                uint64_t st[kLook];
+#pragma unroll
+                for (int q = 0; q < kLook; ++q)
+                    st[q] = (p - q >= 0) ? status_load(&status[(uint64_t)(p - q) * kMaxRadix + t]) : 0ull;
+#pragma unroll
+                for (int q = 0; q < kLook; ++q) {
+                    if (done || p - q < 0) continue;
+                    const uint64_t* sp = &status[(uint64_t)(p - q) * kMaxRadix + t];
+                    while ((st[q] >> 48) != epoch || (st[q] & (3ull << 46)) == 0) {
+                        __nanosleep(32);
+                        st[q] = status_load(sp);
+                    }
+                    excl += st[q] & kValMask;
+                    if (st[q] & kFlagInc) done = true;
                 }
-                excl += st & kValMask;
-                if (st & kFlagInc) break;
+                p -= kLook;
             }
-            *reinterpret_cast<volatile uint64_t*>(&status[(uint64_t)tile * kMaxRadix + t]) =
-                (epoch << 48) | kFlagInc | (excl + tile_cnt);
+            status_store(&status[(uint64_t)tile * kMaxRadix + t], (epoch << 48) | kFlagInc | (excl + tile_cnt));
         }
         s_gofs[t] = digit_base[t] + excl;
     }
