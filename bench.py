@@ -714,6 +714,13 @@ def per_algo(tigr, torch, rec, args, s, peak, gceil):
              "roofline_frac_whole_run": st["bytes_alg"] / (t * 1e-3) / 1e9 / peak}
         if ceil_l2:
             r["gather_frac_l2"] = st["edges_processed"] / (t_relax * 1e-3) / 1e9 / ceil_l2
+            # L1 sector accesses per processed arc by the kernel's access pattern:
+            # one target gather (BFS/CC: the settled-bit test, level reads it does not skip
+            # uncounted) + one access per 8-arc span of each streamed array (col; SSSP/SSWP +wt)
+            unit = 8 if args.K % 8 == 0 else (4 if args.K % 4 == 0 else 1)
+            acc = 1.0 + (2.0 if algo in ("sssp", "sswp") else 1.0) / unit
+            r["l1_accesses_per_arc_model"] = acc
+            r["l1_access_frac_l2"] = r["gather_frac_l2"] * acc
         return r
 
     for algo in ("bfs", "sssp", "sswp", "cc"):

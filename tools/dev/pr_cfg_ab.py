@@ -1,5 +1,6 @@
 """A/B of PageRank push relax kernel shapes (TIGR_PR_CFG) on cfg4 in one process: per-launch
-relax ms (CUDA events) and max |x - x_ref| against the default shape.  Development tool."""
+relax ms (CUDA events) and max |x - x_ref| against the default shape.  Development tool; the
+knob is read only by the -DTIGR_DEV_KNOBS build (TIGR_LIB=build/libtigr_dev.so)."""
 import os
 import sys
 
@@ -11,7 +12,7 @@ import torch  # noqa: E402
 import graphgen  # noqa: E402
 import paper_conf_asplos_sabetq018_b200 as tigr  # noqa: E402
 
-cfgs = sys.argv[1].split(",") if len(sys.argv) > 1 else ["5", "7", "8", "9"]
+cfgs = sys.argv[1].split(",") if len(sys.argv) > 1 else ["5", "0", "1", "6"]
 rec = graphgen.recipe(os.environ.get("CFG", "cfg4"))
 s = torch.cuda.current_stream()
 g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, stream=s)

@@ -1,6 +1,6 @@
-"""A/B of an environment knob on the cfg4 PageRank run (default TIGR_PR_FUSE): total and
-relax ms, max |difference| of the results (development tool).
-    python tools/dev/pr_env_ab.py [VAR] [v1,v2,...]"""
+"""A/B of a development knob on the cfg4 PageRank run (default TIGR_PR_CFG): total and relax
+ms, max |difference| of the results.  Knobs are read only by the -DTIGR_DEV_KNOBS build:
+    TIGR_LIB=build/libtigr_dev.so python tools/dev/pr_env_ab.py [VAR] [v1,v2,...]"""
 import os
 import sys
 
@@ -12,8 +12,8 @@ import torch  # noqa: E402
 import graphgen  # noqa: E402
 import paper_conf_asplos_sabetq018_b200 as tigr  # noqa: E402
 
-var = sys.argv[1] if len(sys.argv) > 1 else "TIGR_PR_FUSE"
-vals = sys.argv[2].split(",") if len(sys.argv) > 2 else ["0", "1"]
+var = sys.argv[1] if len(sys.argv) > 1 else "TIGR_PR_CFG"
+vals = sys.argv[2].split(",") if len(sys.argv) > 2 else ["5", "1"]
 rec = graphgen.recipe("cfg4")
 s = torch.cuda.current_stream()
 g = tigr.tigr_graph_rmat(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, weighted=False, stream=s)

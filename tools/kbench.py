@@ -26,7 +26,7 @@ def main():
     dst = torch.empty_like(src)
     tigr.tigr_rmat_coo(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, 1, 64, src, dst, None, stream=s)
     torch.cuda.synchronize()
-    res = {"variant": os.environ.get("TIGR_PR_VARIANT", "default"), "cfg": cfg, "K": K, "layout": layout}
+    res = {"pr_cfg": os.environ.get("TIGR_PR_CFG", "default"), "cfg": cfg, "K": K, "layout": layout}
     csr, vir = [], []
     for _ in range(reps):
         e = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
