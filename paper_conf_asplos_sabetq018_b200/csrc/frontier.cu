@@ -75,20 +75,90 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
 }
 
 // ------------------------------------------------------------------------------------------
+// packed arcs for SSSP / SSWP: target | (w - wmin) << idbits in one 32-bit slot
+// ------------------------------------------------------------------------------------------
+__global__ void k_weight_range(const uint4* __restrict__ c4, const uint4* __restrict__ w4, uint64_t nchunks,
+                               uint32_t* __restrict__ mm) {
+    uint32_t lo = kInf, hi = 0;
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks; k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 c = __ldg(c4 + k), w = __ldg(w4 + k);
+        const uint32_t cc[4] = {c.x, c.y, c.z, c.w}, ww[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if (cc[q] != kPad) { lo = min(lo, ww[q]); hi = max(hi, ww[q]); }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        lo = min(lo, __shfl_xor_sync(kFull, lo, o));
+        hi = max(hi, __shfl_xor_sync(kFull, hi, o));
+    }
+    if ((threadIdx.x & 31) == 0) { atomicMin(mm, lo); atomicMax(mm + 1, hi); }
+}
+
+__global__ void k_pack_arcs(const uint4* __restrict__ c4, const uint4* __restrict__ w4, uint64_t nchunks,
+                            uint32_t idbits, uint32_t wmin, uint4* __restrict__ out) {
+    for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks; k += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 c = __ldg(c4 + k), w = __ldg(w4 + k);
+        uint32_t cc[4] = {c.x, c.y, c.z, c.w};
+        const uint32_t ww[4] = {w.x, w.y, w.z, w.w};
+#pragma unroll
+        for (int q = 0; q < 4; ++q) cc[q] = cc[q] == kPad ? kPad : (cc[q] | ((ww[q] - wmin) << idbits));
+        out[k] = make_uint4(cc[0], cc[1], cc[2], cc[3]);
+    }
+}
+
+// once per virtual graph: pack when the ids and the weight range fit one 32-bit slot together
+// (idbits: the smallest b with 2^b > n, so the all-ones id field is never a node and marks pads)
+tigr_status pack_arcs_prepare(tigr_vgraph* vg, cudaStream_t s) {
+    Workspace& ws = vg->ws;
+    if (ws.cw_state) return TIGR_OK;
+    const tigr_graph* g = vg->g;
+    ws.cw_state = 2;  // not packable until shown otherwise
+    if (!g->weighted || g->nchunks == 0) return TIGR_OK;
+    uint32_t idbits = 1;
+    while (idbits < 32 && ((1ull << idbits) - 1) < (uint64_t)g->n) ++idbits;
+    TmpBuf mm;
+    TIGR_TRY(mm.alloc(2 * sizeof(uint32_t), s));
+    const uint32_t init[2] = {kInf, 0u};
+    TIGR_CK(cudaMemcpyAsync(mm.p, init, sizeof(init), cudaMemcpyHostToDevice, s));
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const unsigned grid = (unsigned)std::min<uint64_t>(grid_for(g->nchunks), (uint64_t)sms * 8);
+    k_weight_range<<<grid, kFqThreads, 0, s>>>(g->col.as<uint4>(), g->wt.as<uint4>(), g->nchunks, mm.as<uint32_t>());
+    TIGR_CKL("pack: weight range");
+    uint32_t h[2] = {0, 0};
+    TIGR_CK(cudaMemcpyAsync(h, mm.p, sizeof(h), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    if (h[0] > h[1]) return TIGR_OK;  // no arcs
+    uint32_t wbits = 0;
+    while (wbits < 32 && ((uint64_t)(h[1] - h[0]) >> wbits) != 0) ++wbits;
+    if (idbits > 31 || idbits + wbits > 32) return TIGR_OK;
+    TIGR_TRY(ws.cw.alloc(sizeof(uint32_t) * kChunk * g->nchunks, s));
+    k_pack_arcs<<<grid, kFqThreads, 0, s>>>(g->col.as<uint4>(), g->wt.as<uint4>(), g->nchunks, idbits, h[0],
+                                            ws.cw.as<uint4>());
+    TIGR_CKL("pack: arcs");
+    ws.cw_idbits = idbits;
+    ws.cw_wmin = h[0];
+    ws.cw_state = 1;
+    return TIGR_OK;
+}
+
+// ------------------------------------------------------------------------------------------
 // dispatch
 // ------------------------------------------------------------------------------------------
 
-FqFn relax_fq_kernel_bfs(int layout, int unit, bool bsp, bool stats);
-FqFn relax_fq_kernel_sssp(int layout, int unit, bool bsp, bool stats);
-FqFn relax_fq_kernel_sswp(int layout, int unit, bool bsp, bool stats);
-FqFn relax_fq_kernel_cc(int layout, int unit, bool bsp, bool stats);
+FqFn relax_fq_kernel_bfs(int layout, int unit, bool bsp, bool stats, bool packed);
+FqFn relax_fq_kernel_sssp(int layout, int unit, bool bsp, bool stats, bool packed);
+FqFn relax_fq_kernel_sswp(int layout, int unit, bool bsp, bool stats, bool packed);
+FqFn relax_fq_kernel_cc(int layout, int unit, bool bsp, bool stats, bool packed);
 
-FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats) {
+FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats, bool packed) {
     switch (algo) {
-        case TIGR_BFS: return relax_fq_kernel_bfs(layout, unit, bsp, stats);
-        case TIGR_SSSP: return relax_fq_kernel_sssp(layout, unit, bsp, stats);
-        case TIGR_CC: return relax_fq_kernel_cc(layout, unit, bsp, stats);
-        case TIGR_SSWP: return relax_fq_kernel_sswp(layout, unit, bsp, stats);
+        case TIGR_BFS: return relax_fq_kernel_bfs(layout, unit, bsp, stats, false);
+        case TIGR_SSSP: return relax_fq_kernel_sssp(layout, unit, bsp, stats, packed);
+        case TIGR_CC: return relax_fq_kernel_cc(layout, unit, bsp, stats, false);
+        case TIGR_SSWP: return relax_fq_kernel_sswp(layout, unit, bsp, stats, packed);
     }
     return nullptr;
 }

@@ -147,9 +147,13 @@ __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, ui
 }
 
 
-template <int A, int LAYOUT, int U, bool BSP, int B, bool STATS, int MINB, bool PRE>
+// PK (SSSP / SSWP): the arcs come from the packed array f.cw -- target | (w - wmin) << idbits in
+// one 32-bit slot (run.cu packs it once per virtual graph when ids and weights fit), so one span
+// load per 8 arcs brings targets and weights together instead of two.
+template <int A, int LAYOUT, int U, bool BSP, int B, bool STATS, int MINB, bool PRE, bool PK = false>
 __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqArgs f) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
+    static_assert(!PK || W, "packed arcs carry weights");
     constexpr uint32_t kFinal = 0u;  // a settled BFS / CC target reads as 0: never improvable
     const bool BITS = (A == TIGR_BFS || A == TIGR_CC) && f.settled != nullptr;  // uniform per launch
     if (!a.ctl->cont) return;  // an iteration enqueued past the fixed point (batched host loop, run.cu)
@@ -163,9 +167,25 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
     const uint32_t* qo = f.qo + (uint64_t)(it & 1u) * a.n;
     const uint32_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;
     uint32_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
-    const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
+    const uint4* c4 = reinterpret_cast<const uint4*>(PK ? f.cw : a.col);
     const uint4* w4 = reinterpret_cast<const uint4*>(a.wt);
     if (blockIdx.x == 0 && threadIdx.x == 0 && queue) atomicAdd(&a.ctl->queue_iters, 1u);
+    // 8 slots -> targets (kPad for pads) and weights
+    auto decode8 = [&](const uint4& c, const uint4& d, const uint4& wc, const uint4& wd, uint32_t* nb, uint32_t* ww) {
+        const uint32_t raw[8] = {c.x, c.y, c.z, c.w, d.x, d.y, d.z, d.w};
+        const uint32_t wr[8] = {wc.x, wc.y, wc.z, wc.w, wd.x, wd.y, wd.z, wd.w};
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            if (PK) {
+                const uint32_t t = raw[q] & f.idmask;
+                nb[q] = t == f.idmask ? kPad : t;
+                ww[q] = (raw[q] >> f.idbits) + f.wmin;
+            } else {
+                nb[q] = raw[q];
+                ww[q] = W ? wr[q] : 0u;
+            }
+        }
+    };
     const uint64_t total = queue ? (uint64_t)qt : span;
     constexpr uint32_t kTile = 32u * B;
     const uint64_t tiles = (total + kTile - 1) / kTile;
@@ -238,7 +258,8 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             else unit_range<U, LAYOUT>(info[r].y, jj, info[r].w, a.K, k, step[r], kend[r]);
             // the first 8 slots: one span (U = 8) or two chunks (U = 4)
             kn[r] = load8<U>(c4, info[r].x, k, step[r], kend[r], c0[r], c1[r], make_uint4(kPad, kPad, kPad, kPad));
-            if (W) load8<U>(w4, info[r].x, k, step[r], kend[r], w0[r], w1[r], make_uint4(0, 0, 0, 0));
+            if (W && !PK) load8<U>(w4, info[r].x, k, step[r], kend[r], w0[r], w1[r], make_uint4(0, 0, 0, 0));
+            else w0[r] = w1[r] = make_uint4(0, 0, 0, 0);
             if (STATS && act[r]) ++n_vn;
         }
         // settled bitmap (f.settled): the test reads one bit of an n/8-byte array instead of the
@@ -289,24 +310,21 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             uint32_t cur[B][8];
 #pragma unroll
             for (int r = 0; r < B; ++r) {
-                const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
+                uint32_t nb[8], ww[8];
+                decode8(c0[r], c1[r], w0[r], w1[r], nb, ww);
                 gather8(nb, cur[r]);
             }
 #pragma unroll
             for (int r = 0; r < B; ++r) {
-                const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
-                uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-                if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
-                         ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
+                uint32_t nb[8], ww[8];
+                decode8(c0[r], c1[r], w0[r], w1[r], nb, ww);
                 apply8(nb, ww, x[r], cur[r]);
             }
         } else {
 #pragma unroll
             for (int r = 0; r < B; ++r) {
-                const uint32_t nb[8] = {c0[r].x, c0[r].y, c0[r].z, c0[r].w, c1[r].x, c1[r].y, c1[r].z, c1[r].w};
-                uint32_t ww[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-                if (W) { ww[0] = w0[r].x; ww[1] = w0[r].y; ww[2] = w0[r].z; ww[3] = w0[r].w;
-                         ww[4] = w1[r].x; ww[5] = w1[r].y; ww[6] = w1[r].z; ww[7] = w1[r].w; }
+                uint32_t nb[8], ww[8];
+                decode8(c0[r], c1[r], w0[r], w1[r], nb, ww);
                 relax8(nb, ww, x[r]);
             }
         }
@@ -315,10 +333,10 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
             for (uint32_t k = kn[r]; k < kend[r];) {
                 uint4 a0, a1, b0 = make_uint4(0, 0, 0, 0), b1 = b0;
                 const uint32_t next = load8<U>(c4, info[r].x, k, step[r], kend[r], a0, a1, make_uint4(kPad, kPad, kPad, kPad));
-                if (W) load8<U>(w4, info[r].x, k, step[r], kend[r], b0, b1, make_uint4(0, 0, 0, 0));
+                if (W && !PK) load8<U>(w4, info[r].x, k, step[r], kend[r], b0, b1, make_uint4(0, 0, 0, 0));
                 k = next;
-                const uint32_t nb[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-                const uint32_t ww[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+                uint32_t nb[8], ww[8];
+                decode8(a0, a1, b0, b1, nb, ww);
                 relax8(nb, ww, x[r]);
             }
         }
@@ -353,10 +371,13 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
 // BSP / stats variants: 4 vnodes per thread, 80 registers, 3 blocks/SM.  Weighted (SSSP, SSWP; one more 16-byte load per chunk): 2 vnodes
 // per thread with all target gathers of both issued before the first atomic, 3 blocks/SM.
 template <int A, int LAYOUT, int U>
-FqFn pick_fq_u(bool bsp, bool stats) {
+FqFn pick_fq_u(bool bsp, bool stats, bool packed) {
     constexpr bool W = (A == TIGR_SSSP || A == TIGR_SSWP);
     constexpr int B = W ? 2 : 4;
     constexpr bool PRE = W;
+    if constexpr (W) {  // packed target | weight arcs (asynchronous schedule, no stats)
+        if (packed && !bsp && !stats) return &k_relax_fq<A, LAYOUT, U, false, B, false, 3, PRE, true>;
+    }
     if (!bsp && !stats) {  // TIGR_FQ_SHAPE: alternative shapes in development builds
         // BFS and CC with their settled bitmap are latency-bound rather than L1/L2-bound
         // (profiles/README.md): 2 virtual nodes per thread with all gathers issued first,
@@ -372,11 +393,12 @@ FqFn pick_fq_u(bool bsp, bool stats) {
 }
 
 template <int A>
-FqFn pick_fq(int layout, int unit, bool bsp, bool stats) {
+FqFn pick_fq(int layout, int unit, bool bsp, bool stats, bool packed) {
     if (layout == TIGR_LAYOUT_STRIDED)
-        return unit == 8 ? pick_fq_u<A, TIGR_LAYOUT_STRIDED, 8>(bsp, stats) : pick_fq_u<A, TIGR_LAYOUT_STRIDED, 4>(bsp, stats);
-    return unit == 8 ? pick_fq_u<A, TIGR_LAYOUT_CONSECUTIVE, 8>(bsp, stats)
-                     : pick_fq_u<A, TIGR_LAYOUT_CONSECUTIVE, 4>(bsp, stats);
+        return unit == 8 ? pick_fq_u<A, TIGR_LAYOUT_STRIDED, 8>(bsp, stats, packed)
+                         : pick_fq_u<A, TIGR_LAYOUT_STRIDED, 4>(bsp, stats, packed);
+    return unit == 8 ? pick_fq_u<A, TIGR_LAYOUT_CONSECUTIVE, 8>(bsp, stats, packed)
+                     : pick_fq_u<A, TIGR_LAYOUT_CONSECUTIVE, 4>(bsp, stats, packed);
 }
 
 }  // namespace

@@ -3,8 +3,8 @@
 
 namespace tigr {
 
-FqFn relax_fq_kernel_sswp(int layout, int unit, bool bsp, bool stats) {
-    return pick_fq<TIGR_SSWP>(layout, unit, bsp, stats);
+FqFn relax_fq_kernel_sswp(int layout, int unit, bool bsp, bool stats, bool packed) {
+    return pick_fq<TIGR_SSWP>(layout, unit, bsp, stats, packed);
 }
 
 }  // namespace tigr

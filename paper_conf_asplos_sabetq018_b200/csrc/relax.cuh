@@ -43,13 +43,17 @@ struct FqArgs {
     uint32_t* settled;    // BFS / CC: bit v set once v's value is final (nullptr: always test the value)
     const FusedPeers* peers;  // fused exchange: every improvement is also applied to the peers' replicas
     uint32_t run;         // queue tiles per warp run (frontier_kernel.cuh): the search runs once per run
+    const uint32_t* cw;   // SSSP / SSWP packed arcs: target | (w - wmin) << idbits (nullptr: col + wt)
+    uint32_t idmask, idbits, wmin;
 };
 typedef void (*FqFn)(RelaxArgs, FqArgs);
-FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats);  // unit 4 or 8 (vgraph.cuh)
+// unit 4 or 8 (vgraph.cuh); packed: SSSP / SSWP read FqArgs.cw (target | weight slots)
+FqFn relax_fq_kernel(int algo, int layout, int unit, bool bsp, bool stats, bool packed);
 unsigned relax_fq_grid(FqFn fn);   // persistent grid: SMs x resident blocks
 int relax_fq_threads();
 struct Ctl;
 tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStream_t s);
+tigr_status pack_arcs_prepare(tigr_vgraph* vg, cudaStream_t s);  // SSSP / SSWP packed arcs (frontier.cu)
 typedef void (*AssignFn)(RelaxArgs, const uint32_t*, uint32_t*, uint32_t*, uint32_t*, int, int);
 
 RelaxFn relax_kernel(int algo, int layout, int unit, int front, bool bsp, bool stats);

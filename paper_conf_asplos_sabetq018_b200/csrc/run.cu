@@ -167,7 +167,17 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     FrontierPlan p;
     p.vg = vg;
     if ((front == TIGR_FRONTIER_AUTO || front == TIGR_FRONTIER_QUEUE) && vg->vec) {
-        p.fq = relax_fq_kernel(algo, vg->layout, (int)vg->unit, o.schedule == 1, o.collect_stats != 0);
+        // SSSP / SSWP: targets and weights packed into one slot when they fit (frontier.cu)
+        bool packed = false;
+        if ((algo == TIGR_SSSP || algo == TIGR_SSWP) && dev_knob("TIGR_PACK_ARCS", 1)) {
+            TIGR_TRY(pack_arcs_prepare(vg, s));
+            packed = ws.cw_state == 1;
+        }
+        p.fq = relax_fq_kernel(algo, vg->layout, (int)vg->unit, o.schedule == 1, o.collect_stats != 0, packed);
+        p.fa.cw = packed ? ws.cw.as<uint32_t>() : nullptr;
+        p.fa.idbits = packed ? ws.cw_idbits : 0u;
+        p.fa.idmask = packed ? (uint32_t)((1ull << ws.cw_idbits) - 1) : 0u;
+        p.fa.wmin = packed ? ws.cw_wmin : 0u;
         p.fa.qv = ws.qv.as<uint32_t>();
         p.fa.qo = ws.qo.as<uint32_t>();
         p.fa.mode = front == TIGR_FRONTIER_QUEUE ? 1 : 0;

@@ -57,7 +57,10 @@ struct Workspace {
     bool cid_ready = false;
     DevBuf qv;       // uint32[2][n]: active-node queue (node ids), one slot per iteration parity
     DevBuf qo;       // uint32[2][n]: first queue-space virtual node of each entry (exclusive prefix)
-    DevBuf settled;  // uint32[n/32+1]: BFS settled bitmap (frontier.cu)
+    DevBuf settled;  // uint32[n/32+1]: BFS / CC settled bitmap (frontier.cu)
+    DevBuf cw;       // uint32[4 * nchunks]: SSSP / SSWP packed arcs target | (w - wmin) << idbits
+    int cw_state = 0;         // 0 not prepared, 1 packed, 2 ids and weights do not fit 32 bits
+    uint32_t cw_idbits = 0, cw_wmin = 0;
     DevBuf xlist;    // uint2[n]: multi-GPU sparse exchange records {node, value} (exchange.cu)
     DevBuf peers;    // FusedPeers (fused multi-GPU exchange, exchange.cu)
     DevBuf ctl;      // Ctl
