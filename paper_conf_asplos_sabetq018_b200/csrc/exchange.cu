@@ -45,15 +45,16 @@ struct Lists {
 };
 
 // {node, value} of every node stamped for iteration it + 1 (warp-aggregated append)
-__global__ void k_pack(uint32_t n, const uint32_t* __restrict__ val, const uint32_t* __restrict__ stamp, Ctl* ctl,
+__global__ void k_pack(uint32_t n, const uint32_t* __restrict__ val, const stamp_t* __restrict__ stamp, Ctl* ctl,
                        uint2* __restrict__ out) {
     const uint32_t it = ctl->it;
-    const uint32_t* st = stamp + (uint64_t)((it + 1) & 1u) * n;
+    const stamp_t* st = stamp + (uint64_t)((it + 1) & 1u) * n;
+    const stamp_t sn = stamp_of(it + 1);
     const int lane = threadIdx.x & 31;
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     for (uint64_t b = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); b < n; b += stride) {
         const uint64_t v = b + lane;
-        const bool on = v < n && st[v] == it + 1;
+        const bool on = v < n && st[v] == sn;
         const uint32_t mask = __ballot_sync(0xffffffffu, on);
         if (!mask) continue;
         uint32_t base = 0;
@@ -65,18 +66,18 @@ __global__ void k_pack(uint32_t n, const uint32_t* __restrict__ val, const uint3
 
 // apply the other ranks' records with the relax's own atomic; activate every listed node
 template <int A>
-__global__ void k_apply_lists(Lists L, int me, uint32_t n, uint32_t* __restrict__ val, uint32_t* __restrict__ stamp,
+__global__ void k_apply_lists(Lists L, int me, uint32_t n, uint32_t* __restrict__ val, stamp_t* __restrict__ stamp,
                               const Ctl* ctl) {
     const int r = blockIdx.y;
     if (r == me) return;  // this rank's own records are already in its replica and its stamps
     const uint32_t it = ctl->it;
-    uint32_t* st = stamp + (uint64_t)((it + 1) & 1u) * n;
+    stamp_t* st = stamp + (uint64_t)((it + 1) & 1u) * n;
     const uint2* p = L.p[r];
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < L.cnt[r]; i += gridDim.x * blockDim.x) {
         const uint2 e = p[i];
         if (A == TIGR_SSWP) atomicMax(val + e.x, e.y);
         else atomicMin(val + e.x, e.y);
-        st[e.x] = it + 1;
+        st[e.x] = stamp_of(it + 1);
     }
 }
 
@@ -116,7 +117,7 @@ tigr_status dense(const ExchangeArgs& x, cudaStream_t s) {
 // then each rank reads the common verdict.  Before the first iteration every replica must be
 // initialised (barrier after init); in BSP mode the snapshot is taken between two barriers so
 // that no peer's update of the new iteration leaks into it.
-tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, DevBuf& peers_buf,
+tigr_status fused_setup(tigr_comm* c, uint32_t* val, stamp_t* stamp, Ctl* ctl, DevBuf& peers_buf,
                         cudaStream_t s, const FusedPeers** out) {
     if (!c->local) return fail(TIGR_EUNSUPPORTED, "fused exchange needs a thread-group or node communicator");
     if (c->nranks > kMaxPeers) return fail(TIGR_EUNSUPPORTED, "fused exchange: more than 16 ranks");
@@ -128,7 +129,7 @@ tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, 
     h.me = c->rank;
     for (int r = 0; r < c->nranks; ++r) {
         h.val[r] = const_cast<uint32_t*>(static_cast<const uint32_t*>(all[3 * r]));
-        h.stamp[r] = const_cast<uint32_t*>(static_cast<const uint32_t*>(all[3 * r + 1]));
+        h.stamp[r] = const_cast<stamp_t*>(static_cast<const stamp_t*>(all[3 * r + 1]));
         h.ctl[r] = const_cast<Ctl*>(static_cast<const Ctl*>(all[3 * r + 2]));
     }
     if (!peers_buf.p) TIGR_TRY(peers_buf.alloc(sizeof(FusedPeers), s));

@@ -18,7 +18,7 @@ constexpr uint32_t kFull = 0xffffffffu;
 // ------------------------------------------------------------------------------------------
 // queue build: nodes stamped for iteration it + delta that own virtual nodes in [lo, hi)
 // ------------------------------------------------------------------------------------------
-__global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restrict__ stamp,
+__global__ void __launch_bounds__(kFqThreads) k_compact(const stamp_t* __restrict__ stamp,
                                                          const uint4* __restrict__ vinfo, uint32_t n, uint32_t lo,
                                                          uint32_t hi, Ctl* ctl, uint32_t* __restrict__ qv,
                                                          uint32_t* __restrict__ qo, int delta) {
@@ -27,7 +27,8 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
     if (!ctl->cont) return;  // past the fixed point (batched host loop, run.cu); k_init sets cont
     const uint32_t itn = ctl->it + (uint32_t)delta;
     const uint32_t slot = itn & 1u;
-    const uint32_t* st = stamp + (uint64_t)slot * n;
+    const stamp_t* st = stamp + (uint64_t)slot * n;
+    const stamp_t sv = stamp_of(itn);
     uint32_t* ov = qv + (uint64_t)slot * n;
     uint32_t* oo = qo + (uint64_t)slot * n;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -36,11 +37,21 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const uint32_t* __restri
         const uint64_t v0 = tile0 + (uint64_t)threadIdx.x * kCompactPer;
         uint32_t m[kCompactPer];
         unsigned long long mine = 0;  // (entries << 32) | vnodes of this thread's nodes
+        // the thread's 8 stamps: one 8-byte load when aligned (n % 8 == 0 keeps slot 1 aligned)
+        stamp_t sb[kCompactPer];
+        if ((n & 7u) == 0 && v0 + kCompactPer <= n) {
+            const uint2 w = __ldg(reinterpret_cast<const uint2*>(st + v0));
+#pragma unroll
+            for (int q = 0; q < kCompactPer; ++q) sb[q] = (stamp_t)(((q < 4 ? w.x : w.y) >> (8 * (q & 3))) & 0xFFu);
+        } else {
+#pragma unroll
+            for (int q = 0; q < kCompactPer; ++q) sb[q] = v0 + q < n ? __ldg(st + v0 + q) : (stamp_t)0;
+        }
 #pragma unroll
         for (int q = 0; q < kCompactPer; ++q) {
             const uint64_t v = v0 + q;
             m[q] = 0;
-            if (v < n && __ldg(st + v) == itn) {
+            if (v < n && sb[q] == sv) {
                 const uint4 info = __ldg(vinfo + v);
                 if (info.w && info.z >= lo && info.z < hi) m[q] = info.w;
             }
@@ -179,7 +190,7 @@ tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStrea
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const uint64_t tiles = ((uint64_t)n + kFqThreads * kCompactPer - 1) / (kFqThreads * kCompactPer);
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(tiles, (uint64_t)sms * 8));
-    k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<uint32_t>(), vg->vinfo.as<uint4>(), n, vg->lo, vg->hi, ctl,
+    k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<stamp_t>(), vg->vinfo.as<uint4>(), n, vg->lo, vg->hi, ctl,
                                           const_cast<uint32_t*>(vg->ws.qv.as<uint32_t>()),
                                           const_cast<uint32_t*>(vg->ws.qo.as<uint32_t>()), delta);
     TIGR_CK(cudaGetLastError());

@@ -142,7 +142,7 @@ __device__ __forceinline__ void push_peers(const FusedPeers* __restrict__ pp, ui
     for (int r = 0; r < pp->P; ++r) {
         if (r == pp->me) continue;
         atomic_better_sys<A>(pp->val[r] + v, alt);
-        pp->stamp[r][slot + v] = it + 1;
+        pp->stamp[r][slot + v] = stamp_of(it + 1);
     }
 }
 
@@ -165,8 +165,9 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
     const bool queue = f.mode == 1 || (f.mode == 0 && (uint64_t)qt * f.dense_div < span);
     const uint32_t* qv = f.qv + (uint64_t)(it & 1u) * a.n;
     const uint32_t* qo = f.qo + (uint64_t)(it & 1u) * a.n;
-    const uint32_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;
-    uint32_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
+    const stamp_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;
+    stamp_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
+    const stamp_t s_cur = stamp_of(it), s_next = stamp_of(it + 1);
     const uint4* c4 = reinterpret_cast<const uint4*>(PK ? f.cw : a.col);
     const uint4* w4 = reinterpret_cast<const uint4*>(a.wt);
     if (blockIdx.x == 0 && threadIdx.x == 0 && queue) atomicAdd(&a.ctl->queue_iters, 1u);
@@ -232,7 +233,7 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                 j[r] = (uint32_t)i;  // absolute vnode index; made family-relative below
             }
 #pragma unroll
-            for (int r = 0; r < B; ++r) act[r] = v[r] != kPad && __ldg(stamp_cur + v[r]) == it;
+            for (int r = 0; r < B; ++r) act[r] = v[r] != kPad && __ldg(stamp_cur + v[r]) == s_cur;
         }
         uint32_t x[B];
         uint4 info[B];
@@ -295,7 +296,7 @@ __global__ void __launch_bounds__(kFqThreads, MINB) k_relax_fq(RelaxArgs a, FqAr
                     // BFS: the level becomes alt = it, final (see the header); CC: label 0 is final
                     if (BITS && (A == TIGR_BFS || (A == TIGR_CC && alt == 0u)))
                         atomicOr(f.settled + (nb[q] >> 5), 1u << (nb[q] & 31u));
-                    stamp_next[nb[q]] = it + 1;
+                    stamp_next[nb[q]] = s_next;
                     touched = true;
                     if (STATS) ++n_upd;
                 }

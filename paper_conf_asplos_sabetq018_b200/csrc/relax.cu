@@ -82,7 +82,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
     if (i < a.hi) {
         const uint32_t v = a.vn_phys[i];
         bool act = true;
-        if (FRONT == TIGR_FRONTIER_DENSE) act = a.stamp[(uint64_t)(it & 1u) * a.n + v] == it;
+        if (FRONT == TIGR_FRONTIER_DENSE) act = a.stamp[(uint64_t)(it & 1u) * a.n + v] == stamp_of(it);
         uint32_t x = 0;
         if (act) {
             x = BSP ? a.prev[v] : a.val[v];
@@ -108,7 +108,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax(RelaxArgs a) {
                     if (better<A>(alt, cur[t])) {
                         if (A == TIGR_SSWP) atomicMax(a.val + nb[t], alt);
                         else atomicMin(a.val + nb[t], alt);
-                        if (FRONT == TIGR_FRONTIER_DENSE) a.stamp[(uint64_t)((it + 1) & 1u) * a.n + nb[t]] = it + 1;
+                        if (FRONT == TIGR_FRONTIER_DENSE) a.stamp[(uint64_t)((it + 1) & 1u) * a.n + nb[t]] = stamp_of(it + 1);
                         touched = true;
                         if (STATS) ++n_upd;
                     }
@@ -143,8 +143,9 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
     if (!a.ctl->cont) return;  // past the fixed point (batched host loop)
     const uint64_t base = (uint64_t)a.lo + (uint64_t)blockIdx.x * (B * kRelaxThreads) + threadIdx.x;
     const uint32_t it = (FRONT == TIGR_FRONTIER_DENSE) ? a.ctl->it : 0;
-    const uint32_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;   // not written in this launch
-    uint32_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
+    const stamp_t* stamp_cur = a.stamp + (uint64_t)(it & 1u) * a.n;   // not written in this launch
+    stamp_t* stamp_next = a.stamp + (uint64_t)((it + 1) & 1u) * a.n;
+    const stamp_t s_cur = stamp_of(it), s_next = stamp_of(it + 1);
     const uint4* c4 = reinterpret_cast<const uint4*>(a.col);
     const uint4* w4 = reinterpret_cast<const uint4*>(a.wt);
     bool touched = false;
@@ -159,7 +160,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
 #pragma unroll
     for (int r = 0; r < B; ++r) {
         act[r] = v[r] != kPad;
-        if (FRONT == TIGR_FRONTIER_DENSE && act[r]) act[r] = __ldg(stamp_cur + v[r]) == it;
+        if (FRONT == TIGR_FRONTIER_DENSE && act[r]) act[r] = __ldg(stamp_cur + v[r]) == s_cur;
     }
     uint32_t x[B];
     uint4 info[B];
@@ -206,7 +207,7 @@ __global__ void __launch_bounds__(kRelaxThreads) k_relax_mlp(RelaxArgs a) {
             if (better<A>(alt, cur[q])) {
                 if (A == TIGR_SSWP) atomicMax(a.val + nb[q], alt);
                 else atomicMin(a.val + nb[q], alt);
-                if (FRONT == TIGR_FRONTIER_DENSE) stamp_next[nb[q]] = it + 1;
+                if (FRONT == TIGR_FRONTIER_DENSE) stamp_next[nb[q]] = s_next;
                 touched = true;
             }
         }
@@ -363,7 +364,7 @@ RelaxFn relax_kernel(int algo, int layout, int unit, int front, bool bsp, bool s
 // init / control / PR apply / multi-GPU diff / assignment dump
 // ------------------------------------------------------------------------------------------
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
-                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
+                       stamp_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
                        const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order,
                        uint32_t* __restrict__ settled) {
     // reordered graphs (tigr_graph_reorder): the source is an original id, CC labels are
@@ -379,8 +380,8 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
         // BFS: the source's level 0 is final from the start; its settled bit (cleared before this
         // kernel; frontier_kernel.cuh) spares every gather of it -- R-MAT's source is a hub
         if (settled && v == src && algo == TIGR_BFS) atomicOr(settled + (v >> 5), 1u << (v & 31u));
-        stamp[v] = 0u;                                                // parity 0
-        stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == src) ? 1u : 0u;  // parity 1: it = 1
+        stamp[v] = 0;                                                  // parity 0: never stamped
+        stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == src) ? stamp_of(1) : 0;  // parity 1: it = 1
     }
     if (v == 0) {
         ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
@@ -424,14 +425,14 @@ __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle
 
 // multi-GPU: after the all-reduce, activate every node whose replica value moved
 __global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
-                       uint32_t* __restrict__ stamp, Ctl* ctl) {
+                       stamp_t* __restrict__ stamp, Ctl* ctl) {
     if (!ctl->cont) return;  // past the fixed point (batched host loop, run.cu)
     const uint32_t it = ctl->it;
     bool moved = false;
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
     if (v < n) {
         const uint32_t x = val[v];
-        if (x != prev[v]) { prev[v] = x; stamp[(uint64_t)((it + 1) & 1u) * n + v] = it + 1; moved = true; }
+        if (x != prev[v]) { prev[v] = x; stamp[(uint64_t)((it + 1) & 1u) * n + v] = stamp_of(it + 1); moved = true; }
     }
     if (__any_sync(0xffffffffu, moved) && (threadIdx.x & 31) == 0) ctl->changed = 1;
 }

@@ -8,6 +8,14 @@ namespace tigr {
 
 constexpr int kRelaxThreads = 256;
 
+// Worklist stamps (one byte per node and iteration parity): node v is active in iteration it
+// iff stamp[(it & 1) n + v] == stamp_of(it).  Stamp values cycle through 1..255 (0 = never
+// stamped), so a stale byte can only match again 510 iterations later -- a spurious activation,
+// which is harmless: the node re-pushes a value its targets already hold.  One
+// byte instead of four: the per-iteration queue build scans n bytes instead of 4n.
+typedef uint8_t stamp_t;
+__host__ __device__ __forceinline__ stamp_t stamp_of(uint32_t it) { return (stamp_t)(1u + (it - 1u) % 255u); }
+
 struct RelaxArgs {
     const uint32_t* __restrict__ vn_phys;
     const uint4* __restrict__ vinfo;
@@ -16,7 +24,7 @@ struct RelaxArgs {
     uint32_t lo, hi, K, n;
     uint32_t* val;               // values, updated in place with atomics
     const uint32_t* prev;        // BSP snapshot
-    uint32_t* stamp;             // uint32[2n] worklist stamps
+    stamp_t* stamp;              // stamp_t[2n] worklist stamps (stamp_of)
     double* acc;                 // PR accumulator (RED.ADD.F64 target)
     const double* contrib;       // PR x/deg
     Ctl* ctl;
@@ -30,7 +38,7 @@ constexpr int kMaxPeers = 16;
 struct FusedPeers {
     int P, me;
     uint32_t* val[kMaxPeers];
-    uint32_t* stamp[kMaxPeers];
+    stamp_t* stamp[kMaxPeers];
     Ctl* ctl[kMaxPeers];
 };
 
@@ -81,14 +89,14 @@ tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangl
 AssignFn assign_kernel(int layout, int unit);
 
 __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restrict__ val,
-                       uint32_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
+                       stamp_t* __restrict__ stamp, Ctl* ctl, uint32_t max_iters,
                        const uint32_t* __restrict__ cid, const uint32_t* __restrict__ order,
                        uint32_t* __restrict__ settled);
 // out[v] = val[cid[v]] (results of a reordered graph in original ids)
 tigr_status unpermute(uint32_t n, const uint32_t* cid, const void* val, void* out, bool f64, cudaStream_t s);
 __global__ void k_control(Ctl* ctl, cudaGraphConditionalHandle h, int use_handle);
 __global__ void k_diff(uint32_t n, const uint32_t* __restrict__ val, uint32_t* __restrict__ prev,
-                       uint32_t* __restrict__ stamp, Ctl* ctl);
+                       stamp_t* __restrict__ stamp, Ctl* ctl);
 // multi-GPU merge of the replicated frontier values after a relax (exchange.cu)
 struct ExchangeArgs {
     tigr_comm* comm;
@@ -97,12 +105,12 @@ struct ExchangeArgs {
     uint32_t n;
     uint32_t* val;
     uint32_t* prev;
-    uint32_t* stamp;
+    stamp_t* stamp;
     uint2* list;       // uint2[n] records of this rank (sparse mode)
     Ctl* ctl;
 };
 tigr_status exchange_frontier(const ExchangeArgs& x, cudaStream_t s, bool* sparse_used);
-tigr_status fused_setup(tigr_comm* c, uint32_t* val, uint32_t* stamp, Ctl* ctl, DevBuf& peers_buf,
+tigr_status fused_setup(tigr_comm* c, uint32_t* val, stamp_t* stamp, Ctl* ctl, DevBuf& peers_buf,
                         cudaStream_t s, const FusedPeers** out);
 tigr_status fused_barrier(tigr_comm* c, cudaStream_t s);
 tigr_status fused_end_iteration(tigr_comm* c, Ctl* ctl, cudaStream_t s);

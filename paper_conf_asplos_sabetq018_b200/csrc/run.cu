@@ -77,7 +77,7 @@ tigr_status ensure_ws(tigr_vgraph* vg, bool pr, cudaStream_t s) {
     } else if (!ws.val.p) {
         TIGR_TRY(ws.val.alloc(sizeof(uint32_t) * n, s));
         TIGR_TRY(ws.prev.alloc(sizeof(uint32_t) * n, s));
-        TIGR_TRY(ws.stamp.alloc(sizeof(uint32_t) * 2 * n, s));
+        TIGR_TRY(ws.stamp.alloc(sizeof(stamp_t) * 2 * n, s));
     }
     if (!pr && vg->vec && !ws.qv.p) {  // active-node queues (frontier.cu), one per iteration parity
         TIGR_TRY(ws.qv.alloc(sizeof(uint32_t) * 2 * n, s));
@@ -99,7 +99,7 @@ RelaxArgs make_args(tigr_vgraph* vg) {
     a.n = g->n;
     a.val = vg->ws.val.as<uint32_t>();
     a.prev = vg->ws.prev.as<uint32_t>();
-    a.stamp = vg->ws.stamp.as<uint32_t>();
+    a.stamp = vg->ws.stamp.as<stamp_t>();
     a.acc = vg->ws.acc.as<double>();
     a.contrib = vg->ws.contrib.as<double>();
     a.ctl = vg->ws.ctl.as<Ctl>();

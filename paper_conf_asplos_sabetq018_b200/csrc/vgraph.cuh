@@ -12,7 +12,7 @@ namespace tigr {
 // Device-side control block of one run (one per vgraph workspace).
 struct Ctl {
     uint32_t changed;      // set by relax when any value improved this iteration
-    uint32_t it;           // current iteration (1-based; node v is active iff stamp[v] == it)
+    uint32_t it;           // current iteration (1-based; node v is active iff stamp[v] == stamp_of(it))
     uint32_t max_iters;
     uint32_t cont;         // 1 while the loop should continue (host-loop mode reads it)
     uint32_t notconv;      // 1 if the cap was hit while values still changed
@@ -45,7 +45,7 @@ struct CachedGraph {
 struct Workspace {
     DevBuf val;      // uint32[n] values (BFS/SSSP/CC/SSWP)
     DevBuf prev;     // uint32[n] BSP snapshot / multi-GPU pre-exchange copy
-    DevBuf stamp;    // uint32[2n] worklist: node v active in iteration it iff stamp[(it&1)n + v] == it;
+    DevBuf stamp;    // uint8[2n] worklist: node v active in iteration it iff stamp[(it&1)n + v] == stamp_of(it);
                      // relax(it) writes only the other parity, so activations never race reads
     DevBuf x;        // double[n] PR rank
     DevBuf contrib;  // double[n] PR x/deg
