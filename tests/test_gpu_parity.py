@@ -646,3 +646,76 @@ def test_reordered_cfg2_and_iterations(tigr):
     _, st1 = tigr.tigr_run(vg, "bfs", 0, schedule=1, return_stats=True)
     lv, st2 = tigr.tigr_run(vg2, "bfs", 0, schedule=1, return_stats=True)
     assert np.array_equal(lv, want) and st1["iterations"] == st2["iterations"]
+
+
+# ------------------------------------------------------------------------- round-2 paths
+@pytest.mark.parametrize("frontier", [0, 1, 3])
+@pytest.mark.parametrize("schedule", [0, 1])
+def test_long_path_stamp_wraparound(tigr, frontier, schedule):
+    """A 1300-node path (plus a hub feeding its first nodes) needs ~1300 iterations: the one-byte
+    worklist stamps (values 1..255, relax.cuh stamp_of) wrap around five times, and a stale byte
+    may re-activate a node 510 iterations later.  Values must still equal the oracle, and BSP
+    iteration counts must equal the paper-literal push's."""
+    n = 1300
+    src = list(range(n - 1)) + [0] * 40
+    dst = list(range(1, n)) + list(range(2, 42))
+    w = [(i % 64) + 1 for i in range(n - 1)] + [64] * 40
+    src, dst, w = (np.asarray(x, dtype=np.uint32) for x in (src, dst, w))
+    got = _run_all(tigr, n, src, dst, w, 8, frontier=frontier, schedule=schedule)
+    _assert_parity(got, _oracle_all(n, src, dst, w))
+    if schedule == 1:
+        o = oracle.csr_build(n, src, dst, w)
+        vg = tigr.tigr_virtualize(tigr.tigr_graph_from_coo(n, src, dst, w), 8)
+        _, want_it, _ = oracle.push_virtual(o, oracle.Virtual(o, 8), oracle.BFS, 0, schedule=1, worklist=1)
+        _, st = tigr.tigr_run(vg, "bfs", 0, schedule=1, frontier=frontier, return_stats=True)
+        assert st["iterations"] == want_it > 510
+
+
+@pytest.mark.parametrize("weights", ["offset", "wide", "max"])
+@pytest.mark.parametrize("K", [4, 8])
+def test_packed_arcs_and_fallback(tigr, weights, K):
+    """SSSP/SSWP pack target | (w - wmin) << idbits when ids and the weight range fit 32 bits
+    (frontier.cu pack_arcs_prepare): weights in [100, 163] exercise the wmin offset; weights up to
+    2^30 (30 bits + 11 id bits) and up to 2^32 - 2 do not fit and run from the two arrays."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, _ = graphgen.generate(rec)
+    rng = np.random.default_rng(5)
+    if weights == "offset":
+        w = rng.integers(100, 164, len(src), dtype=np.uint32)
+    elif weights == "wide":
+        w = rng.integers(1, 1 << 30, len(src), dtype=np.uint32)
+    else:
+        w = rng.integers(1, 0xFFFFFFFE, len(src), dtype=np.uint32)
+    o = oracle.csr_build(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(tigr.tigr_graph_from_coo(rec.n, src, dst, w), K)
+    for _ in range(2):  # the second run reuses the packed array
+        assert np.array_equal(tigr.tigr_run(vg, "sswp", 0), oracle.sswp(o, 0))
+        if weights != "max":  # 2^32-scale SSSP sums saturate (reading R14); SSWP covers that case
+            assert np.array_equal(tigr.tigr_run(vg, "sssp", 0), oracle.sssp(o, 0))
+    if weights != "max":  # the BSP schedule runs the unpacked kernel on the same graph
+        assert np.array_equal(tigr.tigr_run(vg, "sssp", 0, schedule=1), oracle.sssp(o, 0))
+
+
+@pytest.mark.parametrize("sym", [False, True])
+def test_host_input_multi_chunk(tigr, sym):
+    """Host arc lists are copied in 2^24-arc chunks overlapped with the arc-list scan (sort.cu):
+    2^24 + 12345 arcs from host memory (two chunks, the second ragged) must build the same CSR
+    as the oracle's stable counting sort, symmetrised or not, and the same as the device-input
+    build."""
+    n, m = 1 << 20, (1 << 24) + 12345
+    rng = np.random.default_rng(9)
+    src = rng.integers(0, n, m, dtype=np.uint32)
+    dst = rng.integers(0, n, m, dtype=np.uint32)
+    w = rng.integers(1, 65, m, dtype=np.uint32)
+    g = tigr.tigr_graph_from_coo(n, src, dst, None if sym else w, symmetrize=sym)
+    rp, col, ww = tigr.tigr_graph_export_csr(g)
+    if sym:
+        o = oracle.csr_build(n, np.concatenate([src, dst]), np.concatenate([dst, src]))
+    else:
+        o = oracle.csr_build(n, src, dst, w)
+        assert np.array_equal(ww, o.wt)
+    assert np.array_equal(rp, o.row_ptr) and np.array_equal(col, o.col)
+    gd = tigr.tigr_graph_from_coo(n, torch.from_numpy(src.view(np.int32)).cuda(), torch.from_numpy(dst.view(np.int32)).cuda(),
+                                  None if sym else torch.from_numpy(w.view(np.int32)).cuda(), symmetrize=sym)
+    rpd, cold, _ = tigr.tigr_graph_export_csr(gd)
+    assert np.array_equal(rpd, rp) and np.array_equal(cold, col)
