@@ -491,7 +491,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
         // of the f64 accumulator), per virtual node 4, per node with arcs its source value: 20
         // with the apply fused in (previous accumulator 8 + cid 4 + row pair 8), else 16
         // (contrib 8 + row pair 8)
-        st->bytes_alg = (uint64_t)launches * (vg->g->m * 20 + (uint64_t)(vg->hi - vg->lo) * 4 + vg->n_out * (fuse ? 20 : 16));
+        st->bytes_alg = (uint64_t)launches * (vg->m_local * 20 + (uint64_t)(vg->hi - vg->lo) * 4 + vg->n_out * (fuse ? 20 : 16));
     }
     return TIGR_OK;
 }
@@ -641,6 +641,12 @@ tigr_status partition_host(tigr_vgraph* vg, int nranks, int rank) {
     vg->lo = h[0];
     vg->hi = h[1];
     vg->n_out = hn;
+    // this rank's arcs: row_ptr[cut(rank + 1)] - row_ptr[cut(rank)] (the byte model's arc count)
+    int64_t rp[2] = {0, 0};
+    TIGR_CK(cudaMemcpyAsync(&rp[0], g->row_ptr.as<int64_t>() + h[2], sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaMemcpyAsync(&rp[1], g->row_ptr.as<int64_t>() + h[3], sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    vg->m_local = (uint64_t)(rp[1] - rp[0]);
     return TIGR_OK;
 }
 

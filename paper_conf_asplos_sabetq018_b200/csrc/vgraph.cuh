@@ -86,6 +86,7 @@ struct tigr_vgraph {
     tigr::DevBuf vinfo;          // uint4[n] = {first 16-byte chunk, degree, first vnode, family size}
     uint32_t lo = 0, hi = 0;     // this rank's vnode range
     uint64_t n_out = 0;          // nodes with out-arcs whose virtual nodes lie in [lo, hi)
+    uint64_t m_local = 0;        // arcs of the nodes whose virtual nodes lie in [lo, hi)
     double ms_build = 0.0;
     tigr::Workspace ws;
 };

@@ -99,6 +99,7 @@ tigr_status virtualize_device(const tigr_graph* g, uint32_t K, tigr_layout layou
     cudaError_t e = cudaEventSynchronize(e1);
     if (e != cudaSuccess) return bail(cuda_fail(e, "virtualize", __FILE__, __LINE__));
     vg->n_out = n_out;
+    vg->m_local = g->m;
     float ms = 0.f;
     cudaEventElapsedTime(&ms, e0, e1);
     cudaEventDestroy(e0);

@@ -719,3 +719,36 @@ def test_host_input_multi_chunk(tigr, sym):
                                   None if sym else torch.from_numpy(w.view(np.int32)).cuda(), symmetrize=sym)
     rpd, cold, _ = tigr.tigr_graph_export_csr(gd)
     assert np.array_equal(rpd, rp) and np.array_equal(cold, col)
+
+
+def test_bytes_alg_byte_model(tigr):
+    """tigr_stats.bytes_alg is SURVEY §8(d)'s byte model, computed in the library: PageRank per
+    relax launch 20 B/arc + 4 B/virtual node + 20 B per node with arcs (apply fused in), over
+    this rank's range after tigr_vgraph_partition; frontier algorithms with collect_stats from the
+    device counters (0 without them)."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    deg = np.bincount(src, minlength=rec.n)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    vg = tigr.tigr_virtualize(g, 8)
+    nv = vg.info()["nv"]
+    _, st = tigr.tigr_run(vg, "pr", return_stats=True)
+    assert st["bytes_alg"] == 20 * (rec.m * 20 + nv * 4 + int((deg > 0).sum()) * 20)
+    assert abs(st["ms_kernels"] - (st["ms_total"] - st["ms_exchange"])) < 1e-9
+    # one rank of two: its node range's arcs, virtual nodes and nodes with arcs
+    vp, _ = tigr.tigr_vgraph_export(vg)
+    rp = np.concatenate([[0], np.cumsum(deg)]).astype(np.int64)
+    lo, hi = tigr.tigr_partition_ranges(rp, vp, 2)
+    for r in range(2):
+        tigr.tigr_vgraph_partition(vg, 2, r)
+        info = vg.info()
+        assert (info["lo"], info["hi"]) == (lo[r], hi[r])
+        nodes = np.flatnonzero((vp[:-1] >= lo[r]) & (vp[:-1] < hi[r]) & (deg > 0))
+        _, st = tigr.tigr_run(vg, "pr", return_stats=True, pr_iters=3)
+        assert st["bytes_alg"] == 3 * (int(deg[nodes].sum()) * 20 + (int(hi[r]) - int(lo[r])) * 4 + len(nodes) * 20)
+    tigr.tigr_vgraph_partition(vg, 1, 0)
+    _, st = tigr.tigr_run(vg, "bfs", 0, return_stats=True)
+    assert st["bytes_alg"] == 0
+    _, st = tigr.tigr_run(vg, "bfs", 0, return_stats=True, collect_stats=1)
+    assert st["bytes_alg"] == (st["edges_processed"] * 8 + st["updates"] * 4 + st["active_vnodes"] * 4
+                               + st["active_nodes"] * 12 + st["iterations"] * 2 * rec.n)
