@@ -304,13 +304,7 @@ tigr_status graph_from_coo_part_device(uint32_t n, uint64_t m, const uint32_t* s
     tigr_status st = csr_build_sorted(n, m, src, dst, w, symmetrize, s, g, src_lo, src_hi, host);
     g->part_lo = src_lo;
     g->part_hi = src_hi < n ? src_hi : n;
-    if (st == TIGR_OK) {
-        k_pad<<<grid_for(n), kBlock, 0, s>>>(g->deg.as<uint32_t>(), g->cptr.as<uint32_t>(), n, g->col.as<uint32_t>(),
-                                              g->wt.as<uint32_t>());
-        count_launch();
-        cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess) st = cuda_fail(e, "graph_from_coo pad", __FILE__, __LINE__);
-    }
+    // pad slots are written by the placement itself (sort.cu k_place)
     if (st != TIGR_OK) { delete g; return st; }
     *out = g;
     return TIGR_OK;

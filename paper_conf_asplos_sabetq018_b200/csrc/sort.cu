@@ -169,6 +169,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
     // arcs whose source lies outside [klo, khi) are dropped (partitioned builds)
     uint32_t key[SI];
     uint32_t valid = 0;  // FILT: bit r = item r of this thread passed the filter
+    const bool fwd_tile = base + (uint64_t)(kST * SI) <= m;  // FIRST: no reversed item in this tile
     auto keep = [&](int r) -> bool {
         if constexpr (FILT) return (valid >> r) & 1u;
         else return (uint32_t)(wp * (SI * 32) + r * 32 + lane) < cnt;
@@ -180,7 +181,9 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         key[r] = 0;
         if (li < cnt) {
             if constexpr (FIRST) {
-                const bool rev = idx >= m;
+                // a tile wholly before the reversed half (every tile without symmetrising) reads
+                // the arc list straight; only tiles that reach into it select per item
+                const bool rev = !fwd_tile && idx >= m;
                 const uint64_t f = rev ? idx - m : idx;
                 key[r] = rev ? dst[f] : src[f];
                 if (!FILT || (key[r] >= klo && key[r] < khi)) {
@@ -356,7 +359,19 @@ __global__ void k_deg_from_runs(const uint32_t* __restrict__ start, const uint32
     if (v < n) deg[v] = end[v] - start[v];
 }
 
-// sorted arcs -> padded, 32-byte-aligned segments
+// sorted arcs -> padded, 32-byte-aligned segments.  The thread that places a node's last arc
+// (the next sorted key differs) also fills the node's pad slots up to its next span boundary
+// (pads = kPad, weight 0), so no separate padding pass runs.
+template <bool W>
+__device__ __forceinline__ void place_pads(uint32_t v, uint64_t pos, const uint32_t* __restrict__ cptr,
+                                           uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
+    const uint64_t end = (uint64_t)__ldg(cptr + v + 1) * kSpan;
+    for (uint64_t q = pos + 1; q < end; ++q) {
+        col[q] = kPad;
+        if constexpr (W) wt[q] = 0;
+    }
+}
+
 template <bool W>
 __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>::T* __restrict__ val, uint64_t M,
                         const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ cptr,
@@ -367,6 +382,7 @@ __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>
     for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < M4; g += (uint64_t)gridDim.x * blockDim.x) {
         const uint4 k4 = reinterpret_cast<const uint4*>(key)[g];
         const uint32_t v[4] = {k4.x, k4.y, k4.z, k4.w};
+        const uint32_t after = 4 * g + 4 < M ? __ldg(key + 4 * g + 4) : kPad;  // key past this group
         VT x[4];
         uint64_t base[4];
 #pragma unroll
@@ -379,6 +395,7 @@ __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>
             const uint64_t pos = base[q] + 4 * g + q;
             col[pos] = (uint32_t)x[q];
             if constexpr (W) wt[pos] = (uint32_t)(x[q] >> 32);
+            if ((q < 3 ? v[q + 1] : after) != v[q]) place_pads<W>(v[q], pos, cptr, col, wt);
         }
     }
     for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
@@ -388,6 +405,7 @@ __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>
         const VT x = val[i];
         col[pos] = (uint32_t)x;
         if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
+        if (i + 1 == M || key[i + 1] != v) place_pads<W>(v, pos, cptr, col, wt);
     }
 }
 
