@@ -132,9 +132,32 @@ __device__ __forceinline__ void cp_async4(void* smem_dst, const void* gsrc) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" :: "r"(d), "l"(gsrc) : "memory");
 }
 
+// Bulk (TMA-engine) tile staging: one thread arms an mbarrier with the byte count and issues a
+// single cp.async.bulk per array; the other threads wait on the barrier's phase 0.
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" :: "r"((uint32_t)__cvta_generic_to_shared(bar)) : "memory");
+}
+
+__device__ __forceinline__ void bulk_load(void* smem_dst, const void* gsrc, uint32_t bytes, uint64_t* bar) {
+    const uint32_t b = (uint32_t)__cvta_generic_to_shared(bar);
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(b), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"((uint32_t)__cvta_generic_to_shared(smem_dst)), "l"(gsrc), "r"(bytes), "r"(b) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait0(uint64_t* bar) {
+    const uint32_t b = (uint32_t)__cvta_generic_to_shared(bar);
+    uint32_t done = 0;
+    while (!done)
+        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(done) : "r"(b) : "memory");
+}
+
 // One pass of the stable LSD radix sort over a tile of 4096 arcs.  Values are staged into
-// shared memory with cp.async as soon as the tile is known (no registers held across the
-// ranking / look-back); keys stay in registers; digits are recomputed from the keys.
+// shared memory as soon as the tile is known (no registers held across the ranking /
+// look-back); keys stay in registers; digits are recomputed from the keys.  A full tile whose
+// arrays are contiguous and 16-byte aligned (bulk_ok) is staged with two bulk copies (keys via
+// s_key, which is free until the reorder); other tiles with per-item 4-byte cp.async.
 template <bool W, bool FIRST, int SI, bool FILT>
 __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_onesweep(const uint32_t* __restrict__ kin,
                                                   const typename ValT<W>::T* __restrict__ vin,
@@ -143,7 +166,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
                                                   int bits, const uint64_t* __restrict__ digit_base,
                                                   uint64_t* status, uint32_t* tile_counter, uint64_t epoch,
                                                   uint32_t* __restrict__ kout, typename ValT<W>::T* __restrict__ vout,
-                                                  uint32_t klo, uint32_t khi) {
+                                                  uint32_t klo, uint32_t khi, int bulk_ok) {
     typedef typename ValT<W>::T VT;
     extern __shared__ __align__(16) unsigned char smem[];
     VT* s_vin = reinterpret_cast<VT*>(smem);                                   // tile values, input order
@@ -154,9 +177,17 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
     __shared__ uint64_t s_gofs[kMaxRadix];
     __shared__ uint32_t s_tile;
     __shared__ uint32_t s_wsum[kSW];
+    __shared__ __align__(8) uint64_t s_bar[2];  // bulk staging: keys, values
 
     const int t = threadIdx.x, lane = t & 31, wp = t >> 5;
-    if (t == 0) s_tile = atomicAdd(tile_counter, 1u);
+    if (t == 0) {
+        s_tile = atomicAdd(tile_counter, 1u);
+        if (bulk_ok) {
+            mbar_init(&s_bar[0]);
+            mbar_init(&s_bar[1]);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+    }
     for (int i = t; i < kSW * (kMaxRadix + 1); i += kST) (&s_wcnt[0][0])[i] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
@@ -174,6 +205,17 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         if constexpr (FILT) return (valid >> r) & 1u;
         else return (uint32_t)(wp * (SI * 32) + r * 32 + lane) < cnt;
     };
+    const bool bulk = bulk_ok && cnt == (uint32_t)(kST * SI) && (!FIRST || (!W && !FILT && fwd_tile));
+    if (bulk) {
+        if (t == 0) {
+            bulk_load(s_key, FIRST ? src + base : kin + base, sizeof(uint32_t) * (kST * SI), &s_bar[0]);
+            bulk_load(s_vin, FIRST ? reinterpret_cast<const VT*>(dst + base) : vin + base, sizeof(VT) * (kST * SI),
+                      &s_bar[1]);
+        }
+        mbar_wait0(&s_bar[0]);
+#pragma unroll
+        for (int r = 0; r < SI; ++r) key[r] = s_key[wp * (SI * 32) + r * 32 + lane];
+    } else
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
         const uint32_t li = wp * (SI * 32) + r * 32 + lane;
@@ -257,7 +299,8 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         s_dstart[t] = wofs + v - tile_cnt;
         if (FILT && t == kST - 1) s_dstart[kMaxRadix] = wofs + v;  // the tile's kept items
     }
-    asm volatile("cp.async.wait_all;" ::: "memory");
+    if (bulk) mbar_wait0(&s_bar[1]);
+    else asm volatile("cp.async.wait_all;" ::: "memory");
     __syncthreads();
     // reorder the tile by digit in shared memory (needs no global offset: done before the
     // look-back, so that the predecessors have had that much longer to publish)
@@ -525,7 +568,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     for (int p = 0; p < passes && M; ++p) {
         void (*kern)(const uint32_t*, const VT*, const uint32_t*, const uint32_t*, const uint32_t*, uint64_t,
                      uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*, uint64_t, uint32_t*, VT*, uint32_t,
-                     uint32_t);
+                     uint32_t, int);
         switch (SI) {
             case 12: kern = p == 0 ? &k_onesweep<W, true, 12, false> : &k_onesweep<W, false, 12, false>; break;
             case 20: kern = p == 0 ? &k_onesweep<W, true, 20, false> : &k_onesweep<W, false, 20, false>; break;
@@ -539,10 +582,14 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
         const uint64_t Mp = (p == 0) ? M : Mloc;  // the first pass reads (and filters) the full list
         const uint64_t tp = (Mp + tile_items - 1) / tile_items;
         if (tp == 0) break;
+        // bulk tile staging needs 16-byte aligned sources (the arc arrays of the first pass may
+        // be caller pointers); development builds can turn it off with TIGR_SORT_BULK=0
+        const uintptr_t al = p == 0 ? ((uintptr_t)src | (uintptr_t)dst) : ((uintptr_t)kb[cur].p | (uintptr_t)vb[cur].p);
+        const int bulk_ok = (al & 15) == 0 && dev_knob("TIGR_SORT_BULK", 1) != 0;
         kern<<<(unsigned)tp, kST, smem, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), src, dst, w, m, Mp, p * bits,
                                              bits, dbase.as<uint64_t>() + p * kMaxRadix, status.as<uint64_t>(),
                                              counters.as<uint32_t>() + p, (uint64_t)(p + 1), kb[out].as<uint32_t>(),
-                                             vb[out].as<VT>(), klo, khi);
+                                             vb[out].as<VT>(), klo, khi, bulk_ok);
         TIGR_CKL("onesweep");
         trace(s, "sort: onesweep pass");
         cur = out;
