@@ -119,7 +119,7 @@ struct tigr_graph {
     tigr::DevBuf col;        // uint32[4 * nchunks], padded segments, pads = 0xFFFFFFFF
     tigr::DevBuf wt;         // uint32[4 * nchunks] or empty
     // in-degree sketch from the arc-list scan (PageRank accumulator order, pr.cu)
-    tigr::DevBuf in_flag;    // uint8[n]: node has an in-arc
+    tigr::DevBuf in_flag;    // uint32[n/32 + 1] bitmap: node has an in-arc
     tigr::DevBuf in_sample;  // uint32[n]: in-arcs among every 16th arc
     bool has_in_sketch = false;
     // transposed graphs (tigr_graph_transpose): arcs reversed; src_deg = out-degrees of the

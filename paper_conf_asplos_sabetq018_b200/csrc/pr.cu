@@ -31,29 +31,29 @@ __global__ void k_hot_sample(const uint4* __restrict__ c4, uint64_t nchunks, uin
 namespace {
 
 
-__global__ void k_indeg_flag(const uint4* __restrict__ c4, uint64_t nchunks, uint8_t* __restrict__ flag) {
+__global__ void k_indeg_flag(const uint4* __restrict__ c4, uint64_t nchunks, uint32_t* __restrict__ flag) {
     for (uint64_t k = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nchunks;
          k += (uint64_t)gridDim.x * blockDim.x) {
         // test before setting: hot targets would otherwise serialise millions of stores on one
         // L2 sector; a (possibly stale) read of 1 skips the store, a stale 0 only repeats it
         const uint4 c = ldg_chunk(c4 + k);
         const uint32_t t4[4] = {c.x, c.y, c.z, c.w};
-        uint8_t f[4];
+        uint32_t f[4];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) f[q] = t4[q] != kPad ? flag[t4[q]] : 1;
+        for (int q = 0; q < 4; ++q) f[q] = t4[q] != kPad ? flag[t4[q] >> 5] & (1u << (t4[q] & 31)) : 1u;
 #pragma unroll
         for (int q = 0; q < 4; ++q)
-            if (!f[q]) flag[t4[q]] = 1;
+            if (!f[q]) atomicOr(flag + (t4[q] >> 5), 1u << (t4[q] & 31));
     }
 }
 
 // sort key: vertices with in-arcs first, by decreasing floor(log2(sampled count)); ties by id
-__global__ void k_pr_key(const uint8_t* __restrict__ flag, const uint32_t* __restrict__ cnt, uint32_t n,
+__global__ void k_pr_key(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ cnt, uint32_t n,
                          uint32_t* __restrict__ key, uint32_t* __restrict__ ids, uint32_t* __restrict__ n_in) {
     const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
     bool in = false;
     if (v < n) {
-        in = flag[v] != 0;
+        in = (flag[v >> 5] >> (v & 31)) & 1u;
         const uint32_t c = cnt[v];
         const uint32_t b = c ? 32u - __clz(c) : 0u;  // 0..32
         key[v] = in ? 32u - b : 33u;                 // 0..33
@@ -224,20 +224,21 @@ tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s) {
     TIGR_TRY(nin.alloc(sizeof(uint32_t), s));
     TIGR_CK(cudaMemsetAsync(nin.p, 0, sizeof(uint32_t), s));
     const uint4* c4 = g->col.as<uint4>();
-    const uint8_t* flag = g->in_flag.as<uint8_t>();
+    const uint32_t* flag = g->in_flag.as<uint32_t>();
     const uint32_t* cnt = g->in_sample.as<uint32_t>();
     if (!g->has_in_sketch) {  // graph built from a CSR: sketch the in-degrees from the arc array
-        TIGR_TRY(flag_t.alloc(n ? n : 1, s));
+        const size_t fw = ((size_t)n + 31) / 32 + 1;  // bitmap words
+        TIGR_TRY(flag_t.alloc(sizeof(uint32_t) * fw, s));
         TIGR_TRY(cnt_t.alloc(sizeof(uint32_t) * (n ? n : 1), s));
-        TIGR_CK(cudaMemsetAsync(flag_t.p, 0, n, s));
+        TIGR_CK(cudaMemsetAsync(flag_t.p, 0, sizeof(uint32_t) * fw, s));
         TIGR_CK(cudaMemsetAsync(cnt_t.p, 0, sizeof(uint32_t) * n, s));
         if (g->nchunks) {
-            k_indeg_flag<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, flag_t.as<uint8_t>());
+            k_indeg_flag<<<grid_cap(g->nchunks, 16), kBlock, 0, s>>>(c4, g->nchunks, flag_t.as<uint32_t>());
             TIGR_CKL("pr indeg flag");
             k_hot_sample<<<grid_cap(g->nchunks / 16 + 1, 16), kBlock, 0, s>>>(c4, g->nchunks, cnt_t.as<uint32_t>());
             TIGR_CKL("pr sample");
         }
-        flag = flag_t.as<uint8_t>();
+        flag = flag_t.as<uint32_t>();
         cnt = cnt_t.as<uint32_t>();
     }
     trace(s, "pr cid: sketch");

@@ -51,15 +51,16 @@ __device__ __forceinline__ void coo_item(const uint32_t* __restrict__ src, const
 
 // One read of the arc list before sorting: the digit histograms of every pass, the largest id
 // (validation: checked on the host before any id is used as an index), and optionally the
-// in-degree sketch the PageRank accumulator order uses (pr.cu): a has-in-arcs flag per node
-// (tested before set, so hub targets do not serialise stores) and an in-degree count sampled
+// in-degree sketch the PageRank accumulator order uses (pr.cu): a has-in-arcs bit per node
+// (a 2 MB bitmap at scale 24, tested before set, so hub targets do not serialise; measured
+// 0.6 ms of the cfg4 build as a byte per node) and an in-degree count sampled
 // on every 16th item.  Covers the input arcs f in [f0, f1) -- the host-input build scans each
 // chunk as its copy lands (api.cu) -- and, when symmetrising (sym), their reversed items
 // m + f too.  Item e: key = source, t = target.
 __global__ void k_coo_scan(const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst, uint64_t m,
                            uint64_t f0, uint64_t f1, int sym, int passes, int bits,
                            unsigned long long* __restrict__ hist, uint32_t* __restrict__ maxid, uint32_t n,
-                           uint8_t* __restrict__ in_flag, uint32_t* __restrict__ in_sample, uint32_t klo,
+                           uint32_t* __restrict__ in_flag, uint32_t* __restrict__ in_sample, uint32_t klo,
                            uint32_t khi, unsigned long long* __restrict__ n_local) {
     // one arc per thread and step: measured faster (1.40 ms at cfg4) than 8 arcs per step with
     // 16-byte loads (1.59 ms; 40 registers, occupancy 97 -> 65 %): the scan is bound by the
@@ -80,7 +81,8 @@ __global__ void k_coo_scan(const uint32_t* __restrict__ src, const uint32_t* __r
                 for (int p = 0; p < passes; ++p) atomicAdd(&h[p][(k >> (p * bits)) & mask], 1u);
             }
             if (in_flag && t < n) {
-                if (!in_flag[t]) in_flag[t] = 1;
+                const uint32_t bit = 1u << (t & 31);  // test first: hub targets are set once
+                if (!(in_flag[t >> 5] & bit)) atomicOr(in_flag + (t >> 5), bit);
                 if ((e & 15) == 0) atomicAdd(in_sample + t, 1u);
             }
         }
@@ -151,6 +153,22 @@ __device__ __forceinline__ void mbar_wait0(uint64_t* bar) {
     while (!done)
         asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], 0; selp.u32 %0, 1, 0, p; }"
                      : "=r"(done) : "r"(b) : "memory");
+}
+
+// Lanes of the warp holding the same digit (and the same validity): one ballot per digit bit
+// instead of match.any, whose result latency stalled every ranking round.
+__device__ __forceinline__ uint32_t match_digit(uint32_t d, int nbits, bool valid) {
+    uint32_t m = __ballot_sync(0xffffffffu, valid);
+    m = valid ? m : ~m;
+#pragma unroll
+    for (int b = 0; b < 8; ++b) {
+        if (b < nbits) {
+            const bool on = (d >> b) & 1u;
+            const uint32_t v = __ballot_sync(0xffffffffu, on);
+            m &= on ? v : ~v;
+        }
+    }
+    return m;
 }
 
 // One pass of the stable LSD radix sort over a tile of 4096 arcs.  Values are staged into
@@ -257,8 +275,9 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
     uint32_t rank[SI / 2];  // two 16-bit ranks per register
 #pragma unroll
     for (int r = 0; r < SI; ++r) {
-        const uint32_t d = keep(r) ? (key[r] >> shift) & mask : (uint32_t)radix;
-        peers[r] = __match_any_sync(0xffffffffu, d);
+        const bool kr = keep(r);
+        const uint32_t d = kr ? (key[r] >> shift) & mask : (uint32_t)radix;
+        peers[r] = match_digit(d, bits, kr);
         uint32_t got = 0;
         if ((peers[r] & lt) == 0) got = atomicAdd(&s_wcnt[wp][d], (uint32_t)__popc(peers[r]));
         if (r & 1) rank[r >> 1] |= got << 16; else rank[r >> 1] = got;
@@ -483,7 +502,7 @@ cudaStream_t copy_stream() {
 template <bool W>
 tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* w, uint64_t m, uint64_t M,
                       uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out, bool validate,
-                      uint8_t* in_flag = nullptr, uint32_t* in_sample = nullptr, uint32_t klo = 0,
+                      uint32_t* in_flag = nullptr, uint32_t* in_sample = nullptr, uint32_t klo = 0,
                       uint32_t khi = 0xFFFFFFFFu, uint64_t* M_out = nullptr, const HostArcs* host = nullptr) {
     typedef typename ValT<W>::T VT;
     int key_bits = 0;
@@ -610,11 +629,12 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     uint64_t M = Mall;
     TmpBuf keys, vals;
     keys.s = vals.s = s;
-    TIGR_TRY(g->in_flag.alloc(n ? n : 1, s));
+    const size_t fw = ((size_t)n + 31) / 32 + 1;  // in_flag bitmap words
+    TIGR_TRY(g->in_flag.alloc(sizeof(uint32_t) * fw, s));
     TIGR_TRY(g->in_sample.alloc(sizeof(uint32_t) * (n ? n : 1), s));
-    TIGR_CK(cudaMemsetAsync(g->in_flag.p, 0, n, s));
+    TIGR_CK(cudaMemsetAsync(g->in_flag.p, 0, sizeof(uint32_t) * fw, s));
     TIGR_CK(cudaMemsetAsync(g->in_sample.p, 0, sizeof(uint32_t) * n, s));
-    TIGR_TRY(sort_arcs<W>(src, dst, w, m, Mall, n, s, keys, vals, true, g->in_flag.as<uint8_t>(),
+    TIGR_TRY(sort_arcs<W>(src, dst, w, m, Mall, n, s, keys, vals, true, g->in_flag.as<uint32_t>(),
                           g->in_sample.as<uint32_t>(), klo, khi, &M, host));
     g->has_in_sketch = true;
     g->m = M;  // arcs of this build's source range (all arcs unless partitioned)
