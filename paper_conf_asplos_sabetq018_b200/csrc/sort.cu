@@ -8,9 +8,9 @@
 // warp match-any (stable), the tile's per-digit offsets come from a decoupled look-back over
 // the preceding tiles, and the tile is written back grouped by digit (coalesced runs).
 // No global atomics on the keys themselves, so the heavy skew of power-law sources (the
-// hottest vertex owns 0.14% of all arcs at scale 24) costs nothing.  Degrees come from the
-// run boundaries of the sorted keys; a final kernel places each arc into the 32-byte-aligned,
-// padded segment of its source.
+// hottest vertex owns 0.14% of all arcs at scale 24) costs nothing.  The last pass also
+// counts the degrees from the runs of equal keys in its tiles; a final kernel places each arc
+// into the 32-byte-aligned, padded segment of its source.
 #include <algorithm>
 #include <cstdlib>
 #include <map>
@@ -184,7 +184,8 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
                                                   int bits, const uint64_t* __restrict__ digit_base,
                                                   uint64_t* status, uint32_t* tile_counter, uint64_t epoch,
                                                   uint32_t* __restrict__ kout, typename ValT<W>::T* __restrict__ vout,
-                                                  uint32_t klo, uint32_t khi, int bulk_ok) {
+                                                  uint32_t klo, uint32_t khi, int bulk_ok,
+                                                  uint32_t* __restrict__ deg) {
     typedef typename ValT<W>::T VT;
     extern __shared__ __align__(16) unsigned char smem[];
     VT* s_vin = reinterpret_cast<VT*>(smem);                                   // tile values, input order
@@ -377,48 +378,18 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
             const uint64_t pos = s_gofs[d] + (i - s_dstart[d]);
             kout[pos] = k;
             vout[pos] = s_val[i];
-        }
-    }
-}
-
-// degrees from the runs of the sorted keys: start/end of each present key
-__global__ void k_runs(const uint32_t* __restrict__ key, uint64_t M, uint32_t* __restrict__ start,
-                       uint32_t* __restrict__ end) {
-    // four keys per thread and step (one 16-byte load; neighbours across the group from the
-    // adjacent lanes' registers, the first / last lane reads one extra key)
-    const uint64_t M4 = M / 4;
-    const int lane = threadIdx.x & 31;
-    for (uint64_t b = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); b < M4;
-         b += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t g = b + lane;
-        uint4 k4 = make_uint4(0, 0, 0, 0);
-        if (g < M4) k4 = reinterpret_cast<const uint4*>(key)[g];
-        uint32_t prev = __shfl_up_sync(0xffffffffu, k4.w, 1);
-        uint32_t next = __shfl_down_sync(0xffffffffu, k4.x, 1);
-        if (g < M4) {
-            const uint64_t i0 = 4 * g;
-            if (lane == 0) prev = i0 ? key[i0 - 1] : ~k4.x;
-            if (lane == 31 || g + 1 == M4) next = (i0 + 4 < M) ? key[i0 + 4] : ~k4.w;
-            const uint32_t k[6] = {prev, k4.x, k4.y, k4.z, k4.w, next};
-#pragma unroll
-            for (int q = 1; q <= 4; ++q) {
-                if (k[q - 1] != k[q]) start[k[q]] = (uint32_t)(i0 + q - 1);
-                if (k[q + 1] != k[q]) end[k[q]] = (uint32_t)(i0 + q);
+            // last pass (deg != nullptr): the tile's input is sorted by the lower digits and the
+            // stable rank adds the top one, so s_key is sorted by the whole key -- equal keys are
+            // runs.  A run [i0, i1] adds i1 + 1 - i0 to its key's degree as +(i1 + 1) from its
+            // last item and -i0 from its first (one atomic for a run of one); a key whose run
+            // spans tiles collects one such pair per tile.
+            if (deg) {
+                const bool first = i == 0 || s_key[i - 1] != k;
+                const bool last = i + 1 == nvalid || s_key[i + 1] != k;
+                if (first || last) atomicAdd(deg + k, (last ? i + 1 : 0u) - (first ? i : 0u));
             }
         }
     }
-    for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t k = key[i];
-        if (i == 0 || key[i - 1] != k) start[k] = (uint32_t)i;
-        if (i + 1 == M || key[i + 1] != k) end[k] = (uint32_t)(i + 1);
-    }
-}
-
-__global__ void k_deg_from_runs(const uint32_t* __restrict__ start, const uint32_t* __restrict__ end, uint32_t n,
-                                uint32_t* __restrict__ deg) {
-    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
-    if (v < n) deg[v] = end[v] - start[v];
 }
 
 // sorted arcs -> padded, 32-byte-aligned segments.  The thread that places a node's last arc
@@ -503,7 +474,8 @@ template <bool W>
 tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* w, uint64_t m, uint64_t M,
                       uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out, bool validate,
                       uint32_t* in_flag = nullptr, uint32_t* in_sample = nullptr, uint32_t klo = 0,
-                      uint32_t khi = 0xFFFFFFFFu, uint64_t* M_out = nullptr, const HostArcs* host = nullptr) {
+                      uint32_t khi = 0xFFFFFFFFu, uint64_t* M_out = nullptr, const HostArcs* host = nullptr,
+                      uint32_t* deg = nullptr) {
     typedef typename ValT<W>::T VT;
     int key_bits = 0;
     while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
@@ -587,7 +559,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     for (int p = 0; p < passes && M; ++p) {
         void (*kern)(const uint32_t*, const VT*, const uint32_t*, const uint32_t*, const uint32_t*, uint64_t,
                      uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*, uint64_t, uint32_t*, VT*, uint32_t,
-                     uint32_t, int);
+                     uint32_t, int, uint32_t*);
         switch (SI) {
             case 12: kern = p == 0 ? &k_onesweep<W, true, 12, false> : &k_onesweep<W, false, 12, false>; break;
             case 20: kern = p == 0 ? &k_onesweep<W, true, 20, false> : &k_onesweep<W, false, 20, false>; break;
@@ -608,7 +580,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
         kern<<<(unsigned)tp, kST, smem, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), src, dst, w, m, Mp, p * bits,
                                              bits, dbase.as<uint64_t>() + p * kMaxRadix, status.as<uint64_t>(),
                                              counters.as<uint32_t>() + p, (uint64_t)(p + 1), kb[out].as<uint32_t>(),
-                                             vb[out].as<VT>(), klo, khi, bulk_ok);
+                                             vb[out].as<VT>(), klo, khi, bulk_ok, p == passes - 1 ? deg : nullptr);
         TIGR_CKL("onesweep");
         trace(s, "sort: onesweep pass");
         cur = out;
@@ -634,24 +606,13 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     TIGR_TRY(g->in_sample.alloc(sizeof(uint32_t) * (n ? n : 1), s));
     TIGR_CK(cudaMemsetAsync(g->in_flag.p, 0, sizeof(uint32_t) * fw, s));
     TIGR_CK(cudaMemsetAsync(g->in_sample.p, 0, sizeof(uint32_t) * n, s));
+    // degrees: counted by the last radix pass from the runs of equal keys in its tiles
+    TIGR_TRY(g->deg.alloc(sizeof(uint32_t) * (n ? n : 1), s));
+    TIGR_CK(cudaMemsetAsync(g->deg.p, 0, sizeof(uint32_t) * n, s));
     TIGR_TRY(sort_arcs<W>(src, dst, w, m, Mall, n, s, keys, vals, true, g->in_flag.as<uint32_t>(),
-                          g->in_sample.as<uint32_t>(), klo, khi, &M, host));
+                          g->in_sample.as<uint32_t>(), klo, khi, &M, host, g->deg.as<uint32_t>()));
     g->has_in_sketch = true;
     g->m = M;  // arcs of this build's source range (all arcs unless partitioned)
-    // degrees from runs
-    TmpBuf st, en;
-    TIGR_TRY(st.alloc(sizeof(uint32_t) * n, s));
-    TIGR_TRY(en.alloc(sizeof(uint32_t) * n, s));
-    TIGR_CK(cudaMemsetAsync(st.p, 0, sizeof(uint32_t) * n, s));
-    TIGR_CK(cudaMemsetAsync(en.p, 0, sizeof(uint32_t) * n, s));
-    if (M) {
-        k_runs<<<sort_grid(M), kBlock, 0, s>>>(keys.as<uint32_t>(), M, st.as<uint32_t>(), en.as<uint32_t>());
-        TIGR_CKL("runs");
-    }
-    trace(s, "csr: runs");
-    TIGR_TRY(g->deg.alloc(sizeof(uint32_t) * n, s));
-    k_deg_from_runs<<<grid_for(n), kBlock, 0, s>>>(st.as<uint32_t>(), en.as<uint32_t>(), n, g->deg.as<uint32_t>());
-    TIGR_CKL("deg");
     // node array, padded chunk offsets, edge buffers
     TIGR_TRY(g->row_ptr.alloc(sizeof(int64_t) * ((size_t)n + 1), s));
     TIGR_TRY(exclusive_scan_u64(g->deg.as<uint32_t>(), n, SCAN_U32, 1, reinterpret_cast<uint64_t*>(g->row_ptr.p), s));
