@@ -157,16 +157,19 @@ __device__ __forceinline__ void mbar_wait0(uint64_t* bar) {
 
 // Lanes of the warp holding the same digit (and the same validity): one ballot per digit bit
 // instead of match.any, whose result latency stalled every ranking round.
-__device__ __forceinline__ uint32_t match_digit(uint32_t d, int nbits, bool valid) {
-    uint32_t m = __ballot_sync(0xffffffffu, valid);
-    m = valid ? m : ~m;
+// All 8 bits are tested whatever the digit width (bits above it are 0 in every lane and leave
+// the mask unchanged), so the loop has no predication; the validity ballot is only needed in
+// tiles with dropped or missing items (check, warp-uniform).
+__device__ __forceinline__ uint32_t match_digit(uint32_t d, bool check, bool valid) {
+    uint32_t m = 0xffffffffu;
+    if (check) {
+        const uint32_t v = __ballot_sync(0xffffffffu, valid);
+        m = valid ? v : ~v;
+    }
 #pragma unroll
     for (int b = 0; b < 8; ++b) {
-        if (b < nbits) {
-            const bool on = (d >> b) & 1u;
-            const uint32_t v = __ballot_sync(0xffffffffu, on);
-            m &= on ? v : ~v;
-        }
+        const uint32_t v = __ballot_sync(0xffffffffu, (d >> b) & 1u);
+        m &= ~(v ^ (0u - ((d >> b) & 1u)));  // lanes whose bit b equals this lane's
     }
     return m;
 }
@@ -278,7 +281,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
     for (int r = 0; r < SI; ++r) {
         const bool kr = keep(r);
         const uint32_t d = kr ? (key[r] >> shift) & mask : (uint32_t)radix;
-        peers[r] = match_digit(d, bits, kr);
+        peers[r] = match_digit(d, FILT || cnt < (uint32_t)(kST * SI), kr);
         uint32_t got = 0;
         if ((peers[r] & lt) == 0) got = atomicAdd(&s_wcnt[wp][d], (uint32_t)__popc(peers[r]));
         if (r & 1) rank[r >> 1] |= got << 16; else rank[r >> 1] = got;
