@@ -254,7 +254,8 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     if (use_graph) {
         GraphKey key{algo, vg->layout * 16 + (int)vg->unit,
                      p.fq ? 16 + p.fa.mode * 4 + (int)p.fa.dense_div * 16 + (p.fa.settled ? 1 << 30 : 0) : front,
-                     p.bsp ? 1 : 0, o.collect_stats ? 1 : 0, p.comm ? 1 : 0, vg->lo, vg->hi};
+                     p.bsp ? 1 : 0, o.collect_stats ? 1 : 0, p.comm ? 1 : 0, vg->lo, vg->hi,
+                     p.fq ? (const void*)p.fq : (const void*)p.relax};
         auto itg = ws.graphs.find(key);
         if (itg == ws.graphs.end()) {
             CachedGraph cg;

@@ -30,9 +30,10 @@ struct Ctl {
 struct GraphKey {
     int algo, layout_vec, frontier, schedule, stats, comm;
     uint32_t lo, hi;
+    const void* relax;  // the relax kernel the graph launches (it depends on packed arcs, dev knobs)
     bool operator<(const GraphKey& o) const {
-        return std::tie(algo, layout_vec, frontier, schedule, stats, comm, lo, hi) <
-               std::tie(o.algo, o.layout_vec, o.frontier, o.schedule, o.stats, o.comm, o.lo, o.hi);
+        return std::tie(algo, layout_vec, frontier, schedule, stats, comm, lo, hi, relax) <
+               std::tie(o.algo, o.layout_vec, o.frontier, o.schedule, o.stats, o.comm, o.lo, o.hi, o.relax);
     }
 };
 
