@@ -386,7 +386,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
             // runs.  A run [i0, i1] adds i1 + 1 - i0 to its key's degree as +(i1 + 1) from its
             // last item and -i0 from its first (one atomic for a run of one); a key whose run
             // spans tiles collects one such pair per tile.
-            if (deg) {
+            if (deg && k < khi) {  // khi: the id bound in host-input run builds (ids not yet validated)
                 const bool first = i == 0 || s_key[i - 1] != k;
                 const bool last = i + 1 == nvalid || s_key[i + 1] != k;
                 if (first || last) atomicAdd(deg + k, (last ? i + 1 : 0u) - (first ? i : 0u));
@@ -442,6 +442,69 @@ __global__ void k_place(const uint32_t* __restrict__ key, const typename ValT<W>
         col[pos] = (uint32_t)x;
         if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
         if (i + 1 == M || key[i + 1] != v) place_pads<W>(v, pos, cptr, col, wt);
+    }
+}
+
+// Host-input builds in sorted runs (build_sorted_runs): after chunk c is sorted, its nodes'
+// chunk-local degrees deg_c and their chunk-local run starts start_c (exclusive scan of deg_c)
+// turn into delta_c[v] = (arcs of v in chunks < c) - start_c[v] (mod 2^32), so that the arc at
+// chunk-local sorted index li sits at offset li + delta_c[v] of v's row: chunks are in input
+// order, so the rows stay stable.  D accumulates the degrees; deg_c is cleared for the next chunk.
+__global__ void k_run_delta(uint32_t n, uint32_t* __restrict__ deg_c, const uint32_t* __restrict__ start_c,
+                            uint32_t* __restrict__ D, uint32_t* __restrict__ delta_c) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        const uint32_t pre = D[v];
+        delta_c[v] = pre - start_c[v];
+        D[v] = pre + deg_c[v];
+        deg_c[v] = 0;
+    }
+}
+
+// the sorted runs -> padded segments (k_place with the row offset from the run's delta; the
+// thread placing a node's last arc, offset d_v - 1, fills the node's pad slots)
+template <bool W>
+__global__ void k_place_runs(const uint32_t* __restrict__ key, const typename ValT<W>::T* __restrict__ val,
+                             uint64_t M, uint64_t chunk, uint32_t n, const uint32_t* __restrict__ delta,
+                             const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ cptr,
+                             uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
+    typedef typename ValT<W>::T VT;
+    // four arcs per thread and step (chunk is a multiple of 4: a group never straddles runs)
+    const uint64_t M4 = M / 4;
+    for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < M4; g += (uint64_t)gridDim.x * blockDim.x) {
+        const uint4 k4 = reinterpret_cast<const uint4*>(key)[g];
+        const uint32_t v[4] = {k4.x, k4.y, k4.z, k4.w};
+        const uint64_t c = (4 * g) / chunk;
+        const uint32_t li = (uint32_t)(4 * g - c * chunk);
+        const uint32_t* dl = delta + c * n;
+        VT x[4];
+        uint32_t r[4];
+        uint64_t base[4];
+        int64_t d[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            x[q] = val[4 * g + q];
+            r[q] = li + q + __ldg(dl + v[q]);
+            base[q] = (uint64_t)__ldg(cptr + v[q]) * kSpan;
+            d[q] = __ldg(row_ptr + v[q] + 1) - __ldg(row_ptr + v[q]);
+        }
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const uint64_t pos = base[q] + r[q];
+            col[pos] = (uint32_t)x[q];
+            if constexpr (W) wt[pos] = (uint32_t)(x[q] >> 32);
+            if ((int64_t)r[q] + 1 == d[q]) place_pads<W>(v[q], pos, cptr, col, wt);
+        }
+    }
+    for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = key[i];
+        const uint64_t c = i / chunk;
+        const uint32_t r = (uint32_t)(i - c * chunk) + delta[c * n + v];
+        const uint64_t pos = (uint64_t)cptr[v] * kSpan + r;
+        const VT x = val[i];
+        col[pos] = (uint32_t)x;
+        if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
+        if ((int64_t)r + 1 == row_ptr[v + 1] - row_ptr[v]) place_pads<W>(v, pos, cptr, col, wt);
     }
 }
 
@@ -595,6 +658,130 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     return TIGR_OK;
 }
 
+// Host-input build in sorted runs (tigr_graph_from_coo with host arrays, no symmetrising, no
+// source filter): the arc list arrives in chunks on the copy stream, and each chunk is scanned
+// AND fully radix-sorted on the build stream while the next chunks are still in flight.  A
+// sorted chunk is a stable run; the runs are merged into the rows by k_place_runs (chunk c's
+// arcs of v follow those of chunks < c: input order), so after the last chunk lands only its own
+// sort, the degree scans and the placement remain -- instead of the whole three-pass sort.
+// The result is element-identical to build_sorted's (same canonical stable CSR).
+// Ids are validated (maxid < n) before the placement, the first step that indexes by target;
+// the sort's degree counting skips ids >= n (k_onesweep's khi guard).
+template <bool W>
+tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
+                              cudaStream_t s, tigr_graph* g, const HostArcs* host, uint64_t chunk) {
+    typedef typename ValT<W>::T VT;
+    int key_bits = 0;
+    while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
+    const int passes = key_bits == 0 ? 1 : (key_bits + 7) / 8;
+    const int bits = key_bits == 0 ? 1 : (key_bits + passes - 1) / passes;
+    constexpr int SI = 16;
+    const uint64_t tile_items = (uint64_t)kST * SI;
+    const uint64_t nch = (m + chunk - 1) / chunk;
+    const uint64_t ctiles = (chunk + tile_items - 1) / tile_items;
+    if (nch * passes >= 0xFFFF) return fail(TIGR_ERANGE, "graph_from_coo: too many copy chunks");
+
+    TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid, nloc, deg_c, start_c, delta;
+    for (int i = 0; i < 2; ++i) {
+        TIGR_TRY(kb[i].alloc(sizeof(uint32_t) * m, s));
+        TIGR_TRY(vb[i].alloc(sizeof(VT) * m, s));
+    }
+    TIGR_TRY(hist.alloc(sizeof(unsigned long long) * 4 * kMaxRadix * nch, s));
+    TIGR_TRY(dbase.alloc(sizeof(uint64_t) * 4 * kMaxRadix * nch, s));
+    TIGR_TRY(status.alloc(sizeof(uint64_t) * kMaxRadix * ctiles, s));
+    TIGR_TRY(counters.alloc(sizeof(uint32_t) * 4 * nch, s));
+    TIGR_TRY(maxid.alloc(sizeof(uint32_t), s));
+    TIGR_TRY(nloc.alloc(sizeof(unsigned long long), s));
+    TIGR_TRY(deg_c.alloc(sizeof(uint32_t) * n, s));
+    TIGR_TRY(start_c.alloc(sizeof(uint32_t) * ((size_t)n + 1), s));
+    TIGR_TRY(delta.alloc(sizeof(uint32_t) * n * nch, s));
+    TIGR_CK(cudaMemsetAsync(hist.p, 0, sizeof(unsigned long long) * 4 * kMaxRadix * nch, s));
+    TIGR_CK(cudaMemsetAsync(status.p, 0, sizeof(uint64_t) * kMaxRadix * ctiles, s));  // epoch 0 matches nothing
+    TIGR_CK(cudaMemsetAsync(counters.p, 0, sizeof(uint32_t) * 4 * nch, s));
+    TIGR_CK(cudaMemsetAsync(maxid.p, 0, sizeof(uint32_t), s));
+    TIGR_CK(cudaMemsetAsync(nloc.p, 0, sizeof(unsigned long long), s));
+    TIGR_CK(cudaMemsetAsync(deg_c.p, 0, sizeof(uint32_t) * n, s));
+    uint32_t* D = g->deg.as<uint32_t>();  // zeroed by the caller
+
+    cudaStream_t cs = copy_stream();
+    if (!cs) return fail(TIGR_ECUDA, "graph_from_coo: copy stream creation failed");
+    cudaEvent_t ready;
+    TIGR_CK(cudaEventCreateWithFlags(&ready, cudaEventDisableTiming));
+    TIGR_CK(cudaEventRecord(ready, s));  // the destinations (fresh allocations) are free on s
+    TIGR_CK(cudaStreamWaitEvent(cs, ready, 0));
+    cudaEventDestroy(ready);
+    // every copy is queued up front, so the copy engine never waits for the build stream
+    std::vector<cudaEvent_t> landed(nch);
+    for (uint64_t c = 0; c < nch; ++c) {
+        const uint64_t f0 = c * chunk, f1 = std::min<uint64_t>(m, f0 + chunk);
+        const size_t bytes = sizeof(uint32_t) * (f1 - f0);
+        TIGR_CK(cudaMemcpyAsync(const_cast<uint32_t*>(src) + f0, host->src + f0, bytes, cudaMemcpyHostToDevice, cs));
+        TIGR_CK(cudaMemcpyAsync(const_cast<uint32_t*>(dst) + f0, host->dst + f0, bytes, cudaMemcpyHostToDevice, cs));
+        if (W) TIGR_CK(cudaMemcpyAsync(const_cast<uint32_t*>(w) + f0, host->w + f0, bytes, cudaMemcpyHostToDevice, cs));
+        TIGR_CK(cudaEventCreateWithFlags(&landed[c], cudaEventDisableTiming));
+        TIGR_CK(cudaEventRecord(landed[c], cs));
+    }
+    const size_t smem = (2 * sizeof(VT) + sizeof(uint32_t)) * tile_items;
+    auto k_first = &k_onesweep<W, true, SI, false>;
+    auto k_next = &k_onesweep<W, false, SI, false>;
+    TIGR_CK(cudaFuncSetAttribute(k_first, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    TIGR_CK(cudaFuncSetAttribute(k_next, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    int cur = 0;
+    for (uint64_t c = 0; c < nch; ++c) {
+        const uint64_t f0 = c * chunk, f1 = std::min<uint64_t>(m, f0 + chunk), Mc = f1 - f0;
+        TIGR_CK(cudaStreamWaitEvent(s, landed[c], 0));
+        cudaEventDestroy(landed[c]);  // released once it has completed
+        unsigned long long* hc = hist.as<unsigned long long>() + c * 4 * kMaxRadix;
+        uint64_t* bc = dbase.as<uint64_t>() + c * 4 * kMaxRadix;
+        k_coo_scan<<<sort_grid(Mc), kBlock, 0, s>>>(src, dst, m, f0, f1, 0, passes, bits, hc, maxid.as<uint32_t>(), n,
+                                                     g->in_flag.as<uint32_t>(), g->in_sample.as<uint32_t>(), 0,
+                                                     0xFFFFFFFFu, nloc.as<unsigned long long>());
+        TIGR_CKL("coo scan (run)");
+        k_digit_base<<<1, kMaxRadix, 0, s>>>(hc, passes, bc);
+        TIGR_CKL("digit base (run)");
+        cur = 0;
+        const uint64_t tp = (Mc + tile_items - 1) / tile_items;
+        for (int p = 0; p < passes; ++p) {
+            const int out = (p == 0) ? 0 : 1 - cur;
+            const uintptr_t al = p == 0 ? ((uintptr_t)(src + f0) | (uintptr_t)(dst + f0))
+                                        : ((uintptr_t)(kb[cur].as<uint32_t>() + f0) | (uintptr_t)(vb[cur].as<VT>() + f0));
+            const int bulk_ok = (al & 15) == 0 && dev_knob("TIGR_SORT_BULK", 1) != 0;
+            (p == 0 ? k_first : k_next)<<<(unsigned)tp, kST, smem, s>>>(
+                kb[cur].as<uint32_t>() + f0, vb[cur].as<VT>() + f0, src + f0, dst + f0, W ? w + f0 : nullptr, Mc, Mc,
+                p * bits, bits, bc + p * kMaxRadix, status.as<uint64_t>(), counters.as<uint32_t>() + c * 4 + p,
+                (uint64_t)(c * passes + p + 1), kb[out].as<uint32_t>() + f0, vb[out].as<VT>() + f0, 0, n, bulk_ok,
+                p == passes - 1 ? deg_c.as<uint32_t>() : nullptr);
+            TIGR_CKL("onesweep (run)");
+            cur = out;
+        }
+        TIGR_TRY(exclusive_scan_u32(deg_c.as<uint32_t>(), n, SCAN_U32, 1, start_c.as<uint32_t>(), s, nullptr));
+        k_run_delta<<<grid_for(n), kBlock, 0, s>>>(n, deg_c.as<uint32_t>(), start_c.as<uint32_t>(), D,
+                                                    delta.as<uint32_t>() + c * n);
+        TIGR_CKL("run delta");
+    }
+    uint32_t hmax = 0;
+    TIGR_CK(cudaMemcpyAsync(&hmax, maxid.p, sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    if (hmax >= n) return fail(TIGR_EINVAL, "graph_from_coo: vertex id >= n");
+    g->has_in_sketch = true;
+    g->m = m;
+    TIGR_TRY(g->row_ptr.alloc(sizeof(int64_t) * ((size_t)n + 1), s));
+    TIGR_TRY(exclusive_scan_u64(D, n, SCAN_U32, 1, reinterpret_cast<uint64_t*>(g->row_ptr.p), s));
+    TIGR_TRY(g->cptr.alloc(sizeof(uint32_t) * ((size_t)n + 1), s));
+    uint64_t spans = 0;
+    TIGR_TRY(exclusive_scan_u32(D, n, SCAN_CEIL_DIV, kSpan, g->cptr.as<uint32_t>(), s, &spans));
+    if (spans >= (1ull << 31)) return fail(TIGR_ERANGE, "graph: padded edge spans exceed 2^31");
+    g->nchunks = spans * 2;  // 16-byte chunks
+    TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
+    if (W) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
+    k_place_runs<W><<<sort_grid(m), kBlock, 0, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), m, chunk, n,
+                                                     delta.as<uint32_t>(), g->row_ptr.as<int64_t>(),
+                                                     g->cptr.as<uint32_t>(), g->col.as<uint32_t>(),
+                                                     W ? g->wt.as<uint32_t>() : nullptr);
+    TIGR_CKL("place (runs)");
+    return TIGR_OK;
+}
+
 template <bool W>
 tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
                          int symmetrize, cudaStream_t s, tigr_graph* g, uint32_t klo, uint32_t khi,
@@ -612,6 +799,10 @@ tigr_status build_sorted(uint32_t n, uint64_t m, const uint32_t* src, const uint
     // degrees: counted by the last radix pass from the runs of equal keys in its tiles
     TIGR_TRY(g->deg.alloc(sizeof(uint32_t) * (n ? n : 1), s));
     TIGR_CK(cudaMemsetAsync(g->deg.p, 0, sizeof(uint32_t) * n, s));
+    // host arrays, whole graph, more than one copy chunk: sort the chunks as they land
+    const uint64_t run_chunk = std::max<uint64_t>(kCopyChunk, ((m / 64 + (1u << 20) - 1) >> 20) << 20);
+    if (host && !symmetrize && klo == 0 && khi >= n && m > run_chunk && dev_knob("TIGR_HOST_RUNS", 1))
+        return build_sorted_runs<W>(n, m, src, dst, w, s, g, host, run_chunk);
     TIGR_TRY(sort_arcs<W>(src, dst, w, m, Mall, n, s, keys, vals, true, g->in_flag.as<uint32_t>(),
                           g->in_sample.as<uint32_t>(), klo, khi, &M, host, g->deg.as<uint32_t>()));
     g->has_in_sketch = true;

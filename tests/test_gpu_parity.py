@@ -721,6 +721,29 @@ def test_host_input_multi_chunk(tigr, sym):
     assert np.array_equal(rpd, rp) and np.array_equal(cold, col)
 
 
+def test_host_input_sorted_runs_skewed(tigr):
+    """Host arc lists of more than one copy chunk are sorted chunk by chunk as they land and the
+    sorted runs are merged into the rows (sort.cu build_sorted_runs): three chunks (the last
+    ragged), unweighted, with hub sources whose rows span every chunk and nodes without arcs,
+    must give the oracle's stable CSR; an id >= n in the last chunk is rejected (EINVAL)."""
+    n, m = (1 << 22) + 3, 2 * (1 << 24) + 4099
+    rng = np.random.default_rng(17)
+    src = np.minimum((n * rng.random(m) ** 6).astype(np.uint32), n - 1)  # heavy skew toward 0
+    dst = rng.integers(0, n, m, dtype=np.uint32)
+    g = tigr.tigr_graph_from_coo(n, src, dst, None)
+    rp, col, _ = tigr.tigr_graph_export_csr(g)
+    o = oracle.csr_build(n, src, dst)
+    assert np.array_equal(rp, o.row_ptr) and np.array_equal(col, o.col)
+    # PageRank's in-degree sketch is collected on the same chunked path
+    vg = tigr.tigr_virtualize(g, 8)
+    assert float(np.abs(tigr.tigr_run(vg, "pr") - oracle.pagerank(o, 20)).max()) <= 1e-6
+    bad = dst.copy()
+    bad[-1] = n
+    with pytest.raises(tigr.TigrError) as ei:
+        tigr.tigr_graph_from_coo(n, src, bad, None)
+    assert ei.value.status == tigr.TIGR_EINVAL
+
+
 def test_bytes_alg_byte_model(tigr):
     """tigr_stats.bytes_alg is SURVEY §8(d)'s byte model, computed in the library: PageRank per
     relax launch 20 B/arc + 4 B/virtual node + 20 B per node with arcs (apply fused in), over
