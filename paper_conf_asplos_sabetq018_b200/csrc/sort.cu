@@ -460,13 +460,15 @@ __global__ void k_run_delta(uint32_t n, uint32_t* __restrict__ deg_c, const uint
     }
 }
 
-// the sorted runs -> padded segments (k_place with the row offset from the run's delta; the
-// thread placing a node's last arc, offset d_v - 1, fills the node's pad slots)
+// the sorted runs -> padded segments: the arc at chunk-local sorted index li of chunk c goes to
+// offset li + delta_c[v] of v's row.  Per arc it reads only delta_c[v] and cptr[v] (within a run
+// the keys ascend, so both are swept in order): each chunk touches most nodes, so every other
+// per-node read would be repeated once per chunk.  The pad slots are written by k_pad_runs.
 template <bool W>
 __global__ void k_place_runs(const uint32_t* __restrict__ key, const typename ValT<W>::T* __restrict__ val,
                              uint64_t M, uint64_t chunk, uint32_t n, const uint32_t* __restrict__ delta,
-                             const int64_t* __restrict__ row_ptr, const uint32_t* __restrict__ cptr,
-                             uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
+                             const uint32_t* __restrict__ cptr, uint32_t* __restrict__ col,
+                             uint32_t* __restrict__ wt) {
     typedef typename ValT<W>::T VT;
     // four arcs per thread and step (chunk is a multiple of 4: a group never straddles runs)
     const uint64_t M4 = M / 4;
@@ -477,34 +479,39 @@ __global__ void k_place_runs(const uint32_t* __restrict__ key, const typename Va
         const uint32_t li = (uint32_t)(4 * g - c * chunk);
         const uint32_t* dl = delta + c * n;
         VT x[4];
-        uint32_t r[4];
-        uint64_t base[4];
-        int64_t d[4];
+        uint64_t pos[4];
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
             x[q] = val[4 * g + q];
-            r[q] = li + q + __ldg(dl + v[q]);
-            base[q] = (uint64_t)__ldg(cptr + v[q]) * kSpan;
-            d[q] = __ldg(row_ptr + v[q] + 1) - __ldg(row_ptr + v[q]);
+            pos[q] = (uint64_t)__ldg(cptr + v[q]) * kSpan + (uint32_t)(li + q + __ldg(dl + v[q]));
         }
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
-            const uint64_t pos = base[q] + r[q];
-            col[pos] = (uint32_t)x[q];
-            if constexpr (W) wt[pos] = (uint32_t)(x[q] >> 32);
-            if ((int64_t)r[q] + 1 == d[q]) place_pads<W>(v[q], pos, cptr, col, wt);
+            col[pos[q]] = (uint32_t)x[q];
+            if constexpr (W) wt[pos[q]] = (uint32_t)(x[q] >> 32);
         }
     }
     for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
          i += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t v = key[i];
         const uint64_t c = i / chunk;
-        const uint32_t r = (uint32_t)(i - c * chunk) + delta[c * n + v];
-        const uint64_t pos = (uint64_t)cptr[v] * kSpan + r;
+        const uint64_t pos = (uint64_t)cptr[v] * kSpan + (uint32_t)((uint32_t)(i - c * chunk) + delta[c * n + v]);
         const VT x = val[i];
         col[pos] = (uint32_t)x;
         if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
-        if ((int64_t)r + 1 == row_ptr[v + 1] - row_ptr[v]) place_pads<W>(v, pos, cptr, col, wt);
+    }
+}
+
+// pad slots of every node: from the end of its arcs to its next 32-byte span boundary
+template <bool W>
+__global__ void k_pad_runs(const uint32_t* __restrict__ deg, const uint32_t* __restrict__ cptr, uint32_t n,
+                           uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        const uint64_t end = (uint64_t)cptr[v + 1] * kSpan;
+        for (uint64_t q = (uint64_t)cptr[v] * kSpan + deg[v]; q < end; ++q) {
+            col[q] = kPad;
+            if constexpr (W) wt[q] = 0;
+        }
     }
 }
 
@@ -775,10 +782,12 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
     TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
     if (W) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
     k_place_runs<W><<<sort_grid(m), kBlock, 0, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), m, chunk, n,
-                                                     delta.as<uint32_t>(), g->row_ptr.as<int64_t>(),
-                                                     g->cptr.as<uint32_t>(), g->col.as<uint32_t>(),
-                                                     W ? g->wt.as<uint32_t>() : nullptr);
+                                                     delta.as<uint32_t>(), g->cptr.as<uint32_t>(),
+                                                     g->col.as<uint32_t>(), W ? g->wt.as<uint32_t>() : nullptr);
     TIGR_CKL("place (runs)");
+    k_pad_runs<W><<<grid_for(n), kBlock, 0, s>>>(D, g->cptr.as<uint32_t>(), n, g->col.as<uint32_t>(),
+                                                  W ? g->wt.as<uint32_t>() : nullptr);
+    TIGR_CKL("pads (runs)");
     return TIGR_OK;
 }
 
