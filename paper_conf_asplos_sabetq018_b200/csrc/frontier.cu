@@ -11,7 +11,7 @@ namespace tigr {
 
 namespace {
 constexpr int kFqThreads = 256;
-constexpr int kCompactPer = 8;  // nodes per thread in k_compact
+constexpr int kCompactPer = 8;  // nodes per thread in k_compact (8 or 16)
 constexpr uint32_t kFull = 0xffffffffu;
 }  // namespace
 
@@ -33,26 +33,37 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const stamp_t* __restric
     uint32_t* oo = qo + (uint64_t)slot * n;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     constexpr uint32_t kTileNodes = kFqThreads * kCompactPer;
+    // the thread's stamps: one kCompactPer-byte load when the slot is aligned (n % kCompactPer == 0)
+    const bool vec = (n & (kCompactPer - 1u)) == 0;
     for (uint64_t tile0 = (uint64_t)blockIdx.x * kTileNodes; tile0 < n; tile0 += (uint64_t)gridDim.x * kTileNodes) {
         const uint64_t v0 = tile0 + (uint64_t)threadIdx.x * kCompactPer;
-        uint32_t m[kCompactPer];
-        unsigned long long mine = 0;  // (entries << 32) | vnodes of this thread's nodes
-        // the thread's 8 stamps: one 8-byte load when aligned (n % 8 == 0 keeps slot 1 aligned)
-        stamp_t sb[kCompactPer];
-        if ((n & 7u) == 0 && v0 + kCompactPer <= n) {
-            const uint2 w = __ldg(reinterpret_cast<const uint2*>(st + v0));
+        uint32_t act = 0;  // bit q: node v0 + q is stamped for iteration itn
+        if (vec && v0 + kCompactPer <= n) {
+            uint32_t ww[kCompactPer / 4];
+            if constexpr (kCompactPer == 16) {
+                const uint4 w = __ldg(reinterpret_cast<const uint4*>(st + v0));
+                ww[0] = w.x; ww[1] = w.y; ww[2] = w.z; ww[3] = w.w;
+            } else {
+                const uint2 w = __ldg(reinterpret_cast<const uint2*>(st + v0));
+                ww[0] = w.x; ww[1] = w.y;
+            }
 #pragma unroll
-            for (int q = 0; q < kCompactPer; ++q) sb[q] = (stamp_t)(((q < 4 ? w.x : w.y) >> (8 * (q & 3))) & 0xFFu);
+            for (int q = 0; q < kCompactPer; ++q)
+                if (((ww[q >> 2] >> (8 * (q & 3))) & 0xFFu) == sv) act |= 1u << q;
         } else {
 #pragma unroll
-            for (int q = 0; q < kCompactPer; ++q) sb[q] = v0 + q < n ? __ldg(st + v0 + q) : (stamp_t)0;
+            for (int q = 0; q < kCompactPer; ++q)
+                if (v0 + q < n && __ldg(st + v0 + q) == sv) act |= 1u << q;
         }
+        // a tile without a stamped node costs one barrier (most tiles of a sparse iteration)
+        if (!__syncthreads_or(act != 0)) continue;
+        uint32_t m[kCompactPer];
+        unsigned long long mine = 0;  // (entries << 32) | vnodes of this thread's nodes
 #pragma unroll
         for (int q = 0; q < kCompactPer; ++q) {
-            const uint64_t v = v0 + q;
             m[q] = 0;
-            if (v < n && sb[q] == sv) {
-                const uint4 info = __ldg(vinfo + v);
+            if ((act >> q) & 1u) {
+                const uint4 info = __ldg(vinfo + v0 + q);
                 if (info.w && info.z >= lo && info.z < hi) m[q] = info.w;
             }
             if (m[q]) mine += (1ull << 32) | m[q];
@@ -72,8 +83,8 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const stamp_t* __restric
             s_base = run ? atomicAdd(&ctl->qpack[slot], run) : 0ull;
         }
         __syncthreads();
+        // (s_warp / s_base are next written after the next tile's __syncthreads_or)
         unsigned long long pos = s_base + s_warp[wid] + (inc - mine);
-        __syncthreads();  // s_warp / s_base reused by the next tile
 #pragma unroll
         for (int q = 0; q < kCompactPer; ++q) {
             if (!m[q]) continue;

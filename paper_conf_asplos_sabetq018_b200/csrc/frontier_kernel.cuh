@@ -66,7 +66,6 @@ namespace tigr {
 namespace {
 
 constexpr int kFqThreads = 256;
-constexpr int kCompactPer = 8;  // nodes per thread in k_compact
 constexpr uint32_t kFull = 0xffffffffu;
 
 // largest k in [0, qn) with qo[k] <= t (qo increasing, qo[0] == 0 <= t): 32-ary search, one

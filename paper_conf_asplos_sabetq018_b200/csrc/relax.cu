@@ -370,20 +370,34 @@ __global__ void k_init(int algo, uint32_t n, uint32_t source, uint32_t* __restri
     // reordered graphs (tigr_graph_reorder): the source is an original id, CC labels are
     // original ids (the minimum original id of the component)
     const uint32_t src = cid ? cid[source] : source;
-    const uint32_t v = blockIdx.x * blockDim.x + threadIdx.x;
-    if (v < n) {
+    // four nodes per thread (16-byte value and 4-byte stamp stores) when n % 4 == 0
+    const bool vec = (n & 3u) == 0;
+    const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+    auto init_val = [&](uint32_t v) -> uint32_t {
         uint32_t x = kInf;
         if (algo == TIGR_CC) x = order ? order[v] : v;
         else if (algo == TIGR_SSWP) x = 0;
         if (v == src && algo != TIGR_CC) x = (algo == TIGR_SSWP) ? kInf : 0;
-        val[v] = x;
-        // BFS: the source's level 0 is final from the start; its settled bit (cleared before this
-        // kernel; frontier_kernel.cuh) spares every gather of it -- R-MAT's source is a hub
-        if (settled && v == src && algo == TIGR_BFS) atomicOr(settled + (v >> 5), 1u << (v & 31u));
-        stamp[v] = 0;                                                  // parity 0: never stamped
-        stamp[(uint64_t)n + v] = (algo == TIGR_CC || v == src) ? stamp_of(1) : 0;  // parity 1: it = 1
+        return x;
+    };
+    auto init_stamp1 = [&](uint32_t v) -> uint32_t {  // parity 1: active in iteration 1
+        return (algo == TIGR_CC || v == src) ? stamp_of(1) : 0;
+    };
+    const uint32_t v0 = vec ? 4 * t : t;
+    if (vec && v0 < n) {
+        reinterpret_cast<uint4*>(val)[t] = make_uint4(init_val(v0), init_val(v0 + 1), init_val(v0 + 2), init_val(v0 + 3));
+        reinterpret_cast<uint32_t*>(stamp)[t] = 0u;  // parity 0: never stamped
+        reinterpret_cast<uint32_t*>(stamp + n)[t] = init_stamp1(v0) | (init_stamp1(v0 + 1) << 8) |
+                                                    (init_stamp1(v0 + 2) << 16) | (init_stamp1(v0 + 3) << 24);
+    } else if (!vec && v0 < n) {
+        val[v0] = init_val(v0);
+        stamp[v0] = 0;
+        stamp[(uint64_t)n + v0] = (stamp_t)init_stamp1(v0);
     }
-    if (v == 0) {
+    // BFS: the source's level 0 is final from the start; its settled bit (cleared before this
+    // kernel; frontier_kernel.cuh) spares every gather of it -- R-MAT's source is a hub
+    if (settled && t == 0 && algo == TIGR_BFS && src < n) atomicOr(settled + (src >> 5), 1u << (src & 31u));
+    if (t == 0) {
         ctl->changed = 0; ctl->it = 1; ctl->max_iters = max_iters; ctl->cont = 1; ctl->notconv = 0;
         ctl->xchanged[0] = 0; ctl->xchanged[1] = 0;
         ctl->edges = 0; ctl->updates = 0; ctl->vnodes = 0; ctl->dsum[0] = 0.0; ctl->dsum[1] = 0.0;

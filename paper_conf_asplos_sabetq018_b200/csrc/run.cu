@@ -236,7 +236,7 @@ tigr_status run_frontier(tigr_vgraph* vg, int algo, uint32_t source, const tigr_
     TIGR_CK(cudaEventRecord(t0, s));
     const tigr_graph* gg = vg->g;
     if (p.fq && p.fa.settled) TIGR_CK(cudaMemsetAsync(p.fa.settled, 0, sizeof(uint32_t) * ((size_t)n / 32 + 1), s));
-    k_init<<<grid_for(n), kBlock, 0, s>>>(algo, n, source, p.args.val, p.args.stamp, p.args.ctl, max_iters,
+    k_init<<<grid_for((n & 3u) ? n : n / 4), kBlock, 0, s>>>(algo, n, source, p.args.val, p.args.stamp, p.args.ctl, max_iters,
                                           gg->reordered ? gg->perm_cid.as<uint32_t>() : nullptr,
                                           gg->reordered ? gg->perm_order.as<uint32_t>() : nullptr,
                                           p.fq ? p.fa.settled : nullptr);
