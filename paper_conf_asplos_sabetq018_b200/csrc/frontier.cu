@@ -19,7 +19,7 @@ constexpr uint32_t kFull = 0xffffffffu;
 // queue build: nodes stamped for iteration it + delta that own virtual nodes in [lo, hi)
 // ------------------------------------------------------------------------------------------
 __global__ void __launch_bounds__(kFqThreads) k_compact(const stamp_t* __restrict__ stamp,
-                                                         const uint4* __restrict__ vinfo, uint32_t n, uint32_t lo,
+                                                         const uint32_t* __restrict__ vptr, uint32_t n, uint32_t lo,
                                                          uint32_t hi, Ctl* ctl, uint32_t* __restrict__ qv,
                                                          uint32_t* __restrict__ qo, int delta) {
     __shared__ unsigned long long s_warp[kFqThreads / 32];
@@ -59,12 +59,29 @@ __global__ void __launch_bounds__(kFqThreads) k_compact(const stamp_t* __restric
         if (!__syncthreads_or(act != 0)) continue;
         uint32_t m[kCompactPer];
         unsigned long long mine = 0;  // (entries << 32) | vnodes of this thread's nodes
+        // family sizes m_v = vnode_ptr[v + 1] - vnode_ptr[v] (and the first virtual node, for this
+        // rank's range): the thread's kCompactPer + 1 offsets in vector loads -- in dense
+        // iterations a sweep of the 4-byte offsets instead of one 16-byte vinfo gather per node
+        uint32_t vp[kCompactPer + 1];
+        if (act) {
+            if (v0 + kCompactPer <= n) {  // v0 is a multiple of kCompactPer: aligned
+#pragma unroll
+                for (int h = 0; h < kCompactPer / 4; ++h) {
+                    const uint4 w = __ldg(reinterpret_cast<const uint4*>(vptr + v0) + h);
+                    vp[4 * h] = w.x; vp[4 * h + 1] = w.y; vp[4 * h + 2] = w.z; vp[4 * h + 3] = w.w;
+                }
+                vp[kCompactPer] = __ldg(vptr + v0 + kCompactPer);
+            } else {
+#pragma unroll
+                for (int q = 0; q <= kCompactPer; ++q) vp[q] = v0 + q <= n ? __ldg(vptr + v0 + q) : 0u;
+            }
+        }
 #pragma unroll
         for (int q = 0; q < kCompactPer; ++q) {
             m[q] = 0;
             if ((act >> q) & 1u) {
-                const uint4 info = __ldg(vinfo + v0 + q);
-                if (info.w && info.z >= lo && info.z < hi) m[q] = info.w;
+                const uint32_t f = vp[q], mv = vp[q + 1] - vp[q];
+                if (mv && f >= lo && f < hi) m[q] = mv;
             }
             if (m[q]) mine += (1ull << 32) | m[q];
         }
@@ -201,7 +218,7 @@ tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStrea
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const uint64_t tiles = ((uint64_t)n + kFqThreads * kCompactPer - 1) / (kFqThreads * kCompactPer);
     const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(tiles, (uint64_t)sms * 8));
-    k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<stamp_t>(), vg->vinfo.as<uint4>(), n, vg->lo, vg->hi, ctl,
+    k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<stamp_t>(), vg->vnode_ptr.as<uint32_t>(), n, vg->lo, vg->hi, ctl,
                                           const_cast<uint32_t*>(vg->ws.qv.as<uint32_t>()),
                                           const_cast<uint32_t*>(vg->ws.qo.as<uint32_t>()), delta);
     TIGR_CK(cudaGetLastError());
