@@ -461,44 +461,77 @@ __global__ void k_run_delta(uint32_t n, uint32_t* __restrict__ deg_c, const uint
 }
 
 // the sorted runs -> padded segments: the arc at chunk-local sorted index li of chunk c goes to
-// offset li + delta_c[v] of v's row.  Per arc it reads only delta_c[v] and cptr[v] (within a run
-// the keys ascend, so both are swept in order): each chunk touches most nodes, so every other
-// per-node read would be repeated once per chunk.  The pad slots are written by k_pad_runs.
+// offset li + delta_c[v] of v's row.  Block b owns the arcs [b, b + 1) * kRunArcs of the row space
+// (row_ptr order) and places them from every chunk in turn: chunk c's arcs that land in this
+// window are one contiguous range of its sorted run, found from the window's first and last
+// nodes (their run starts start_c, run lengths and earlier-chunk counts pre_c = start_c + delta_c).
+// So the writes of all chunks to a window happen together and its 32-byte sectors fill up in L2
+// (a sweep of each chunk across all rows wrote every sector once per chunk: 2.3 ms at cfg4), and a
+// hub's row is spread over many blocks.  The pad slots are written by k_pad_runs.
+constexpr uint32_t kRunArcs = 16384;
+constexpr int kMaxRuns = 64;
+
 template <bool W>
 __global__ void k_place_runs(const uint32_t* __restrict__ key, const typename ValT<W>::T* __restrict__ val,
-                             uint64_t M, uint64_t chunk, uint32_t n, const uint32_t* __restrict__ delta,
-                             const uint32_t* __restrict__ cptr, uint32_t* __restrict__ col,
-                             uint32_t* __restrict__ wt) {
+                             uint64_t chunk, uint32_t nch, uint32_t n, uint64_t m, const uint32_t* __restrict__ delta,
+                             const uint32_t* __restrict__ starts, const int64_t* __restrict__ row_ptr,
+                             const uint32_t* __restrict__ cptr, uint32_t* __restrict__ col, uint32_t* __restrict__ wt) {
     typedef typename ValT<W>::T VT;
-    // four arcs per thread and step (chunk is a multiple of 4: a group never straddles runs)
-    const uint64_t M4 = M / 4;
-    for (uint64_t g = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; g < M4; g += (uint64_t)gridDim.x * blockDim.x) {
-        const uint4 k4 = reinterpret_cast<const uint4*>(key)[g];
-        const uint32_t v[4] = {k4.x, k4.y, k4.z, k4.w};
-        const uint64_t c = (4 * g) / chunk;
-        const uint32_t li = (uint32_t)(4 * g - c * chunk);
-        const uint32_t* dl = delta + c * n;
-        VT x[4];
-        uint64_t pos[4];
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            x[q] = val[4 * g + q];
-            pos[q] = (uint64_t)__ldg(cptr + v[q]) * kSpan + (uint32_t)(li + q + __ldg(dl + v[q]));
+    __shared__ uint32_t s_lo[kMaxRuns], s_hi[kMaxRuns];
+    const uint64_t nblk = (m + kRunArcs - 1) / kRunArcs;
+    for (uint64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
+        const uint64_t g0 = b * kRunArcs, g1 = min(m, g0 + kRunArcs);
+        if (threadIdx.x < nch) {
+            // the nodes holding row-space arcs g0 and g1 - 1: last v with row_ptr[v] <= g
+            auto owner = [&](uint64_t g) {
+                uint32_t lo = 0, hi = n;  // row_ptr[lo] <= g < row_ptr[hi]
+                while (hi - lo > 1) {
+                    const uint32_t mid = lo + (hi - lo) / 2;
+                    if ((uint64_t)__ldg(row_ptr + mid) <= g) lo = mid; else hi = mid;
+                }
+                return lo;
+            };
+            const uint32_t vf = owner(g0), vl = owner(g1 - 1);
+            const int64_t r0 = (int64_t)(g0 - (uint64_t)__ldg(row_ptr + vf));
+            const int64_t r1 = (int64_t)(g1 - (uint64_t)__ldg(row_ptr + vl));  // exclusive, in vl's row
+            const uint32_t c = threadIdx.x;
+            const uint32_t* sc = starts + (uint64_t)c * (n + 1);
+            const uint32_t* dl = delta + (uint64_t)c * n;
+            const uint32_t sf = __ldg(sc + vf), df = __ldg(sc + vf + 1) - sf, pf = sf + __ldg(dl + vf);
+            const uint32_t sl = __ldg(sc + vl), dn = __ldg(sc + vl + 1) - sl, pl = sl + __ldg(dl + vl);
+            auto clamp = [](int64_t x, int64_t hi) -> uint32_t { return (uint32_t)(x < 0 ? 0 : (x > hi ? hi : x)); };
+            s_lo[c] = sf + clamp(r0 - (int64_t)pf, (int64_t)df);
+            s_hi[c] = sl + clamp(r1 - (int64_t)pl, (int64_t)dn);
         }
+        __syncthreads();
+        for (uint32_t c = 0; c < nch; ++c) {
+            const uint32_t* kc = key + c * chunk;
+            const VT* vc = val + c * chunk;
+            const uint32_t* dl = delta + (uint64_t)c * n;
+            const uint32_t hi = s_hi[c];
+            for (uint32_t i0 = s_lo[c] + threadIdx.x; i0 < hi; i0 += 4 * blockDim.x) {
+                // four items per thread and step, every load issued before the first store
+                uint32_t v[4];
+                VT x[4];
+                uint64_t pos[4];
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            col[pos[q]] = (uint32_t)x[q];
-            if constexpr (W) wt[pos[q]] = (uint32_t)(x[q] >> 32);
+                for (int q = 0; q < 4; ++q) {
+                    const uint32_t i = i0 + q * blockDim.x;
+                    v[q] = i < hi ? kc[i] : 0u;
+                    x[q] = i < hi ? vc[i] : VT(0);
+                }
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    pos[q] = (uint64_t)__ldg(cptr + v[q]) * kSpan + (uint32_t)(i0 + q * blockDim.x + __ldg(dl + v[q]));
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    if (i0 + q * blockDim.x >= hi) break;
+                    col[pos[q]] = (uint32_t)x[q];
+                    if constexpr (W) wt[pos[q]] = (uint32_t)(x[q] >> 32);
+                }
+            }
         }
-    }
-    for (uint64_t i = 4 * M4 + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < M;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t v = key[i];
-        const uint64_t c = i / chunk;
-        const uint64_t pos = (uint64_t)cptr[v] * kSpan + (uint32_t)((uint32_t)(i - c * chunk) + delta[c * n + v]);
-        const VT x = val[i];
-        col[pos] = (uint32_t)x;
-        if constexpr (W) wt[pos] = (uint32_t)(x >> 32);
+        __syncthreads();  // s_lo / s_hi reused by the next window
     }
 }
 
@@ -686,9 +719,9 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
     const uint64_t tile_items = (uint64_t)kST * SI;
     const uint64_t nch = (m + chunk - 1) / chunk;
     const uint64_t ctiles = (chunk + tile_items - 1) / tile_items;
-    if (nch * passes >= 0xFFFF) return fail(TIGR_ERANGE, "graph_from_coo: too many copy chunks");
+    if (nch > (uint64_t)kMaxRuns || nch * passes >= 0xFFFF) return fail(TIGR_ERANGE, "graph_from_coo: too many copy chunks");
 
-    TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid, nloc, deg_c, start_c, delta;
+    TmpBuf kb[2], vb[2], hist, dbase, status, counters, maxid, nloc, deg_c, delta;
     for (int i = 0; i < 2; ++i) {
         TIGR_TRY(kb[i].alloc(sizeof(uint32_t) * m, s));
         TIGR_TRY(vb[i].alloc(sizeof(VT) * m, s));
@@ -700,8 +733,9 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
     TIGR_TRY(maxid.alloc(sizeof(uint32_t), s));
     TIGR_TRY(nloc.alloc(sizeof(unsigned long long), s));
     TIGR_TRY(deg_c.alloc(sizeof(uint32_t) * n, s));
-    TIGR_TRY(start_c.alloc(sizeof(uint32_t) * ((size_t)n + 1), s));
     TIGR_TRY(delta.alloc(sizeof(uint32_t) * n * nch, s));
+    TmpBuf starts;  // start_c of every chunk: uint32[nch][n + 1]
+    TIGR_TRY(starts.alloc(sizeof(uint32_t) * ((uint64_t)n + 1) * nch, s));
     TIGR_CK(cudaMemsetAsync(hist.p, 0, sizeof(unsigned long long) * 4 * kMaxRadix * nch, s));
     TIGR_CK(cudaMemsetAsync(status.p, 0, sizeof(uint64_t) * kMaxRadix * ctiles, s));  // epoch 0 matches nothing
     TIGR_CK(cudaMemsetAsync(counters.p, 0, sizeof(uint32_t) * 4 * nch, s));
@@ -761,9 +795,9 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
             TIGR_CKL("onesweep (run)");
             cur = out;
         }
-        TIGR_TRY(exclusive_scan_u32(deg_c.as<uint32_t>(), n, SCAN_U32, 1, start_c.as<uint32_t>(), s, nullptr));
-        k_run_delta<<<grid_for(n), kBlock, 0, s>>>(n, deg_c.as<uint32_t>(), start_c.as<uint32_t>(), D,
-                                                    delta.as<uint32_t>() + c * n);
+        uint32_t* sc = starts.as<uint32_t>() + c * ((uint64_t)n + 1);
+        TIGR_TRY(exclusive_scan_u32(deg_c.as<uint32_t>(), n, SCAN_U32, 1, sc, s, nullptr));
+        k_run_delta<<<grid_for(n), kBlock, 0, s>>>(n, deg_c.as<uint32_t>(), sc, D, delta.as<uint32_t>() + c * n);
         TIGR_CKL("run delta");
     }
     uint32_t hmax = 0;
@@ -781,9 +815,11 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
     g->nchunks = spans * 2;  // 16-byte chunks
     TIGR_TRY(g->col.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
     if (W) TIGR_TRY(g->wt.alloc(sizeof(uint32_t) * kChunk * (g->nchunks ? g->nchunks : 1), s));
-    k_place_runs<W><<<sort_grid(m), kBlock, 0, s>>>(kb[cur].as<uint32_t>(), vb[cur].as<VT>(), m, chunk, n,
-                                                     delta.as<uint32_t>(), g->cptr.as<uint32_t>(),
-                                                     g->col.as<uint32_t>(), W ? g->wt.as<uint32_t>() : nullptr);
+    const uint64_t windows = (m + kRunArcs - 1) / kRunArcs;
+    k_place_runs<W><<<(unsigned)std::min<uint64_t>(windows, 1u << 20), kBlock, 0, s>>>(
+        kb[cur].as<uint32_t>(), vb[cur].as<VT>(), chunk, (uint32_t)nch, n, m, delta.as<uint32_t>(),
+        starts.as<uint32_t>(), g->row_ptr.as<int64_t>(), g->cptr.as<uint32_t>(), g->col.as<uint32_t>(),
+        W ? g->wt.as<uint32_t>() : nullptr);
     TIGR_CKL("place (runs)");
     k_pad_runs<W><<<grid_for(n), kBlock, 0, s>>>(D, g->cptr.as<uint32_t>(), n, g->col.as<uint32_t>(),
                                                   W ? g->wt.as<uint32_t>() : nullptr);
