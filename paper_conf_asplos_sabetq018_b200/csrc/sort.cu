@@ -166,11 +166,18 @@ __device__ __forceinline__ uint32_t match_digit(uint32_t d, bool check, bool val
         const uint32_t v = __ballot_sync(0xffffffffu, valid);
         m = valid ? v : ~v;
     }
+    // per bit: the ballot, the lane's bit as a full mask s, and m &= ~(ballot ^ s) in one lop3 --
+    // three instructions once ptxas has loaded the bit predicates (R2P, seven at once); the plain
+    // C++ form compiled to six per bit (shift, mask, compare, mask build, vote, merge)
 #pragma unroll
-    for (int b = 0; b < 8; ++b) {
-        const uint32_t v = __ballot_sync(0xffffffffu, (d >> b) & 1u);
-        m &= ~(v ^ (0u - ((d >> b) & 1u)));  // lanes whose bit b equals this lane's
-    }
+    for (int b = 0; b < 8; ++b)
+        asm("{\n\t.reg .pred p;\n\t.reg .b32 v, s;\n\t"
+            "and.b32 v, %1, %2;\n\t"
+            "setp.ne.u32 p, v, 0;\n\t"
+            "vote.sync.ballot.b32 v, p, 0xffffffff;\n\t"
+            "selp.b32 s, -1, 0, p;\n\t"
+            "lop3.b32 %0, %0, v, s, 0x90;\n\t}"
+            : "+r"(m) : "r"(d), "r"(1u << b));
     return m;
 }
 
