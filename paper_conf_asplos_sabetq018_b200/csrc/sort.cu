@@ -186,7 +186,7 @@ __device__ __forceinline__ uint32_t match_digit(uint32_t d, bool check, bool val
 // look-back); keys stay in registers; digits are recomputed from the keys.  A full tile whose
 // arrays are contiguous and 16-byte aligned (bulk_ok) is staged with two bulk copies (keys via
 // s_key, which is free until the reorder); other tiles with per-item 4-byte cp.async.
-template <bool W, bool FIRST, int SI, bool FILT>
+template <bool W, bool FIRST, int SI, bool FILT, bool DEG>
 __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_onesweep(const uint32_t* __restrict__ kin,
                                                   const typename ValT<W>::T* __restrict__ vin,
                                                   const uint32_t* __restrict__ src, const uint32_t* __restrict__ dst,
@@ -375,7 +375,7 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
             }
             status_store(&status[(uint64_t)tile * kMaxRadix + t], (epoch << 48) | kFlagInc | (excl + tile_cnt));
         }
-        s_gofs[t] = digit_base[t] + excl;
+        s_gofs[t] = digit_base[t] + excl - s_dstart[t];  // output position of tile item i: s_gofs[d] + i
     }
     __syncthreads();
     const uint32_t nvalid = FILT ? s_dstart[kMaxRadix] : cnt;
@@ -385,18 +385,20 @@ __global__ void __launch_bounds__(kST, (SI <= 16 ? TIGR_SORT_MINB : 2)) k_oneswe
         if (i < nvalid) {
             const uint32_t k = s_key[i];
             const uint32_t d = (k >> shift) & mask;
-            const uint64_t pos = s_gofs[d] + (i - s_dstart[d]);
+            const uint64_t pos = s_gofs[d] + i;
             kout[pos] = k;
             vout[pos] = s_val[i];
-            // last pass (deg != nullptr): the tile's input is sorted by the lower digits and the
-            // stable rank adds the top one, so s_key is sorted by the whole key -- equal keys are
-            // runs.  A run [i0, i1] adds i1 + 1 - i0 to its key's degree as +(i1 + 1) from its
-            // last item and -i0 from its first (one atomic for a run of one); a key whose run
+            // last pass with degree counting (DEG): the tile's input is sorted by the lower digits
+            // and the stable rank adds the top one, so s_key is sorted by the whole key -- equal
+            // keys are runs.  A run [i0, i1] adds i1 + 1 - i0 to its key's degree as +(i1 + 1) from
+            // its last item and -i0 from its first (one atomic for a run of one); a key whose run
             // spans tiles collects one such pair per tile.
-            if (deg && k < khi) {  // khi: the id bound in host-input run builds (ids not yet validated)
-                const bool first = i == 0 || s_key[i - 1] != k;
-                const bool last = i + 1 == nvalid || s_key[i + 1] != k;
-                if (first || last) atomicAdd(deg + k, (last ? i + 1 : 0u) - (first ? i : 0u));
+            if constexpr (DEG) {
+                if (k < khi) {  // khi: the id bound in host-input run builds (ids not yet validated)
+                    const bool first = i == 0 || s_key[i - 1] != k;
+                    const bool last = i + 1 == nvalid || s_key[i + 1] != k;
+                    if (first || last) atomicAdd(deg + k, (last ? i + 1 : 0u) - (first ? i : 0u));
+                }
             }
         }
     }
@@ -584,6 +586,20 @@ cudaStream_t copy_stream() {
 }
 
 template <bool W>
+using OnesweepFn = void (*)(const uint32_t*, const typename ValT<W>::T*, const uint32_t*, const uint32_t*,
+                            const uint32_t*, uint64_t, uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*,
+                            uint64_t, uint32_t*, typename ValT<W>::T*, uint32_t, uint32_t, int, uint32_t*);
+
+// the pass kernel: first pass (reads the arc list; optionally filtered by source range), later
+// passes; the degree-counting variant for the last pass of a CSR build
+template <bool W>
+OnesweepFn<W> onesweep_fn(bool first, bool filt, bool deg) {
+    if (first && filt) return deg ? &k_onesweep<W, true, 16, true, true> : &k_onesweep<W, true, 16, true, false>;
+    if (first) return deg ? &k_onesweep<W, true, 16, false, true> : &k_onesweep<W, true, 16, false, false>;
+    return deg ? &k_onesweep<W, false, 16, false, true> : &k_onesweep<W, false, 16, false, false>;
+}
+
+template <bool W>
 tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* w, uint64_t m, uint64_t M,
                       uint32_t n, cudaStream_t s, TmpBuf& keys_out, TmpBuf& vals_out, bool validate,
                       uint32_t* in_flag = nullptr, uint32_t* in_sample = nullptr, uint32_t klo = 0,
@@ -597,8 +613,7 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     // items per thread: 16 (development builds may sweep 12/20/24 with TIGR_SORT_SI; the
     // source-range-filtered first pass exists for 16 only, so filtered builds always use 16)
     const bool filtered = klo != 0 || khi < n;
-    int SI = filtered ? 16 : dev_knob("TIGR_SORT_SI", 16);
-    if (SI != 12 && SI != 20 && SI != 24) SI = 16;
+    constexpr int SI = 16;  // items per thread (a sweep of 12 / 16 / 20 / 24 chose 16)
     const uint64_t tile_items = (uint64_t)kST * SI;
     const uint64_t tiles = (M + tile_items - 1) / tile_items;
 
@@ -670,17 +685,9 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     const size_t smem = (2 * sizeof(VT) + sizeof(uint32_t)) * tile_items;
     int cur = 0;
     for (int p = 0; p < passes && M; ++p) {
-        void (*kern)(const uint32_t*, const VT*, const uint32_t*, const uint32_t*, const uint32_t*, uint64_t,
-                     uint64_t, int, int, const uint64_t*, uint64_t*, uint32_t*, uint64_t, uint32_t*, VT*, uint32_t,
-                     uint32_t, int, uint32_t*);
-        switch (SI) {
-            case 12: kern = p == 0 ? &k_onesweep<W, true, 12, false> : &k_onesweep<W, false, 12, false>; break;
-            case 20: kern = p == 0 ? &k_onesweep<W, true, 20, false> : &k_onesweep<W, false, 20, false>; break;
-            case 24: kern = p == 0 ? &k_onesweep<W, true, 24, false> : &k_onesweep<W, false, 24, false>; break;
-            default: kern = p == 0 ? &k_onesweep<W, true, 16, false> : &k_onesweep<W, false, 16, false>; break;
-        }
-        // partitioned builds: the first pass drops the arcs outside [klo, khi)
-        if (p == 0 && filtered) kern = &k_onesweep<W, true, 16, true>;
+        // partitioned builds: the first pass drops the arcs outside [klo, khi); the last pass
+        // counts the degrees when asked to
+        const auto kern = onesweep_fn<W>(p == 0, p == 0 && filtered, p == passes - 1 && deg != nullptr);
         TIGR_CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         const int out = (p == 0) ? 0 : 1 - cur;
         const uint64_t Mp = (p == 0) ? M : Mloc;  // the first pass reads (and filters) the full list
@@ -770,10 +777,9 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
         TIGR_CK(cudaEventRecord(landed[c], cs));
     }
     const size_t smem = (2 * sizeof(VT) + sizeof(uint32_t)) * tile_items;
-    auto k_first = &k_onesweep<W, true, SI, false>;
-    auto k_next = &k_onesweep<W, false, SI, false>;
-    TIGR_CK(cudaFuncSetAttribute(k_first, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    TIGR_CK(cudaFuncSetAttribute(k_next, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    for (int p = 0; p < passes; ++p)
+        TIGR_CK(cudaFuncSetAttribute(onesweep_fn<W>(p == 0, false, p == passes - 1),
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     int cur = 0;
     for (uint64_t c = 0; c < nch; ++c) {
         const uint64_t f0 = c * chunk, f1 = std::min<uint64_t>(m, f0 + chunk), Mc = f1 - f0;
@@ -794,7 +800,7 @@ tigr_status build_sorted_runs(uint32_t n, uint64_t m, const uint32_t* src, const
             const uintptr_t al = p == 0 ? ((uintptr_t)(src + f0) | (uintptr_t)(dst + f0))
                                         : ((uintptr_t)(kb[cur].as<uint32_t>() + f0) | (uintptr_t)(vb[cur].as<VT>() + f0));
             const int bulk_ok = (al & 15) == 0 && dev_knob("TIGR_SORT_BULK", 1) != 0;
-            (p == 0 ? k_first : k_next)<<<(unsigned)tp, kST, smem, s>>>(
+            onesweep_fn<W>(p == 0, false, p == passes - 1)<<<(unsigned)tp, kST, smem, s>>>(
                 kb[cur].as<uint32_t>() + f0, vb[cur].as<VT>() + f0, src + f0, dst + f0, W ? w + f0 : nullptr, Mc, Mc,
                 p * bits, bits, bc + p * kMaxRadix, status.as<uint64_t>(), counters.as<uint32_t>() + c * 4 + p,
                 (uint64_t)(c * passes + p + 1), kb[out].as<uint32_t>() + f0, vb[out].as<VT>() + f0, 0, n, bulk_ok,
