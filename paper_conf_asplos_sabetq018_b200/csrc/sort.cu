@@ -610,8 +610,6 @@ tigr_status sort_arcs(const uint32_t* src, const uint32_t* dst, const uint32_t* 
     while (key_bits < 32 && (1ull << key_bits) < (uint64_t)n) ++key_bits;
     const int passes = key_bits == 0 ? 1 : (key_bits + 7) / 8;
     const int bits = key_bits == 0 ? 1 : (key_bits + passes - 1) / passes;
-    // items per thread: 16 (development builds may sweep 12/20/24 with TIGR_SORT_SI; the
-    // source-range-filtered first pass exists for 16 only, so filtered builds always use 16)
     const bool filtered = klo != 0 || khi < n;
     constexpr int SI = 16;  // items per thread (a sweep of 12 / 16 / 20 / 24 chose 16)
     const uint64_t tile_items = (uint64_t)kST * SI;
