@@ -136,3 +136,37 @@ def test_cfg4_pull_pagerank_full(tigr, cfg4):
     want = oracle.pagerank(oracle.csr_build(rec.n, src, dst), 20)
     assert np.abs(got - want).max() <= 1e-6
     assert np.abs(rec.n * got - rec.n * want).max() <= 1e-6
+
+
+def _export_csr_device(tigr, g):
+    """row_ptr / col / w of a graph as CUDA tensors (tigr_graph_export_csr to device buffers)."""
+    info = g.info()
+    rp = torch.empty(info["n"] + 1, dtype=torch.int64, device="cuda")
+    col = torch.empty(max(info["m"], 1), dtype=torch.int32, device="cuda")
+    w = torch.empty_like(col) if info["weighted"] else None
+    tigr._check(tigr._lib.tigr_graph_export_csr(g.ptr, rp.data_ptr(), col.data_ptr(),
+                                                None if w is None else w.data_ptr(), 1, None))
+    torch.cuda.synchronize()
+    return rp, col, w
+
+
+def test_cfg5_host_input_sorted_runs(tigr):
+    """Config 5's 1.47 B weighted arcs from pinned host memory: 64 copy chunks of 23 M arcs, each
+    radix-sorted as it lands, merged into the rows by row-space windows (sort.cu
+    build_sorted_runs) -- row_ptr, targets and weights equal element by element to the
+    device-input build (whose BFS, SSSP and CC are oracle-exact at this size, test_cfg5_twitter_shaped_full)."""
+    rec = graphgen.recipe("cfg5")
+    src = torch.empty(rec.m, dtype=torch.int32, device="cuda")
+    dst, w = torch.empty_like(src), torch.empty_like(src)
+    tigr.tigr_rmat_coo(rec.n, rec.m, rec.a, rec.b, rec.c, rec.seed, rec.wseed, rec.wmin, rec.wmax, src, dst, w)
+    gd = tigr.tigr_graph_from_coo(rec.n, src, dst, w)
+    want = _export_csr_device(tigr, gd)
+    gd.free()
+    hs, hd, hw = src.cpu().pin_memory(), dst.cpu().pin_memory(), w.cpu().pin_memory()
+    del src, dst, w
+    torch.cuda.empty_cache()
+    gh = tigr.tigr_graph_from_coo(rec.n, hs, hd, hw)
+    got = _export_csr_device(tigr, gh)
+    gh.free()
+    for a, b in zip(got, want):
+        assert torch.equal(a, b)
