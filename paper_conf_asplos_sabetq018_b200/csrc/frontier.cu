@@ -217,7 +217,10 @@ tigr_status compact_launch(const tigr_vgraph* vg, Ctl* ctl, int delta, cudaStrea
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const uint64_t tiles = ((uint64_t)n + kFqThreads * kCompactPer - 1) / (kFqThreads * kCompactPer);
-    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(tiles, (uint64_t)sms * 8));
+    // one tile per block up to 64 blocks per SM: a block walking several tiles paid one stamp-load
+    // latency per tile in sequence (an empty cfg4 sweep took 15 us for 16.8 MB)
+    const uint64_t cap = (uint64_t)sms * (uint64_t)dev_knob("TIGR_COMPACT_BPS", 64);
+    const unsigned grid = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap));
     k_compact<<<grid, kFqThreads, 0, s>>>(vg->ws.stamp.as<stamp_t>(), vg->vnode_ptr.as<uint32_t>(), n, vg->lo, vg->hi, ctl,
                                           const_cast<uint32_t*>(vg->ws.qv.as<uint32_t>()),
                                           const_cast<uint32_t*>(vg->ws.qo.as<uint32_t>()), delta);
