@@ -744,6 +744,23 @@ def test_host_input_sorted_runs_skewed(tigr):
     assert ei.value.status == tigr.TIGR_EINVAL
 
 
+@pytest.mark.parametrize("n", [1, 2, 300])
+def test_host_input_sorted_runs_tiny_n(tigr, n):
+    """Sorted runs with one-pass keys: n = 1 (every arc a self-loop of node 0, one run per chunk
+    holding a single row), n = 2 and n = 300 (one 8-bit or 9-bit-in-two-passes key), two copy
+    chunks, weighted; CSR and SSSP against the oracle."""
+    m = (1 << 24) + 5
+    rng = np.random.default_rng(n)
+    src = rng.integers(0, n, m, dtype=np.uint32)
+    dst = rng.integers(0, n, m, dtype=np.uint32)
+    w = rng.integers(1, 65, m, dtype=np.uint32)
+    g = tigr.tigr_graph_from_coo(n, src, dst, w)
+    rp, col, ww = tigr.tigr_graph_export_csr(g)
+    o = oracle.csr_build(n, src, dst, w)
+    assert np.array_equal(rp, o.row_ptr) and np.array_equal(col, o.col) and np.array_equal(ww, o.wt)
+    assert np.array_equal(tigr.tigr_run(tigr.tigr_virtualize(g, 8), "sssp", 0), oracle.sssp(o, 0))
+
+
 def test_bytes_alg_byte_model(tigr):
     """tigr_stats.bytes_alg is SURVEY §8(d)'s byte model, computed in the library: PageRank per
     relax launch 20 B/arc + 4 B/virtual node + 20 B per node with arcs (apply fused in), over
