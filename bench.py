@@ -50,6 +50,24 @@ PAPER_CONTEXT = {
 }
 
 
+def ablation_context():
+    """This build's Fig. 13 analogue beside the paper's: cfg3 (LiveJournal-shaped) SSSP speedups
+    of the virtual transformations over the untransformed engine, K = 8, from the committed
+    ablation run (tools/ablation.py -> profiles/r02_ablation_cfg3.jsonl)."""
+    path = os.path.join(ROOT, "profiles", "r02_ablation_cfg3.jsonl")
+    want = {"Tigr-V+ K=8 strided": "tigr_v_plus", "Tigr-V K=8 consecutive": "tigr_v", "Tigr-UDT K=8": "tigr_udt"}
+    out = {}
+    try:
+        for line in open(path):
+            d = json.loads(line)
+            if d.get("algo") == "sssp" and d.get("mode") == "worklist async" and d.get("variant") in want:
+                out[want[d["variant"]]] = round(d["speedup_vs_baseline"], 2)
+    except (OSError, ValueError):
+        return None
+    out["source"] = "profiles/r02_ablation_cfg3.jsonl (tools/ablation.py, B200, same engine, cfg3 SSSP, K = 8)"
+    return out
+
+
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -423,7 +441,7 @@ def main():
                          "pagerank_20it": statistics.mean(phase[2]), "relax_total": relax_ms / args.steps},
         "algo_gteps": 20 * m / (statistics.mean(phase[2]) * 1e-3) / 1e9,
         "nv": nv[0], "gpu_launches": launches, "clocks": clk,
-        "paper_context": PAPER_CONTEXT,
+        "paper_context": dict(PAPER_CONTEXT, fig13_analogue_this_build=ablation_context()),
     }
     if rec_note:
         result["note"] = rec_note
