@@ -301,6 +301,22 @@ def gather_ceiling():
     return out
 
 
+def red_ceiling(n_elems, reds):
+    """Best-of-5 ms for `reds` uniform random float64 REDs into an n_elems array
+    (tools/micro/gather_ceiling.cu micro_red), or None."""
+    import ctypes
+    path = os.path.join(ROOT, "build", "libmicro.so")
+    if not os.path.exists(path) or n_elems == 0:
+        return None
+    lib = ctypes.CDLL(path)
+    if not hasattr(lib, "micro_red"):
+        return None
+    lib.micro_red.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_int, ctypes.POINTER(ctypes.c_double)]
+    lib.micro_red.restype = ctypes.c_int
+    ms = ctypes.c_double()
+    return ms.value if lib.micro_red(n_elems, reds, 5, ctypes.byref(ms)) == 0 else None
+
+
 def main():
     args = parse()
     rank = int(os.environ.get("RANK", "0"))
@@ -566,6 +582,23 @@ def main():
         del houts
 
     if not args.no_extra and not args.profile and world == 1:
+        # the PR relax against its own ceiling: the global float64 reductions one launch issues
+        # (arcs missing the shared-memory hot table; tigr_vgraph_pr_profile) per second of the
+        # live relax time, over the measured random-RED rate into an array of the accumulator's size
+        g = tigr.tigr_graph_from_coo(n, src, dst, None, stream=s)
+        vg = tigr.tigr_virtualize(g, args.K, args.layout, stream=s)
+        prof = tigr.tigr_vgraph_pr_profile(vg, stream=s)
+        vg.free()
+        g.free()
+        red_ms = red_ceiling(prof["n_in"], 1 << 30)
+        ach = prof["global_reds"] / (relax_avg_ms * 1e-3) / 1e9
+        ceil = (1 << 30) / (red_ms * 1e-3) / 1e9 if red_ms else None
+        result["roofline"]["l2_red"] = {
+            "arcs_per_launch": prof["arcs"], "global_reds_per_launch": prof["global_reds"],
+            "hot_slots": prof["hot_slots"], "accumulator_entries": prof["n_in"],
+            "achieved_gred_s": ach, "ceiling_gred_s": ceil, "frac": (ach / ceil) if ceil else None,
+            "ceiling_source": "tools/micro/gather_ceiling.cu micro_red: uniform random float64 REDs into "
+                              "n_in doubles, 8 per thread in flight, 148 x 8 blocks of 256, best of 5"}
         peak_g = gather_ceiling()
         result["gather_ceiling"] = peak_g
         result["per_algo"] = per_algo(tigr, torch, rec, args, s, peak, peak_g)

@@ -259,6 +259,18 @@ tigr_status tigr_virtualize(const tigr_graph* g, uint32_t K, tigr_layout layout,
 tigr_status tigr_vgraph_info(const tigr_vgraph* vg, uint64_t* nv, uint64_t* bytes, double* ms_build,
                              uint32_t* vnode_lo, uint32_t* vnode_hi);
 
+/* Diagnostic (measurement, not the hot path): how the push PageRank relax of this virtual
+ * graph splits its arcs (fn. 7 L1078: one float64 accumulate per arc) between the per-SM
+ * shared-memory table of the hot accumulator ids and global float64 reductions.  Prepares the
+ * accumulator order if no PageRank ran yet (it is cached with the vgraph), then counts over this
+ * rank's vnode range: arcs = its arcs, global_reds = the arcs whose accumulator id is >=
+ * hot_slots (one L2 RED each per relax launch), n_in = nodes with in-arcs (the accumulator
+ * entries ever written).  Any output may be NULL.  Synchronises the stream.  Errors: EINVAL (NULL
+ * vgraph), EUNSUPPORTED (4 does not divide K, or a transposed graph: those run other kernels),
+ * ECUDA. */
+tigr_status tigr_vgraph_pr_profile(tigr_vgraph* vg, void* stream, uint64_t* arcs, uint64_t* global_reds,
+                                   uint32_t* hot_slots, uint32_t* n_in);
+
 /* Copy vnode_ptr[n+1] and vn_phys[NV] out (either may be NULL). */
 tigr_status tigr_vgraph_export(const tigr_vgraph* vg, uint32_t* vnode_ptr, uint32_t* vn_phys,
                                int is_device_ptr, void* stream);

@@ -86,6 +86,8 @@ _SIGS = {
     "tigr_vgraph_info": (_I, [_P, ctypes.POINTER(_U64), ctypes.POINTER(_U64), ctypes.POINTER(_D),
                               ctypes.POINTER(_U32), ctypes.POINTER(_U32)]),
     "tigr_vgraph_export": (_I, [_P, _P, _P, _I, _P]),
+    "tigr_vgraph_pr_profile": (_I, [_P, _P, ctypes.POINTER(_U64), ctypes.POINTER(_U64), ctypes.POINTER(_U32),
+                                    ctypes.POINTER(_U32)]),
     "tigr_vgraph_assignment": (_I, [_P, _P, _P, _P, _I, _P]),
     "tigr_vgraph_partition": (_I, [_P, _I, _I]),
     "tigr_partition_ranges": (_I, [_U32, _P, _P, _I, _P, _P]),
@@ -383,6 +385,14 @@ def tigr_vgraph_export(vg: VGraph, stream=None):
     ph = np.empty(max(nv, 1), dtype=np.uint32)
     _check(_lib.tigr_vgraph_export(vg.ptr, vp.ctypes.data, ph.ctypes.data, 0, _stream_ptr(stream)))
     return vp, ph[:nv]
+
+
+def tigr_vgraph_pr_profile(vg: VGraph, stream=None) -> dict:
+    """Push PageRank's split of this rank's arcs: shared-memory hot slots vs global float64 REDs."""
+    a, r, h, ni = _U64(), _U64(), _U32(), _U32()
+    _check(_lib.tigr_vgraph_pr_profile(vg.ptr, _stream_ptr(stream), ctypes.byref(a), ctypes.byref(r),
+                                       ctypes.byref(h), ctypes.byref(ni)))
+    return {"arcs": a.value, "global_reds": r.value, "hot_slots": h.value, "n_in": ni.value}
 
 
 def tigr_vgraph_assignment(vg: VGraph, stream=None):

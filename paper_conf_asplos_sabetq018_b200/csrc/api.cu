@@ -490,6 +490,13 @@ tigr_status tigr_vgraph_info(const tigr_vgraph* vg, uint64_t* nv, uint64_t* byte
     return TIGR_OK;
 }
 
+tigr_status tigr_vgraph_pr_profile(tigr_vgraph* vg, void* stream, uint64_t* arcs, uint64_t* global_reds,
+                                   uint32_t* hot_slots, uint32_t* n_in) {
+    if (!vg) return fail(TIGR_EINVAL, "vgraph_pr_profile: NULL vgraph");
+    TIGR_TRY(need_device());
+    return tigr::pr_cid_profile(vg, (cudaStream_t)stream, arcs, global_reds, hot_slots, n_in);
+}
+
 tigr_status tigr_vgraph_export(const tigr_vgraph* vg, uint32_t* vnode_ptr, uint32_t* vn_phys, int is_device_ptr,
                                void* stream) {
     if (!vg) return fail(TIGR_EINVAL, "vgraph_export: NULL vgraph");

@@ -155,3 +155,10 @@ struct tigr_comm_group {
 };
 
 struct tigr_vgraph;  // defined in vgraph.cuh
+
+namespace tigr {
+// push PageRank's split of a rank's arcs into hot shared-memory slots and global float64
+// reductions (pr.cu; the C-ABI diagnostic tigr_vgraph_pr_profile)
+tigr_status pr_cid_profile(tigr_vgraph* vg, cudaStream_t s, uint64_t* arcs, uint64_t* reds, uint32_t* hot,
+                           uint32_t* n_in);
+}  // namespace tigr

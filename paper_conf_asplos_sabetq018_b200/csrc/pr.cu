@@ -318,6 +318,7 @@ static void fill_plan(PrCidPlan& p, int layout, int unit) {
     p.threads = T;
     p.per_thread = B;
     p.smem = sizeof(double) * SLOTS;
+    p.hot = SLOTS;
 }
 
 // Kernel shape: one 768-thread block per SM (24 warps), 24576 hot slots (192 KB of shared
@@ -342,6 +343,52 @@ PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
     p.tiles = (unsigned)(((uint64_t)(vg->hi - vg->lo) + per_tile - 1) / per_tile);
     p.grid = (unsigned)std::min<uint64_t>(p.tiles, (uint64_t)sms * (per_sm > 0 ? per_sm : 1));
     return p;
+}
+
+// arcs (non-pad slots) of the vnode range [lo, hi) and those among them with id >= hot
+__global__ void k_count_reds(const uint32_t* __restrict__ col_pr,
+                             const uint32_t* __restrict__ cptr, const uint32_t* __restrict__ vptr, uint32_t n,
+                             uint32_t lo, uint32_t hi, uint32_t hot, unsigned long long* __restrict__ out) {
+    unsigned long long a = 0, r = 0;
+    for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+        const uint32_t f = vptr[v];
+        if (vptr[v + 1] == f || f < lo || f >= hi) continue;  // no arcs, or another rank's family
+        for (uint64_t q = (uint64_t)cptr[v] * kSpan; q < (uint64_t)cptr[v + 1] * kSpan; ++q) {
+            const uint32_t c = col_pr[q];
+            if (c == kPad) continue;
+            ++a;
+            r += c >= hot;
+        }
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+        a += __shfl_xor_sync(0xffffffffu, a, o);
+        r += __shfl_xor_sync(0xffffffffu, r, o);
+    }
+    if ((threadIdx.x & 31) == 0) { atomicAdd(out, a); atomicAdd(out + 1, r); }
+}
+
+tigr_status pr_cid_profile(tigr_vgraph* vg, cudaStream_t s, uint64_t* arcs, uint64_t* reds, uint32_t* hot,
+                           uint32_t* n_in) {
+    if (!vg->vec) return fail(TIGR_EUNSUPPORTED, "vgraph_pr_profile: the accumulator-order relax needs 4 | K");
+    if (vg->g->transposed) return fail(TIGR_EUNSUPPORTED, "vgraph_pr_profile: push PageRank only");
+    TIGR_TRY(pr_cid_prepare(vg, s));
+    const PrCidPlan p = pr_cid_plan(vg);
+    TmpBuf cnt;
+    TIGR_TRY(cnt.alloc(2 * sizeof(unsigned long long), s));
+    TIGR_CK(cudaMemsetAsync(cnt.p, 0, 2 * sizeof(unsigned long long), s));
+    const uint32_t n = vg->g->n;
+    k_count_reds<<<grid_cap(n, 16), kBlock, 0, s>>>(vg->ws.col_pr.as<uint32_t>(), vg->g->cptr.as<uint32_t>(),
+                                                    vg->vnode_ptr.as<uint32_t>(), n, vg->lo, vg->hi, p.hot,
+                                                    cnt.as<unsigned long long>());
+    TIGR_CKL("pr profile");
+    unsigned long long h[2] = {0, 0};
+    TIGR_CK(cudaMemcpyAsync(h, cnt.p, sizeof(h), cudaMemcpyDeviceToHost, s));
+    TIGR_CK(cudaStreamSynchronize(s));
+    if (arcs) *arcs = h[0];
+    if (reds) *reds = h[1];
+    if (hot) *hot = p.hot;
+    if (n_in) *n_in = (uint32_t)vg->ws.n_in;
+    return TIGR_OK;
 }
 
 tigr_status pr_cid_apply(tigr_vgraph* vg, double base, double damping, int dangling, const double* dsum_cur,

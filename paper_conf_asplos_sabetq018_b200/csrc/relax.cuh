@@ -80,6 +80,7 @@ struct PrCidPlan {
     unsigned grid = 0, tiles = 0;
     int threads = 256, per_thread = 4;
     size_t smem = 0;
+    uint32_t hot = 0;  // accumulator ids below this are summed in shared memory
 };
 RelaxFn relax_pr_pull_kernel(int layout, int unit, int* per_thread);   // pull PageRank (pr.cu, NEXT-1)
 tigr_status pr_cid_prepare(tigr_vgraph* vg, cudaStream_t s);

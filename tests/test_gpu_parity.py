@@ -761,6 +761,32 @@ def test_host_input_sorted_runs_tiny_n(tigr, n):
     assert np.array_equal(tigr.tigr_run(tigr.tigr_virtualize(g, 8), "sssp", 0), oracle.sssp(o, 0))
 
 
+def test_vgraph_pr_profile(tigr):
+    """tigr_vgraph_pr_profile: the push PageRank relax's arcs split into shared-memory hot slots
+    and global float64 reductions.  cfg1 (n < hot slots): no global reduction at all; cfg2 (2^20
+    nodes): every arc counted once, n_in = nodes with in-arcs, and the global reductions at least
+    the arcs outside the true top-hot_slots in-degrees; a rank of two counts its range's arcs."""
+    rec = graphgen.recipe("cfg1")
+    src, dst, w = graphgen.generate(rec)
+    p = tigr.tigr_vgraph_pr_profile(tigr.tigr_virtualize(tigr.tigr_graph_from_coo(rec.n, src, dst, w), 8))
+    assert p["arcs"] == rec.m and p["global_reds"] == 0 and p["hot_slots"] >= rec.n
+    rec = graphgen.recipe("cfg2")
+    src, dst, _ = graphgen.generate(rec, weighted=False)
+    g = tigr.tigr_graph_from_coo(rec.n, src, dst, None)
+    vg = tigr.tigr_virtualize(g, 8)
+    p = tigr.tigr_vgraph_pr_profile(vg)
+    indeg = np.bincount(dst, minlength=rec.n)
+    assert p["arcs"] == rec.m and p["n_in"] == int((indeg > 0).sum())
+    top = int(np.sort(indeg)[::-1][:p["hot_slots"]].sum())
+    assert rec.m - top <= p["global_reds"] < rec.m
+    tigr.tigr_vgraph_partition(vg, 2, 0)
+    vp, _ = tigr.tigr_vgraph_export(vg)
+    lo, hi = vg.info()["lo"], vg.info()["hi"]
+    deg = np.bincount(src, minlength=rec.n)
+    mine = (vp[:-1] >= lo) & (vp[:-1] < hi) & (deg > 0)
+    assert tigr.tigr_vgraph_pr_profile(vg)["arcs"] == int(deg[mine].sum())
+
+
 def test_bytes_alg_byte_model(tigr):
     """tigr_stats.bytes_alg is SURVEY §8(d)'s byte model, computed in the library: PageRank per
     relax launch 20 B/arc + 4 B/virtual node + 20 B per node with arcs (apply fused in), over

@@ -84,3 +84,56 @@ extern "C" int micro_gather(uint64_t n, uint64_t gathers, int reps, double* ms_b
     *ms_best = best;
     return 0;
 }
+
+// ---- float64 reductions ---------------------------------------------------------------------
+// The PageRank push relax (pr.cu) sends every arc whose accumulator id misses the shared-memory
+// hot table to L2 as one fire-and-forget float64 reduction (RED.E.ADD.F64).  This kernel
+// measures the rate of such reductions at uniform random addresses of an n-entry float64 array
+// (the accumulator's size: L2-resident at scale 24), 8 per thread and step, same grid.
+//   extern "C" int micro_red(uint64_t n, uint64_t reds, int reps, double* ms_best);
+namespace {
+__global__ void __launch_bounds__(256) k_red(double* __restrict__ a, uint64_t n, uint64_t per_thread) {
+    const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (uint64_t k = 0; k < per_thread; k += 8) {
+#pragma unroll
+        for (int q = 0; q < 8; ++q) {
+            const uint32_t h = mix((t << 24) ^ (k + q) ^ 0x5bd1e995ull);
+            atomicAdd(a + ((uint64_t)h * n >> 32), 1.0);  // result unused: compiles to RED
+        }
+    }
+}
+}  // namespace
+
+extern "C" int micro_red(uint64_t n, uint64_t reds, int reps, double* ms_best) {
+    int dev = 0, sms = 148;
+    if (cudaGetDevice(&dev) != cudaSuccess) return -1;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    double* a = nullptr;
+    if (cudaMalloc(&a, n * sizeof(double)) != cudaSuccess) return -2;
+    cudaMemset(a, 0, n * sizeof(double));
+    const unsigned grid = (unsigned)sms * 8;
+    const uint64_t threads = (uint64_t)grid * 256;
+    const uint64_t per_thread = ((reds + threads - 1) / threads + 7) / 8 * 8;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    k_red<<<grid, 256>>>(a, n, per_thread);  // warm-up (fills L2)
+    double best = 1e30;
+    for (int r = 0; r < reps; ++r) {
+        cudaEventRecord(e0);
+        k_red<<<grid, 256>>>(a, n, per_thread);
+        cudaEventRecord(e1);
+        cudaEventSynchronize(e1);
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, e0, e1);
+        const double scaled = ms * (double)reds / (double)(per_thread * threads);
+        if (scaled < best) best = scaled;
+    }
+    const cudaError_t err = cudaGetLastError();
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(a);
+    if (err != cudaSuccess) return -3;
+    *ms_best = best;
+    return 0;
+}
