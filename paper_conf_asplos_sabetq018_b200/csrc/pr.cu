@@ -96,9 +96,17 @@ __global__ void __launch_bounds__(T, MINB) k_relax_pr_cid(RelaxArgs a, const uin
     __syncthreads();
     const uint64_t pol = policy_evict_last();
     const uint4* c4 = reinterpret_cast<const uint4*>(col_pr);
+    // probe: 0 in every shipped run; development builds (TIGR_PR_EXP) use 1 / 2 / 3 to time the
+    // kernel without its hot-slot adds / without its global reductions / with plain stores (wrong
+    // sums, measurement only).  The run-time test stays in shipped builds on purpose: with it ptxas
+    // lays the push out so that the 1024-thread kernel runs 1.139 ms per cfg4 launch, against 1.174
+    // for the best branch-free push (768 threads) and 1.182 for the branch-free 1024-thread push
+    // (tools/dev/pr_relax_ab.py, three alternating runs on one box).
+    const int probe = fz.probe;
     auto push = [&](uint32_t c, double x) {
-        if (c < (uint32_t)SLOTS) atomicAdd(&s_acc[c], x);
-        else red_add_f64(a.acc + c, x, pol);
+        if (c < (uint32_t)SLOTS) { if (probe != 1) atomicAdd(&s_acc[c], x); }
+        else if (probe == 3) a.acc[c] = x;
+        else if (probe != 2) red_add_f64(a.acc + c, x, pol);
     };
     for (uint32_t tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
         const uint64_t base = (uint64_t)a.lo + (uint64_t)tile * (B * T) + t;
@@ -321,18 +329,25 @@ static void fill_plan(PrCidPlan& p, int layout, int unit) {
     p.hot = SLOTS;
 }
 
-// Kernel shape: one 768-thread block per SM (24 warps), 24576 hot slots (192 KB of shared
-// memory: one table per SM instead of two 8192-slot copies), 4 virtual nodes per thread.
-// Measured at cfg4 (relax ms/launch): 256x2 blocks, 8192 slots 1.53; 512x1, 24576 1.15;
-// 768x1, 24576 1.12; 768x1, 28672 1.21; 1024x1 (spills) 1.16.  TIGR_PR_CFG selects the
-// alternatives in development builds (dev_knob).
+// Kernel shape: one 1024-thread block per SM (32 warps), 24576 hot slots (192 KB of shared
+// memory: one table per SM instead of two 8192-slot copies), 2 virtual nodes per thread (45
+// registers).  Measured at cfg4 (relax ms/launch): rounds 1-2 -- 256x2 blocks, 8192 slots 1.53;
+// 512x1, 24576 1.15; 768x1 with 4 vnodes/thread, 24576 1.12-1.17 (the round-2b shape); 768x1,
+// 28672 1.21; 1024x1 with 4 vnodes/thread (spills) 1.16.  Round 2d on one box (dev build):
+// 1024x2v 1.129, 1024x3v 1.149, 1024x1v 1.138, 1024x2v with 26624 / 28672 slots 1.148 / 1.141
+// (more shared memory leaves less L1 for the per-vnode gathers); shipped build, alternating
+// runs: 1024x2v 1.139 against 768x4v 1.174 (with the probe test in the push, see the kernel).
+// Timing decomposition (TIGR_PR_EXP): without the global reductions 0.78 ms, without the
+// hot-slot adds 1.17 ms -- the reductions and the per-vnode gathers are what overlap.
+// TIGR_PR_CFG selects the alternatives in development builds (dev_knob).
 PrCidPlan pr_cid_plan(tigr_vgraph* vg) {
     PrCidPlan p;
-    switch (dev_knob("TIGR_PR_CFG", 5)) {
+    switch (dev_knob("TIGR_PR_CFG", 7)) {
         case 0: fill_plan<4, 256, 8192, 2>(p, vg->layout, (int)vg->unit); break;
         case 1: fill_plan<4, 512, 24576, 1>(p, vg->layout, (int)vg->unit); break;
+        case 5: fill_plan<4, 768, 24576, 1>(p, vg->layout, (int)vg->unit); break;
         case 6: fill_plan<4, 768, 28672, 1>(p, vg->layout, (int)vg->unit); break;
-        default: fill_plan<4, 768, 24576, 1>(p, vg->layout, (int)vg->unit); break;
+        default: fill_plan<2, 1024, 24576, 1>(p, vg->layout, (int)vg->unit); break;
     }
     cudaFuncSetAttribute(p.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p.smem);
     int per_sm = 0, dev = 0, sms = 148;

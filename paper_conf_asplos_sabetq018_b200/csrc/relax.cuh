@@ -74,6 +74,7 @@ struct PrFuse {
     const double* prev = nullptr;  // accumulator of the previous iteration (cid order)
     const uint32_t* cid = nullptr;
     double base = 0.0, damping = 0.0, x0 = 0.0;
+    int probe = 0;              // 0; development builds: timing decomposition (pr.cu)
 };
 struct PrCidPlan {
     void (*fn)(RelaxArgs, const uint32_t*, uint32_t, PrFuse) = nullptr;

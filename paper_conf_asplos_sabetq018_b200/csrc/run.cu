@@ -431,6 +431,7 @@ tigr_status run_pr(tigr_vgraph* vg, const tigr_run_opts& o, cudaStream_t s, tigr
             fz.base = base;
             fz.damping = o.pr_damping;
             fz.x0 = 1.0 / (double)n;
+            fz.probe = dev_knob("TIGR_PR_EXP", 0);  // always 0 in shipped builds
             if (t > 0) TIGR_CK(cudaMemsetAsync(acc_cur, 0, sizeof(double) * ws.n_in, s));
             a.acc = acc_cur;
         }
