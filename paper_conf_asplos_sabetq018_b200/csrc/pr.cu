@@ -335,7 +335,8 @@ static void fill_plan(PrCidPlan& p, int layout, int unit) {
 // 512x1, 24576 1.15; 768x1 with 4 vnodes/thread, 24576 1.12-1.17 (the round-2b shape); 768x1,
 // 28672 1.21; 1024x1 with 4 vnodes/thread (spills) 1.16.  Round 2d on one box (dev build):
 // 1024x2v 1.129, 1024x3v 1.149, 1024x1v 1.138, 1024x2v with 26624 / 28672 slots 1.148 / 1.141
-// (more shared memory leaves less L1 for the per-vnode gathers); shipped build, alternating
+// (more shared memory leaves less L1 for the per-vnode gathers; fewer slots lose hot coverage:
+// 20480 / 16384 / 12288 slots 1.150 / 1.160 / 1.371); shipped build, alternating
 // runs: 1024x2v 1.139 against 768x4v 1.174 (with the probe test in the push, see the kernel).
 // Timing decomposition (TIGR_PR_EXP): without the global reductions 0.78 ms, without the
 // hot-slot adds 1.17 ms -- the reductions and the per-vnode gathers are what overlap.
