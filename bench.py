@@ -623,6 +623,20 @@ def main():
                                             f"arc list), {dt:.1f} s; oracle/oracle.c or_pagerank, single thread "
                                             f"pinned to core {core}",
                                   "host": host_cpu()}
+        # SURVEY §8(d)'s optional secondary baseline: OpenMP pull PageRank on all host cores (not
+        # the oracle; tools/cpu_baseline/omp_pagerank.c, tested against the oracle in
+        # tests/test_cpu_baseline.py).  A bounded sample: 5 of the 20 iterations, in-CSR build untimed.
+        try:
+            from tools import cpu_baseline
+            its = 5
+            _, mb, mi = cpu_baseline.omp_pagerank(n, hs, hd, its, 0.85, 0)
+            result["cpu_baseline_multicore"] = {
+                "value": its * m / (mi * 1e-3) / 1e9, "unit": "GTEPS", "cores": os.cpu_count(),
+                "kind": "openmp pull PageRank (tools/cpu_baseline/omp_pagerank.c), not the oracle",
+                "sample": f"{its} of the 20 PageRank iterations on the full cfg4 graph, {mi / 1e3:.1f} s "
+                          f"(in-CSR build {mb / 1e3:.1f} s, untimed)"}
+        except (OSError, MemoryError) as e:
+            result["cpu_baseline_multicore"] = {"error": str(e)}
     if rank == 0:
         print(json.dumps(result), flush=True)
     if world > 1:
