@@ -635,6 +635,11 @@ def main():
                 "kind": "openmp pull PageRank (tools/cpu_baseline/omp_pagerank.c), not the oracle",
                 "sample": f"{its} of the 20 PageRank iterations on the full cfg4 graph, {mi / 1e3:.1f} s "
                           f"(in-CSR build {mb / 1e3:.1f} s, untimed)"}
+            lv, bb, br = cpu_baseline.omp_bfs(n, hs, hd, 0, 0)  # the per_algo BFS graph's arcs, source 0
+            reach = int(np.bincount(hs, minlength=n)[lv != 0xFFFFFFFF].sum())
+            result["cpu_baseline_multicore"]["bfs"] = {
+                "gteps_input": reach / (br * 1e-3) / 1e9, "ms": br, "levels": int(lv[lv != 0xFFFFFFFF].max()) + 1,
+                "kind": "level-synchronous OpenMP BFS from vertex 0 (out-CSR build untimed)"}
         except (OSError, MemoryError) as e:
             result["cpu_baseline_multicore"] = {"error": str(e)}
     if rank == 0:

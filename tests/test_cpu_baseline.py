@@ -35,3 +35,13 @@ def test_omp_pagerank_edge_graphs(omp):
     assert np.allclose(got, (1 - 0.85) / 5, rtol=0, atol=1e-17)
     got, _, _ = omp.omp_pagerank(3, np.array([0, 1, 2], np.uint32), np.array([1, 2, 0], np.uint32), 20, 0.85, 2)
     assert np.allclose(got, 1.0 / 3, rtol=0, atol=1e-15)
+
+
+@pytest.mark.parametrize("cfg", ["cfg1", "cfg2"])
+def test_omp_bfs_matches_oracle(omp, cfg):
+    rec = graphgen.recipe(cfg)
+    src, dst, w = graphgen.generate(rec, weighted=(cfg == "cfg1"))
+    want = oracle.bfs(oracle.csr_build(rec.n, src, dst, w), 0)
+    for threads in (1, 4):
+        got, _, _ = omp.omp_bfs(rec.n, src, dst, 0, threads)
+        assert np.array_equal(got, want)

@@ -64,3 +64,54 @@ int omp_pagerank(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* ds
     free(rp); free(outdeg); free(in_src); free(cur); free(contrib);
     return 0;
 }
+
+/* Level-synchronous top-down BFS from `source` on all cores (the same secondary baseline, for
+ * BFS): out-CSR by atomic counting (untimed), then one parallel sweep of the frontier per level
+ * with an atomic compare-and-swap claiming each newly reached vertex.  level[n] receives the
+ * levels (0xFFFFFFFF = unreached), exactly the oracle's (BFS levels are unique). */
+int omp_bfs(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst, uint32_t source, int threads,
+            uint32_t* level, double* ms_build, double* ms_run) {
+    if (threads > 0) omp_set_num_threads(threads);
+    double t0 = now_ms();
+    uint64_t* rp = calloc((size_t)n + 1, sizeof(uint64_t));
+    uint32_t* adj = malloc((m ? m : 1) * sizeof(uint32_t));
+    uint64_t* cur = malloc(((size_t)n + 1) * sizeof(uint64_t));
+    uint32_t* fa = malloc((n ? n : 1) * sizeof(uint32_t));
+    uint32_t* fb = malloc((n ? n : 1) * sizeof(uint32_t));
+    if (!rp || !adj || !cur || !fa || !fb) {
+        free(rp); free(adj); free(cur); free(fa); free(fb);
+        return -1;
+    }
+#pragma omp parallel for schedule(static)
+    for (uint64_t e = 0; e < m; ++e) __atomic_fetch_add(&rp[src[e] + 1], 1, __ATOMIC_RELAXED);
+    for (uint32_t v = 0; v < n; ++v) rp[v + 1] += rp[v];
+    memcpy(cur, rp, ((size_t)n + 1) * sizeof(uint64_t));
+#pragma omp parallel for schedule(static)
+    for (uint64_t e = 0; e < m; ++e) adj[__atomic_fetch_add(&cur[src[e]], 1, __ATOMIC_RELAXED)] = dst[e];
+    double t1 = now_ms();
+#pragma omp parallel for schedule(static)
+    for (uint32_t v = 0; v < n; ++v) level[v] = 0xFFFFFFFFu;
+    uint64_t nf = 0, nn = 0;
+    if (source < n) { level[source] = 0; fa[nf++] = source; }
+    for (uint32_t lv = 1; nf; ++lv) {
+        nn = 0;
+#pragma omp parallel for schedule(dynamic, 64)
+        for (uint64_t i = 0; i < nf; ++i) {
+            const uint32_t u = fa[i];
+            for (uint64_t e = rp[u]; e < rp[u + 1]; ++e) {
+                const uint32_t v = adj[e];
+                uint32_t expect = 0xFFFFFFFFu;
+                if (level[v] == 0xFFFFFFFFu &&
+                    __atomic_compare_exchange_n(&level[v], &expect, lv, 0, __ATOMIC_RELAXED, __ATOMIC_RELAXED))
+                    fb[__atomic_fetch_add(&nn, 1, __ATOMIC_RELAXED)] = v;
+            }
+        }
+        uint32_t* t = fa; fa = fb; fb = t;
+        nf = nn;
+    }
+    double t2 = now_ms();
+    if (ms_build) *ms_build = t1 - t0;
+    if (ms_run) *ms_run = t2 - t1;
+    free(rp); free(adj); free(cur); free(fa); free(fb);
+    return 0;
+}
