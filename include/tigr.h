@@ -151,6 +151,11 @@ void tigr_run_opts_default(tigr_run_opts* opts);
  * (arc e before arc f iff e < f), so the device CSR is the canonical one (a stable counting sort
  * by source) and tigr_graph_export_coo returns the arcs in that order.
  * symmetrize=1 appends (dst[e] -> src[e], w[e]) for every arc (weak connectivity, CC).
+ * is_device_ptr = 0: src / dst / w are host arrays (pinned memory transfers at the link's rate);
+ * the call copies them in chunks and, for a whole unsymmetrised graph of more than one chunk,
+ * sorts each chunk on the device as it lands and merges the sorted runs into the rows, so most
+ * of the build overlaps the transfer (same CSR as the device-input build).  The call returns
+ * after the build completed (the stream is synchronised); the caller's arrays are not retained.
  * Errors: EINVAL (an id >= n, n == 0), ERANGE (n > 0xFFFFFFFE or too many arcs). */
 tigr_status tigr_graph_from_coo(uint32_t n, uint64_t m, const uint32_t* src, const uint32_t* dst,
                                 const uint32_t* w, int is_device_ptr, int symmetrize, void* stream,
