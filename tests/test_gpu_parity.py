@@ -761,6 +761,28 @@ def test_host_input_sorted_runs_tiny_n(tigr, n):
     assert np.array_equal(tigr.tigr_run(tigr.tigr_virtualize(g, 8), "sssp", 0), oracle.sssp(o, 0))
 
 
+def test_host_input_partitioned_multi_chunk(tigr):
+    """tigr_graph_from_coo_part with host arrays of two copy chunks (the multi-GPU e2e path: the
+    filtered first pass, chunked copies overlapped with the arc-list scan): every rank's CSR
+    equals the oracle's CSR restricted to the rank's source range."""
+    n, m = 1 << 20, (1 << 24) + 777
+    rng = np.random.default_rng(23)
+    src = np.minimum((n * rng.random(m) ** 3).astype(np.uint32), n - 1)
+    dst = rng.integers(0, n, m, dtype=np.uint32)
+    w = rng.integers(1, 65, m, dtype=np.uint32)
+    o = oracle.csr_build(n, src, dst, w)
+    cuts = [0, n // 3, n]
+    for r in range(2):
+        lo, hi = cuts[r], cuts[r + 1]
+        g = tigr.tigr_graph_from_coo_part(n, src, dst, w, src_lo=lo, src_hi=hi)
+        rp, col, ww = tigr.tigr_graph_export_csr(g)
+        a, b = o.row_ptr[lo], o.row_ptr[hi]
+        want_rp = np.concatenate([np.zeros(lo, np.int64), o.row_ptr[lo:hi + 1] - a,
+                                  np.full(n - hi, b - a, np.int64)])
+        assert np.array_equal(rp, want_rp)
+        assert np.array_equal(col, o.col[a:b]) and np.array_equal(ww, o.wt[a:b])
+
+
 def test_vgraph_pr_profile(tigr):
     """tigr_vgraph_pr_profile: the push PageRank relax's arcs split into shared-memory hot slots
     and global float64 reductions.  cfg1 (n < hot slots): no global reduction at all; cfg2 (2^20
