@@ -53,8 +53,8 @@ PAPER_CONTEXT = {
 def ablation_context():
     """This build's Fig. 13 analogue beside the paper's: cfg3 (LiveJournal-shaped) SSSP speedups
     of the virtual transformations over the untransformed engine, K = 8, from the committed
-    ablation run (tools/ablation.py -> profiles/r02_ablation_cfg3.jsonl)."""
-    path = os.path.join(ROOT, "profiles", "r02_ablation_cfg3.jsonl")
+    ablation run (tools/ablation.py -> profiles/r02e_ablation_cfg3.jsonl)."""
+    path = os.path.join(ROOT, "profiles", "r02e_ablation_cfg3.jsonl")
     want = {"Tigr-V+ K=8 strided": "tigr_v_plus", "Tigr-V K=8 consecutive": "tigr_v", "Tigr-UDT K=8": "tigr_udt"}
     out = {}
     try:
@@ -64,7 +64,7 @@ def ablation_context():
                 out[want[d["variant"]]] = round(d["speedup_vs_baseline"], 2)
     except (OSError, ValueError):
         return None
-    out["source"] = "profiles/r02_ablation_cfg3.jsonl (tools/ablation.py, B200, same engine, cfg3 SSSP, K = 8)"
+    out["source"] = "profiles/r02e_ablation_cfg3.jsonl (tools/ablation.py, B200, same engine, cfg3 SSSP, K = 8)"
     return out
 
 
